@@ -1,0 +1,109 @@
+"""Exact quantities that pin the oracle — TEST INFRASTRUCTURE ONLY (pure Python).
+
+* brute_force_count: the estimand written out as its plain definition (reading A1):
+  the number of injective maps f: V_q -> V_G with L(f(u)) = L_q(u) and every query
+  edge mapped onto a data edge (non-induced).  itertools over all vertex tuples;
+  only for tiny graphs (n <= ~10).
+* tree_walk: expands EVERY branch of the sampler's own candidate-set construction
+  (SURVEY §8(c) R2-R5, P:L538 WanderJoin, P:L540 Alley) with exact rational
+  probabilities.  Unbiasedness of the HT estimator (Eq. 1) means
+  sum over complete leaves of P(leaf) * W(leaf) equals brute_force_count exactly;
+  sum P * W^2 gives E[Y^2] and hence the exact variance of one sample.  It also
+  returns |C_d| for every reachable prefix, so oracle records can be checked node by
+  node.
+Neither function shares code with oracle.c or with the CUDA path.
+"""
+from __future__ import annotations
+
+import itertools
+from fractions import Fraction
+from typing import Dict, Tuple
+
+
+def _adjacency_sets(g):
+    return [set(int(x) for x in g.col[g.row_ptr[v]:g.row_ptr[v + 1]]) for v in range(g.n)]
+
+
+def brute_force_count(g, q) -> int:
+    adj = _adjacency_sets(g)
+    lab = [int(x) for x in g.labels]
+    qlab = [int(x) for x in q.labels]
+    edges = q.edges()
+    count = 0
+    for f in itertools.permutations(range(g.n), q.nq):
+        if any(lab[f[u]] != qlab[u] for u in range(q.nq)):
+            continue
+        if all(f[b] in adj[f[a]] for a, b in edges):
+            count += 1
+    return count
+
+
+def tree_walk(g, q, method: int) -> Tuple[Fraction, Fraction, Dict[tuple, Tuple[int, ...]]]:
+    """Returns (E[Y], E[Y^2], cand) where cand[prefix] = the candidate list C_d the
+    sampler draws from after matching `prefix` (len(prefix) = d)."""
+    adj = _adjacency_sets(g)
+    lab = [int(x) for x in g.labels]
+    order = [int(x) for x in q.order]
+    qlab = [int(q.labels[u]) for u in range(q.nq)]
+    nq = q.nq
+    cand: Dict[tuple, Tuple[int, ...]] = {}
+
+    def local(v: int, l: int):
+        return sorted(w for w in adj[v] if lab[w] == l)
+
+    def candidates(prefix: tuple):
+        d = len(prefix)
+        u = order[d]
+        l = qlab[u]
+        if d == 0:
+            return [v for v in range(g.n) if lab[v] == l], None
+        back = [j for j in range(d) if q.adj[order[j], u]]
+        lists = [local(prefix[j], l) for j in back]
+        p = min(range(len(back)), key=lambda b: (len(lists[b]), b))
+        if method == 0:  # WanderJoin: the smallest local list, unfiltered
+            return lists[p], (back, lists, p)
+        inter = [x for x in lists[p] if all(x in set(lists[b]) for b in range(len(back)))
+                 and x not in prefix]
+        return inter, None
+
+    ey = Fraction(0)
+    ey2 = Fraction(0)
+    stack = [((), Fraction(1), 1)]
+    while stack:
+        prefix, prob, w = stack.pop()
+        d = len(prefix)
+        if d == nq:
+            ey += prob * w
+            ey2 += prob * w * w
+            continue
+        c, info = candidates(prefix)
+        cand[prefix] = tuple(c)
+        if not c:
+            continue
+        w2 = w * len(c)
+        p2 = prob / len(c)
+        for v in c:
+            if method == 0 and d > 0:
+                back, lists, p = info
+                if v in prefix:
+                    continue
+                if any(v not in set(lists[b]) for b in range(len(back)) if b != p):
+                    continue
+            stack.append((prefix + (v,), p2, w2))
+    return ey, ey2, cand
+
+
+def is_embedding_prefix(g, q, path) -> bool:
+    """True iff path[0..len-1] is an injective, label- and edge-preserving partial
+    match of phi[0..len-1] (Def. 3 partial instance)."""
+    adj = _adjacency_sets(g) if not hasattr(g, "_adjsets") else g._adjsets
+    order = [int(x) for x in q.order]
+    if len(set(path)) != len(path):
+        return False
+    for i, v in enumerate(path):
+        if int(g.labels[v]) != int(q.labels[order[i]]):
+            return False
+        for j in range(i):
+            if q.adj[order[j], order[i]] and path[j] not in adj[v]:
+                return False
+    return True

@@ -1,0 +1,329 @@
+/*
+ * oracle.c — plain, slow, obviously-correct CPU reference for the gSWORD hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load this library.  The product path
+ * (paper_journals_pacmmod_yelsg24_b200/) never links, imports or calls it, and it
+ * shares no code, header, table or constant generator with the CUDA path.
+ *
+ * What it computes (PAPER.md = P:L<line>; readings = DESIGN.md §3):
+ *   - Philox4x32-10 counter-based generator (reading A6; Salmon et al. SC'11),
+ *     one call per (seed, sample id, depth).
+ *   - WanderJoin samples (§2.2; Fig. 19 WJ P:L1756-L1774; Alg. 1):
+ *     seed from the global candidate set, each next vertex drawn uniformly from the
+ *     smallest local candidate list of the already-matched query neighbours
+ *     (GetMinCandidate, Alg. 1 l.8 P:L798), then Validate (DupCheck + IsEdge).
+ *   - Alley samples (Fig. 19 AL P:L1775-L1805): the candidate set is the
+ *     intersection of all local candidate lists of matched query neighbours, minus
+ *     already-matched vertices (reading A5); an empty set ends the sample.
+ *   - Horvitz-Thompson value per sample (Eq. 1): Y = prod |C_d| if the
+ *     sample is a complete instance, else 0.  Aggregation (sum / n) is done by the
+ *     Python wrapper with a correctly rounded sum (math.fsum).
+ *   - Exact embedding count by plain backtracking (estimand, reading A1).
+ *
+ * Every step is written in the paper's order with no blocking, fusion or
+ * reordering.  Membership tests use the C library bsearch on ascending lists.
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+#define OR_MAX_QV 16
+
+/* ---- per-sample record (layout is the contract of include/gsword.h, restated) ---- */
+typedef struct {
+    uint64_t sample_id;
+    uint8_t valid;
+    uint8_t depth_reached;
+    uint8_t pad[6];
+    int32_t path[OR_MAX_QV];
+    uint32_t csize[OR_MAX_QV];
+    double weight;
+} or_record; /* 152 bytes */
+
+/* ---- Philox4x32-10 (reading A6 / SURVEY R10) ---------------------------------- */
+void or_philox4x32_10(const uint32_t ctr_in[4], const uint32_t key_in[2], uint32_t out[4]) {
+    uint32_t c0 = ctr_in[0], c1 = ctr_in[1], c2 = ctr_in[2], c3 = ctr_in[3];
+    uint32_t k0 = key_in[0], k1 = key_in[1];
+    for (int round = 0; round < 10; ++round) {
+        uint64_t p0 = (uint64_t)0xD2511F53u * (uint64_t)c0;
+        uint64_t p1 = (uint64_t)0xCD9E8D57u * (uint64_t)c2;
+        uint32_t hi0 = (uint32_t)(p0 >> 32), lo0 = (uint32_t)p0;
+        uint32_t hi1 = (uint32_t)(p1 >> 32), lo1 = (uint32_t)p1;
+        uint32_t n0 = hi1 ^ c1 ^ k0;
+        uint32_t n1 = lo1;
+        uint32_t n2 = hi0 ^ c3 ^ k1;
+        uint32_t n3 = lo0;
+        c0 = n0; c1 = n1; c2 = n2; c3 = n3;
+        k0 += 0x9E3779B9u;
+        k1 += 0xBB67AE85u;
+    }
+    out[0] = c0; out[1] = c1; out[2] = c2; out[3] = c3;
+}
+
+/* r(sid, d): key = seed, counter = (sid, d, 0); r = x1:x0 */
+static uint64_t draw_r(uint64_t seed, uint64_t sid, uint32_t d) {
+    uint32_t ctr[4] = {(uint32_t)sid, (uint32_t)(sid >> 32), d, 0u};
+    uint32_t key[2] = {(uint32_t)seed, (uint32_t)(seed >> 32)};
+    uint32_t x[4];
+    or_philox4x32_10(ctr, key, x);
+    return ((uint64_t)x[1] << 32) | (uint64_t)x[0];
+}
+
+/* uniform index in [0, c): floor(r * c / 2^64) */
+static uint64_t uniform_index(uint64_t r, uint64_t c) {
+    return (uint64_t)(((unsigned __int128)r * (unsigned __int128)c) >> 64);
+}
+
+uint64_t or_uniform_index(uint64_t seed, uint64_t sid, uint32_t d, uint64_t c) {
+    return uniform_index(draw_r(seed, sid, d), c);
+}
+
+/* ---- graph / query --------------------------------------------------------------- */
+typedef struct {
+    int64_t n;
+    const int64_t* row_ptr;
+    const int32_t* col;
+    const int32_t* labels; /* never NULL here: the wrapper passes zeros when unlabelled */
+} or_graph;
+
+typedef struct {
+    int32_t nq;
+    int32_t adj[OR_MAX_QV][OR_MAX_QV]; /* query-vertex adjacency */
+    int32_t label[OR_MAX_QV];          /* L_q(u) */
+    int32_t order[OR_MAX_QV];          /* phi */
+} or_query;
+
+static int cmp_i32(const void* a, const void* b) {
+    int32_t x = *(const int32_t*)a, y = *(const int32_t*)b;
+    return (x > y) - (x < y);
+}
+
+static int contains(const int32_t* list, int64_t len, int32_t x) {
+    if (len <= 0) return 0;
+    return bsearch(&x, list, (size_t)len, sizeof(int32_t), cmp_i32) != NULL;
+}
+
+/* Local candidate set C(u', u, v) with the label-only filter: N(v) ∩ {w : L(w) = l},
+ * ascending id (Def. 4; reading A2/A4).  Returns its size. */
+static int64_t local_candidates(const or_graph* G, int32_t v, int32_t l, int32_t* out) {
+    int64_t len = 0;
+    for (int64_t i = G->row_ptr[v]; i < G->row_ptr[v + 1]; ++i) {
+        int32_t w = G->col[i];
+        if (G->labels[w] == l) out[len++] = w;
+    }
+    return len;
+}
+
+/* ---- one sample (Alg. 1 inner loop) --------------------------------- */
+/* method: 0 = WanderJoin, 1 = Alley.  Returns Y (0 if not a complete instance). */
+static double one_sample(const or_graph* G, const or_query* Q, int method, uint64_t seed, uint64_t sid,
+                         const int32_t* C0, int64_t C0_len, int32_t** S, int32_t* refine,
+                         or_record* rec) {
+    int32_t M[OR_MAX_QV];
+    int nq = Q->nq;
+    double W = 0.0;
+    int valid = 0, depth_reached = 0;
+    if (rec) {
+        memset(rec, 0, sizeof(*rec));
+        rec->sample_id = sid;
+        for (int i = 0; i < OR_MAX_QV; ++i) rec->path[i] = -1;
+    }
+    /* d = 0: seed from the global candidate set C(phi[0]).  W is the running
+     * product prod |C_d| (Eq. 1), taken in depth order (reading A7). */
+    W = (double)C0_len;
+    if (C0_len == 0) goto done;
+    {
+        uint64_t k = uniform_index(draw_r(seed, sid, 0), (uint64_t)C0_len);
+        M[0] = C0[k];
+        if (rec) { rec->path[0] = M[0]; rec->csize[0] = (uint32_t)C0_len; }
+    }
+    for (int d = 1; d < nq; ++d) {
+        depth_reached = d;
+        int32_t u = Q->order[d];
+        int32_t l = Q->label[u];
+        /* backward positions B(d) = { j < d : (phi[j], phi[d]) in E_q } */
+        int B[OR_MAX_QV], nb = 0;
+        for (int j = 0; j < d; ++j)
+            if (Q->adj[Q->order[j]][u]) B[nb++] = j;
+        /* GetMinCandidate (Alg. 1 l.8): local lists S_j of every matched neighbour,
+         * p = the smallest one, ties -> smallest position j (reading A3) */
+        int64_t len[OR_MAX_QV];
+        int p = 0;
+        for (int b = 0; b < nb; ++b) {
+            len[b] = local_candidates(G, M[B[b]], l, S[b]);
+            if (len[b] < len[p]) p = b;
+        }
+        int64_t clen;
+        const int32_t* cand = S[p];
+        if (method == 0) {
+            /* WanderJoin Refine: refine = cand (Fig. 19 WJ) */
+            clen = len[p];
+            W = W * (double)clen;
+            if (clen == 0) goto done;
+            /* Sample: uniform vertex of refine, prob 1/rlen */
+            uint64_t k = uniform_index(draw_r(seed, sid, (uint32_t)d), (uint64_t)clen);
+            int32_t v = cand[k];
+            M[d] = v;
+            if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
+            /* Validate: DupCheck against all matched vertices, IsEdge for every other
+             * matched query neighbour */
+            for (int j = 0; j < d; ++j)
+                if (M[j] == v) goto done;
+            for (int b = 0; b < nb; ++b) {
+                if (b == p) continue;
+                if (!contains(S[b], len[b], v)) goto done;
+            }
+        } else {
+            /* Alley Refine: keep each x of cand that lies in every other local list and
+             * is not already matched (Fig. 19 AL; reading A5) */
+            clen = 0;
+            for (int64_t i = 0; i < len[p]; ++i) {
+                int32_t x = cand[i];
+                int keep = 1;
+                for (int b = 0; b < nb && keep; ++b) {
+                    if (b == p) continue;
+                    if (!contains(S[b], len[b], x)) keep = 0;
+                }
+                for (int j = 0; j < d && keep; ++j)
+                    if (M[j] == x) keep = 0;
+                if (keep) refine[clen++] = x;
+            }
+            W = W * (double)clen;
+            /* empty refined set: the sample stops */
+            if (clen == 0) goto done;
+            uint64_t k = uniform_index(draw_r(seed, sid, (uint32_t)d), (uint64_t)clen);
+            int32_t v = refine[k];
+            M[d] = v;
+            if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
+        }
+    }
+    /* all |V_q| vertices matched: a complete instance */
+    valid = 1;
+    depth_reached = nq - 1;
+done:
+    if (rec) {
+        rec->valid = (uint8_t)valid;
+        rec->depth_reached = (uint8_t)depth_reached;
+        rec->weight = W;
+    }
+    return valid ? W : 0.0;
+}
+
+static int load_query(or_query* Q, int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col,
+                      const int32_t* q_labels, const int32_t* order) {
+    if (nq < 1 || nq > OR_MAX_QV) return -1;
+    memset(Q, 0, sizeof(*Q));
+    Q->nq = nq;
+    for (int u = 0; u < nq; ++u) {
+        Q->label[u] = q_labels[u];
+        Q->order[u] = order[u];
+        for (int32_t i = q_row_ptr[u]; i < q_row_ptr[u + 1]; ++i) Q->adj[u][q_col[i]] = 1;
+    }
+    /* every prefix of the matching order must be connected (reading A13) */
+    for (int d = 1; d < nq; ++d) {
+        int has = 0;
+        for (int j = 0; j < d; ++j) has |= Q->adj[Q->order[j]][Q->order[d]];
+        if (!has) return -2;
+    }
+    return 0;
+}
+
+/*
+ * Run samples [first, first + count).  y_out[i] = Y of sample first+i (may be NULL);
+ * rec_out[i] = its record (may be NULL).  Returns 0, or -1 on bad input / OOM.
+ */
+int or_sample_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                    int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                    const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
+                    double* y_out, or_record* rec_out) {
+    or_graph G = {n, row_ptr, col, labels};
+    or_query Q;
+    int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
+    if (rc) return rc;
+    int64_t maxdeg = 0;
+    for (int64_t v = 0; v < n; ++v)
+        if (row_ptr[v + 1] - row_ptr[v] > maxdeg) maxdeg = row_ptr[v + 1] - row_ptr[v];
+    /* global candidate set of phi[0]: all vertices with its label, ascending (reading A2) */
+    int32_t* C0 = (int32_t*)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+    int32_t* buf = (int32_t*)malloc(sizeof(int32_t) * (size_t)(maxdeg + 1) * (OR_MAX_QV + 1));
+    if (!C0 || !buf) { free(C0); free(buf); return -1; }
+    int64_t C0_len = 0;
+    int32_t l0 = Q.label[Q.order[0]];
+    for (int64_t v = 0; v < n; ++v)
+        if (labels[v] == l0) C0[C0_len++] = (int32_t)v;
+    int32_t* S[OR_MAX_QV];
+    for (int b = 0; b < OR_MAX_QV; ++b) S[b] = buf + (size_t)b * (size_t)(maxdeg + 1);
+    int32_t* refine = buf + (size_t)OR_MAX_QV * (size_t)(maxdeg + 1);
+    for (uint64_t i = 0; i < count; ++i) {
+        double y = one_sample(&G, &Q, method, seed, first + i, C0, C0_len, S, refine,
+                              rec_out ? &rec_out[i] : NULL);
+        if (y_out) y_out[i] = y;
+    }
+    free(C0);
+    free(buf);
+    return 0;
+}
+
+/* ---- exact count of embeddings by plain backtracking (reading A1) --------------- */
+typedef struct {
+    const or_graph* G;
+    const or_query* Q;
+    int32_t M[OR_MAX_QV];
+    unsigned __int128 count;
+    int overflow;
+} enum_state;
+
+static int is_edge(const or_graph* G, int32_t a, int32_t b) {
+    return contains(G->col + G->row_ptr[a], G->row_ptr[a + 1] - G->row_ptr[a], b);
+}
+
+static void extend(enum_state* st, int d) {
+    const or_query* Q = st->Q;
+    const or_graph* G = st->G;
+    if (d == Q->nq) {
+        st->count += 1;
+        return;
+    }
+    int32_t u = Q->order[d];
+    /* candidates: any vertex with the right label for d = 0; otherwise the neighbours
+     * of the first matched query neighbour (every embedding is reached exactly once) */
+    int jfirst = -1;
+    for (int j = 0; j < d && jfirst < 0; ++j)
+        if (Q->adj[Q->order[j]][u]) jfirst = j;
+    int64_t lo, hi;
+    if (d == 0) { lo = 0; hi = G->n; }
+    else { lo = G->row_ptr[st->M[jfirst]]; hi = G->row_ptr[st->M[jfirst] + 1]; }
+    for (int64_t i = lo; i < hi; ++i) {
+        int32_t v = (d == 0) ? (int32_t)i : G->col[i];
+        if (G->labels[v] != Q->label[u]) continue;
+        int ok = 1;
+        for (int j = 0; j < d && ok; ++j) {
+            if (st->M[j] == v) ok = 0;
+            else if (Q->adj[Q->order[j]][u] && !is_edge(G, st->M[j], v)) ok = 0;
+        }
+        if (!ok) continue;
+        st->M[d] = v;
+        extend(st, d + 1);
+    }
+}
+
+/* count_out = low 64 bits, count_hi = high 64 bits of the 128-bit count. */
+int or_count_embeddings(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                        int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                        const int32_t* order, uint64_t* count_lo, uint64_t* count_hi) {
+    or_graph G = {n, row_ptr, col, labels};
+    or_query Q;
+    int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
+    if (rc) return rc;
+    enum_state st;
+    memset(&st, 0, sizeof(st));
+    st.G = &G;
+    st.Q = &Q;
+    extend(&st, 0);
+    *count_lo = (uint64_t)st.count;
+    *count_hi = (uint64_t)(st.count >> 64);
+    return 0;
+}
+
+int or_record_size(void) { return (int)sizeof(or_record); }

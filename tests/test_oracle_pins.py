@@ -1,0 +1,257 @@
+"""Pins of the CPU oracle against values fixed by the paper and by mathematics.
+
+Every test here checks `oracle/` against something other than itself:
+golden vectors (tests/golden), closed forms, brute force, and the exact
+enumeration-tree walk (oracle/exact.py).  DESIGN.md §4 maps each pin to the
+oracle function it covers.
+"""
+import math
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle import exact
+from gsword_testutil import read_golden
+from workloads import gen
+
+
+# ---------------------------------------------------------------- Philox (reading A6)
+def test_philox_known_answers():
+    rows = read_golden("philox4x32_10_kat.txt")
+    assert len(rows) == 3
+    for r in rows:
+        v = [int(x, 16) for x in r]
+        ctr, key, want = v[0:4], v[4:6], tuple(v[6:10])
+        assert oracle.philox4x32_10(ctr, key) == want
+
+
+def test_uniform_index_wiring():
+    # seed=0, sid=0, d=0 -> counter (0,0,0,0), key (0,0): the first KAT vector,
+    # r = x1:x0 = 0xe169c58d_6627e8d5; index = floor(r * c / 2^64).
+    r = 0xE169C58D6627E8D5
+    for c in (1, 2, 3, 7, 1000, 862_664, 2**32 - 1, 2**40 + 3):
+        assert oracle.uniform_index(0, 0, 0, c) == (r * c) >> 64
+    # the counter layout: sid occupies ctr0/ctr1, depth ctr2
+    x = oracle.philox4x32_10([0x89ABCDEF, 0x01234567, 5, 0], [0x9, 0x0])
+    r2 = (x[1] << 32) | x[0]
+    assert oracle.uniform_index(9, 0x0123456789ABCDEF, 5, 12345) == (r2 * 12345) >> 64
+
+
+# ---------------------------------------------------------------- HT estimator, Eq. 1
+def test_ht_example2():
+    g = {r[0]: [float(x) for x in r[1:]] for r in read_golden("ht_example2.txt")}
+    assert math.prod(g["csizes_s2"]) == g["weight_s2"][0]
+    agg = oracle.aggregate(np.array(g["samples"]))
+    assert agg["estimate"] == g["estimate"][0]
+    assert agg["n"] == 2 and agg["n_valid"] == 1
+    # dead samples count in n (reading A8)
+    assert oracle.aggregate(np.array([0.0, 0.0, 24.0, 24.0]))["estimate"] == 12.0
+    assert math.prod(g["csizes_wj_s1"]) == 12 and math.prod(g["csizes_al_s1"]) == 6
+
+
+def test_aggregate_variance_closed_form():
+    y = np.array([0.0, 24.0, 6.0, 6.0, 0.0])
+    agg = oracle.aggregate(y)
+    mean = Fraction(36, 5)
+    s2 = sum((Fraction(v) - mean) ** 2 for v in [0, 24, 6, 6, 0]) / 4  # sample variance
+    assert agg["variance"] == pytest.approx(float(s2 / 5), rel=1e-15)
+
+
+def test_qerror_golden():
+    for c, ch, want in read_golden("qerror_cases.txt"):
+        assert oracle.qerror(float(c), float(ch)) == pytest.approx(float(want), rel=1e-15)
+
+
+# ---------------------------------------------------------------- exact counts (reading A1)
+def _falling(x, k):
+    out = 1
+    for i in range(k):
+        out *= x - i
+    return out
+
+
+def test_brute_force_closed_forms():
+    # K_n: any connected k-vertex q has n!/(n-k)! embeddings
+    k5 = gen.complete_graph(5)
+    assert exact.brute_force_count(k5, gen.clique_query(3)) == 60
+    assert exact.brute_force_count(k5, gen.path_query(4)) == 120
+    # ring C_n: P_k has 2n, C_k has 2n iff k = n
+    r7 = gen.ring_graph(7)
+    assert exact.brute_force_count(r7, gen.path_query(4)) == 14
+    assert exact.brute_force_count(r7, gen.cycle_query(4)) == 0
+    assert exact.brute_force_count(gen.ring_graph(6), gen.cycle_query(6)) == 12
+    # 3x3 grid: C_4 = 8 (a-1)(b-1)
+    assert exact.brute_force_count(gen.grid_graph(3, 3), gen.cycle_query(4)) == 32
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_c_enumerator_equals_brute_force(seed):
+    g = gen.random_small_graph(8, 0.45, n_labels=1 + seed % 3, seed=seed)
+    for qs in range(3):
+        q = gen.random_connected_query(2 + (seed + qs) % 4, 0.4, g.n_labels, seed * 10 + qs)
+        assert oracle.count_embeddings(g, q) == exact.brute_force_count(g, q)
+
+
+def test_c_enumerator_closed_forms_large():
+    assert oracle.count_embeddings(gen.complete_graph(9), gen.clique_query(4)) == 9 * 8 * 7 * 6
+    assert oracle.count_embeddings(gen.ring_graph(50), gen.path_query(6)) == 100
+    assert oracle.count_embeddings(gen.ring_graph(9), gen.cycle_query(9)) == 18
+    a, b = 10, 12
+    grid = gen.grid_graph(a, b)
+    assert oracle.count_embeddings(grid, gen.cycle_query(4)) == 8 * (a - 1) * (b - 1)
+    assert oracle.count_embeddings(grid, gen.path_query(2)) == 2 * (a * (b - 1) + b * (a - 1))
+    deg = grid.degree()
+    assert oracle.count_embeddings(grid, gen.star_query(3)) == int(sum(_falling(int(d), 3) for d in deg))
+
+
+def test_c_enumerator_on_c0_graph_closed_forms(c0):
+    g, _ = c0
+    deg = np.diff(g.row_ptr)
+    unl = gen.Graph(g.row_ptr, g.col, np.zeros(g.n, np.int32), 1)
+    assert oracle.count_embeddings(unl, gen.path_query(3)) == int(sum(int(d) * (int(d) - 1) for d in deg))
+    # triangles: 6 * #triangles, #triangles by sorted-list intersection
+    nb = [set(g.neighbors(v).tolist()) for v in range(g.n)]
+    tri = sum(len(nb[u] & nb[v]) for u in range(g.n) for v in nb[u] if v > u) // 3
+    assert oracle.count_embeddings(unl, gen.clique_query(3)) == 6 * tri
+    # labelled star: centre label a, leaves {b, c}: sum over centres of n_b * n_c (b != c)
+    q = gen.star_query(2, labels=[0, 1, 2])
+    want = 0
+    for v in range(g.n):
+        if g.labels[v] != 0:
+            continue
+        ls = g.labels[g.neighbors(v)]
+        want += int(np.sum(ls == 1)) * int(np.sum(ls == 2))
+    assert oracle.count_embeddings(g, q) == want
+
+
+# ---------------------------------------------------------------- tree walk (unbiasedness)
+@pytest.mark.parametrize("seed", range(10))
+@pytest.mark.parametrize("method", [oracle.WJ, oracle.ALLEY])
+def test_tree_walk_equals_brute_force(seed, method):
+    g = gen.random_small_graph(7, 0.5, n_labels=1 + seed % 2, seed=100 + seed)
+    q = gen.random_connected_query(2 + seed % 3, 0.5, g.n_labels, 200 + seed)
+    ey, ey2, _ = exact.tree_walk(g, q, method)
+    assert ey == exact.brute_force_count(g, q)
+    assert ey2 >= ey * ey
+
+
+# ---------------------------------------------------------------- oracle records vs tree
+def _check_records_against_tree(g, q, method, rec):
+    _, _, cand = exact.tree_walk(g, q, method)
+    for r in rec:
+        dr = int(r["depth_reached"])
+        w = 1.0
+        for d in range(dr + 1):
+            prefix = tuple(int(x) for x in r["path"][:d])
+            c = cand[prefix]
+            assert int(r["csize"][d]) == len(c)
+            w *= len(c)
+            if len(c):
+                assert int(r["path"][d]) in c
+            else:
+                assert int(r["path"][d]) == -1
+        assert all(int(x) == -1 for x in r["path"][dr + 1:])
+        assert all(int(x) == 0 for x in r["csize"][dr + 1:])
+        assert r["weight"] == w
+        full = tuple(int(x) for x in r["path"][:q.nq])
+        assert bool(r["valid"]) == (dr == q.nq - 1 and -1 not in full and exact.is_embedding_prefix(g, q, full))
+        if method == oracle.ALLEY:
+            # every drawn Alley prefix is a valid partial instance
+            drawn = [int(x) for x in r["path"][:dr + 1] if int(x) >= 0]
+            assert exact.is_embedding_prefix(g, q, drawn)
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("method", [oracle.WJ, oracle.ALLEY])
+def test_records_follow_the_tree(seed, method):
+    g = gen.random_small_graph(8, 0.5, n_labels=1 + seed % 2, seed=300 + seed)
+    q = gen.random_connected_query(3 + seed % 3, 0.4, g.n_labels, 400 + seed)
+    _, rec = oracle.sample_range(g, q, method, seed=seed, first=0, count=500)
+    _check_records_against_tree(g, q, method, rec)
+
+
+# ---------------------------------------------------------------- closed forms per sample
+def test_alley_zero_variance_clique():
+    for n, k in ((6, 3), (7, 4), (9, 5)):
+        y, rec = oracle.sample_range(gen.complete_graph(n), gen.clique_query(k), oracle.ALLEY, 3, 0, 300)
+        assert np.all(rec["valid"] == 1)
+        assert np.all(y == math.factorial(n) // math.factorial(n - k))
+
+
+def test_alley_zero_variance_ring_path():
+    for n, k in ((7, 4), (6, 6), (30, 9)):
+        y, rec = oracle.sample_range(gen.ring_graph(n), gen.path_query(k), oracle.ALLEY, 5, 17, 300)
+        assert np.all(y == 2 * n)
+
+
+def test_alley_zero_variance_regular_star():
+    g = gen.regular_circulant(40, 3)  # 6-regular
+    for s in (2, 3, 5):
+        y, _ = oracle.sample_range(g, gen.star_query(s), oracle.ALLEY, 9, 0, 200)
+        assert np.all(y == 40 * _falling(6, s))
+
+
+def test_wanderjoin_ring_path_closed_form():
+    n, k = 11, 5
+    q = gen.path_query(k)
+    y, rec = oracle.sample_range(gen.ring_graph(n), q, oracle.WJ, 1, 0, 4000)
+    for r in rec:
+        dr = int(r["depth_reached"])
+        assert list(r["csize"][:dr + 1]) == [n] + [2] * dr
+    w = n * 2 ** (k - 1)
+    assert set(np.unique(y).tolist()) <= {0.0, float(w)}
+    # valid w.p. 2^-(k-2): each step after the first must not step back
+    frac = float(np.mean(rec["valid"]))
+    assert abs(frac - 2.0 ** -(k - 2)) < 5 * math.sqrt(0.125 * 0.875 / 4000)
+
+
+# ---------------------------------------------------------------- statistics vs exact
+@pytest.mark.parametrize("method", [oracle.WJ, oracle.ALLEY])
+def test_sampler_z_scores_tiny(method):
+    g = gen.random_small_graph(9, 0.5, n_labels=2, seed=77)
+    q = gen.extract_query(g, 4, seed=78, dense=True)
+    ey, ey2, _ = exact.tree_walk(g, q, method)
+    truth = exact.brute_force_count(g, q)
+    assert ey == truth and truth > 0
+    var1 = float(ey2 - ey * ey)
+    n = 3000
+    zs = []
+    for seed in range(30):
+        y, _ = oracle.sample_range(g, q, method, seed, 0, n, records=False)
+        est = oracle.aggregate(y)["estimate"]
+        zs.append((est - truth) / math.sqrt(var1 / n) if var1 > 0 else 0.0)
+        if var1 == 0:
+            assert est == truth
+    zs = np.array(zs)
+    assert np.all(np.abs(zs) < 5)
+    assert abs(zs.mean()) < 5 / math.sqrt(30)
+
+
+@pytest.mark.parametrize("method", [oracle.WJ, oracle.ALLEY])
+def test_sampler_c0_within_4_sigma(c0, method):
+    g, qs = c0
+    for q in qs[:6]:
+        truth = oracle.count_embeddings(g, q)
+        agg = oracle.estimate(g, q, method, seed=1, n_samples=100_000, threads=4)
+        sigma = math.sqrt(agg["variance"]) if agg["variance"] > 0 else 0.0
+        assert abs(agg["estimate"] - truth) <= 4 * sigma + 1e-9, (q.name, truth, agg)
+
+
+def test_split_range_identity(c0):
+    g, qs = c0
+    q = qs[0]
+    y_all, r_all = oracle.sample_range(g, q, oracle.WJ, 11, 1000, 3000)
+    y_a, r_a = oracle.sample_range(g, q, oracle.WJ, 11, 1000, 1234)
+    y_b, r_b = oracle.sample_range(g, q, oracle.WJ, 11, 2234, 1766)
+    assert np.array_equal(y_all, np.concatenate([y_a, y_b]))
+    assert r_all.tobytes() == np.concatenate([r_a, r_b]).tobytes()
+    y_t, _ = oracle.sample_range(g, q, oracle.WJ, 11, 1000, 3000, records=False, threads=4)
+    assert np.array_equal(y_all, y_t)
+
+
+def test_bad_order_rejected():
+    q = gen.query_from_edges(3, [(0, 1), (1, 2)], order=[0, 2, 1])
+    with pytest.raises(ValueError):
+        oracle.sample_range(gen.complete_graph(4), q, oracle.WJ, 0, 0, 10)
