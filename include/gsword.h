@@ -1,0 +1,211 @@
+/*
+ * gsword.h — C ABI of the B200-native gSWORD hot path: the WanderJoin / Alley
+ * random-walk estimator of the number of embeddings of a labelled query graph q in a
+ * labelled data graph G, with Horvitz-Thompson aggregation.
+ *
+ * Citations: P:L<n> = line n of PAPER.md (the gSWORD paper, PACMMOD 2024);
+ * readings A<n> = DESIGN.md §3 (where the paper is silent or garbled).
+ *
+ * Conventions for every entry point
+ *   - Return value: GSWORD_OK (0) on success, a negative gsword_status on error; the
+ *     thread-local message of the last error is available from gsword_last_error().
+ *   - Host pointers are borrowed for the duration of the call only and are never
+ *     written unless documented as outputs.  The context owns every device buffer it
+ *     allocates; nothing is freed by the caller.
+ *   - A context is bound to one CUDA device and is not thread-safe.  All device work
+ *     is issued on the context's stream (gsword_set_stream), in stream order.
+ *   - Results are a pure function of (graph, query, matching order, method, seed,
+ *     first sample id, sample count); the scheduling of samples onto the GPU does not
+ *     change any per-sample result, and aggregates agree to a relative 1e-12.
+ */
+#ifndef GSWORD_H
+#define GSWORD_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GSWORD_MAX_QV 16 /* largest query (P:L1055 uses 4/8/16 vertices; reading A12) */
+
+typedef struct gsword_ctx gsword_ctx; /* opaque */
+
+/* Random-walk estimators (P:L538 WanderJoin, P:L540 Alley). */
+typedef enum { GSWORD_WJ = 0, GSWORD_ALLEY = 1 } gsword_method;
+
+typedef enum {
+    GSWORD_OK = 0,
+    GSWORD_EINVAL = -1,   /* bad argument (NULL pointer, unknown method, label out of range) */
+    GSWORD_ENOGRAPH = -2, /* no graph loaded */
+    GSWORD_ENOQUERY = -3, /* no query loaded (or the graph was reloaded since) */
+    GSWORD_EORDER = -4,   /* order is not a permutation, or an order prefix is disconnected (A13) */
+    GSWORD_EGRAPH = -5,   /* CSR not canonical: unsorted/duplicate/self loop/asymmetric (A10, A11) */
+    GSWORD_ELIMIT = -6,   /* nq > GSWORD_MAX_QV, or |V|, 2|E|, n_labels beyond 32-bit indexing */
+    GSWORD_ECUDA = -7,    /* CUDA runtime error (including: no device) */
+    GSWORD_ENOMEM = -8    /* device or host allocation failed */
+} gsword_status;
+
+/* Aggregate of a sample range (Eq. 1; readings A8, A9).
+ *   estimate = sum / n_samples               (HT estimator, dead samples count in n)
+ *   variance = (sumsq - sum^2/n) / (n (n-1))  (variance of the estimate; NaN if n < 2)
+ *   sum      = sum_i Y_i,  Y_i = prod_d |C_id| if sample i is a complete instance else 0
+ *   sumsq    = sum_i Y_i^2 (Y_i^2 rounded to fp64 per sample)
+ *   seconds  = device time of the sampling kernels (CUDA events), 0 if not measured */
+typedef struct {
+    double estimate;
+    double variance;
+    double sum;
+    double sumsq;
+    uint64_t n_samples;
+    uint64_t n_valid;
+    double seconds;
+} gsword_result;
+
+/* One traced sample (152 bytes, little endian, no implicit padding).
+ *   path[d]  data vertex drawn at depth d (matching-order position), -1 if none
+ *   csize[d] |C_d|, the size of the candidate set drawn from at depth d (0 if unused)
+ *   depth_reached: last depth at which a candidate set was formed (nq-1 if complete)
+ *   valid    1 iff the sample is a complete instance of q
+ *   weight   running fp64 product prod_{d <= depth_reached} csize[d] in depth order (A7);
+ *            Y = weight if valid else 0.
+ * A WanderJoin vertex drawn and then rejected by Validate is recorded (valid = 0);
+ * an empty candidate set at depth d gives path[d] = -1, csize[d] = 0, weight 0. */
+typedef struct {
+    uint64_t sample_id;
+    uint8_t valid;
+    uint8_t depth_reached;
+    uint8_t pad[6];
+    int32_t path[GSWORD_MAX_QV];
+    uint32_t csize[GSWORD_MAX_QV];
+    double weight;
+} gsword_sample_record;
+
+/* Host-side view of a compiled query plan (for inspection / tests).
+ *   back_mask[d]  bit j set iff j < d and (phi[j], phi[d]) is a query edge: B(d)
+ *   dup_mask[d]   bit j set iff j < d and L_q(phi[j]) == L_q(phi[d]) (injectivity
+ *                 checks needed at depth d; SURVEY R5')
+ *   label[d]      L_q(phi[d]) */
+typedef struct {
+    int32_t nq;
+    int32_t label[GSWORD_MAX_QV];
+    uint32_t back_mask[GSWORD_MAX_QV];
+    uint32_t dup_mask[GSWORD_MAX_QV];
+} gsword_plan_info;
+
+/* Tunables for gsword_set_option (defaults chosen by measurement). */
+typedef enum {
+    GSWORD_OPT_BLOCKS_PER_SM = 0,  /* persistent CTAs per SM; 0 = occupancy maximum  */
+    GSWORD_OPT_THREADS = 1,        /* threads per CTA (multiple of 32, 64..256)       */
+    GSWORD_OPT_CHUNK = 2,          /* sample ids a warp takes from the queue at once  */
+    GSWORD_OPT_L2_PERSIST = 3,     /* 1 = L2 access-policy window over the adjacency  */
+    GSWORD_OPT_COOP_THRESHOLD = 4  /* Alley driver length at which a warp cooperates  */
+} gsword_option;
+
+/* ---- context -------------------------------------------------------------------- */
+
+/* Create a context on CUDA device `cuda_device`.  *out receives the handle.
+ * Errors: EINVAL (out NULL), ECUDA (no such device / no driver), ENOMEM. */
+int gsword_create(int cuda_device, gsword_ctx** out);
+
+/* Destroy a context and free every device buffer it owns.  NULL is a no-op. */
+int gsword_destroy(gsword_ctx* ctx);
+
+/* Issue all later device work on `cuda_stream` (a cudaStream_t, e.g.
+ * torch.cuda.Stream.cuda_stream; NULL = the context's own non-blocking stream; the
+ * legacy default stream is cudaStreamLegacy, (void*)0x1).  Borrowed, not destroyed. */
+int gsword_set_stream(gsword_ctx* ctx, void* cuda_stream);
+
+/* Set a tunable (gsword_option).  Errors: EINVAL for an unknown option or value. */
+int gsword_set_option(gsword_ctx* ctx, int option, int64_t value);
+
+/* ---- graph and query -------------------------------------------------------------- */
+
+/* Load the data graph G (P:L404 notation).  Host arrays, copied; the context owns the
+ * device copy.  Canonical CSR required (reading A10/A11):
+ *   row_ptr  int64[n_vertices+1], row_ptr[0] = 0, non-decreasing
+ *   col      int32[row_ptr[n]], each row strictly ascending, no self loop, and the
+ *            adjacency symmetric (u in N(v) iff v in N(u))
+ *   labels   int32[n_vertices] in [0, n_labels), or NULL = unlabelled (n_labels must be 1)
+ * The library re-lays adjacency out sorted by (label, id) so that every label-filtered
+ * local candidate set N_l(v) (Def. 4) is one contiguous ascending run.
+ * Loading a graph invalidates the loaded query.
+ * Errors: EINVAL, EGRAPH, ELIMIT (n_vertices or 2|E| >= 2^31, n_vertices*n_labels >= 2^31),
+ * ENOMEM, ECUDA. */
+int gsword_load_graph(gsword_ctx* ctx, int64_t n_vertices, const int64_t* row_ptr, const int32_t* col,
+                      const int32_t* labels, int32_t n_labels);
+
+/* Load the query q and its matching order phi (Def. 2).  Host arrays, copied:
+ *   q_row_ptr int32[n_qv+1], q_col: symmetric query adjacency over vertices 0..n_qv-1
+ *   q_labels  int32[n_qv] in [0, n_labels of the loaded graph)
+ *   order     int32[n_qv], a permutation of 0..n_qv-1 with every prefix connected
+ * Errors: ENOGRAPH, EINVAL, EORDER, ELIMIT (n_qv > GSWORD_MAX_QV). */
+int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, const int32_t* q_col,
+                      const int32_t* q_labels, const int32_t* order);
+
+/* ---- estimation ----------------------------------------------------------------------- */
+
+/* Draw samples 0 .. n_samples-1 with `method` and `seed`, return the HT aggregate
+ * (Eq. 1).  Synchronous (waits for the context stream).  Same as
+ * gsword_estimate_range(ctx, m, 0, n_samples, seed, out).
+ * Errors: ENOGRAPH, ENOQUERY, EINVAL (n_samples == 0, out NULL, bad method), ECUDA. */
+int gsword_estimate(gsword_ctx* ctx, gsword_method m, uint64_t n_samples, uint64_t seed, gsword_result* out);
+
+/* Same for the sample-id range [first_sample_id, first_sample_id + n_samples): the
+ * multi-GPU split and checkpoint/resume unit (sample ids are global). */
+int gsword_estimate_range(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples,
+                          uint64_t seed, gsword_result* out);
+
+/* Asynchronous form: enqueue the sampling + reduction kernels on the context stream
+ * and write 4 fp64 values {sum, sumsq, n_valid, n_samples} to DEVICE memory d_out4
+ * (caller-owned, 32 bytes, 8-byte aligned).  Returns without waiting; the values are
+ * valid in stream order.  Used by the multi-GPU layer (all_reduce on the same stream)
+ * and by device-side timing.  Counts are exact as fp64 below 2^53. */
+int gsword_estimate_async(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples,
+                          uint64_t seed, double* d_out4);
+
+/* Host-only: turn 4 aggregated values {sum, sumsq, n_valid, n_samples} into a result. */
+int gsword_finalize(const double* host4, gsword_result* out);
+
+/* Parity entry: run samples [first, first+n) through the same kernel code with a
+ * per-sample record writer; host_out receives n records in sample-id order.
+ * Synchronous.  Errors as gsword_estimate_range, ENOMEM. */
+int gsword_trace_samples(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples,
+                         uint64_t seed, gsword_sample_record* host_out);
+
+/* Measurement entry: run [first, first+n) in the counting build of
+ * the kernel and return the ALGORITHMIC 32-byte sectors the method must touch,
+ * summed over the range (model in DESIGN.md §6).  Synchronous. */
+int gsword_count_sectors(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples,
+                         uint64_t seed, double* sectors_out);
+
+/* Device time (CUDA events on the context stream) of the last sampling-kernel launch
+ * alone (without the queue reset and the grid reduction).  Waits for that launch. */
+int gsword_last_kernel_seconds(gsword_ctx* ctx, double* seconds);
+
+/* Launch geometry used by the last estimate: grid CTAs, threads per CTA, kernel
+ * launches per estimate.  Any pointer may be NULL. */
+int gsword_launch_info(gsword_ctx* ctx, int* grid, int* threads, int* launches_per_estimate);
+
+/* ---- host-only helpers (no device needed) ------------------------------------------- */
+
+/* Check that a CSR is canonical (same rules as gsword_load_graph). */
+int gsword_check_graph(int64_t n_vertices, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                       int32_t n_labels);
+
+/* Compile a query + order into its plan (the same plan gsword_load_query stages into
+ * shared memory); n_labels bounds the labels. */
+int gsword_plan_query(int32_t n_qv, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                      const int32_t* order, int32_t n_labels, gsword_plan_info* out);
+
+/* Thread-local message for the last failing call on this thread ("" if none). */
+const char* gsword_last_error(void);
+
+/* ABI version (major*100 + minor). */
+int gsword_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* GSWORD_H */

@@ -1,0 +1,586 @@
+// gsword_host.cpp — host side of the C ABI declared in include/gsword.h.
+//
+// Owns the context (device buffers, stream, events), validates and re-lays out the
+// data graph (canonical CSR -> adjacency sorted by (label, id) + per-(vertex, label)
+// segment offsets + label buckets), compiles the query + matching order into the
+// per-depth plan that the kernels stage in shared memory (Def. 2
+// GetMinCandidate inputs), and launches the sampling + reduction kernels.
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <limits>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "internal.h"
+
+using gsword::DeviceGraph;
+using gsword::LaunchCfg;
+using gsword::Partial;
+using gsword::Plan;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+int fail(int status, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    g_last_error = buf;
+    return status;
+}
+
+int cuda_fail(cudaError_t e, const char* what) {
+    return fail(GSWORD_ECUDA, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+#define CUDA_TRY(expr)                                  \
+    do {                                                \
+        cudaError_t _e = (expr);                        \
+        if (_e != cudaSuccess) return cuda_fail(_e, #expr); \
+    } while (0)
+
+unsigned host_threads() {
+    unsigned t = std::thread::hardware_concurrency();
+    return t == 0 ? 1 : std::min(t, 32u);
+}
+
+// Run f(lo, hi) over [0, n) split into contiguous ranges on host threads.
+template <class F>
+void parallel_for(int64_t n, F f) {
+    const unsigned T = (n < (1 << 16)) ? 1u : host_threads();
+    if (T == 1) {
+        f((int64_t)0, n);
+        return;
+    }
+    std::vector<std::thread> ts;
+    for (unsigned t = 0; t < T; ++t) {
+        const int64_t lo = n * t / T, hi = n * (t + 1) / T;
+        ts.emplace_back([=] { f(lo, hi); });
+    }
+    for (auto& th : ts) th.join();
+}
+
+int check_graph_impl(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                     int32_t n_labels) {
+    if (n < 0 || !row_ptr) return fail(GSWORD_EINVAL, "load_graph: n_vertices < 0 or row_ptr NULL");
+    if (n_labels < 1) return fail(GSWORD_EINVAL, "load_graph: n_labels must be >= 1");
+    if (!labels && n_labels != 1) return fail(GSWORD_EINVAL, "load_graph: labels NULL requires n_labels == 1");
+    if (n >= (int64_t)1 << 31) return fail(GSWORD_ELIMIT, "load_graph: |V| >= 2^31");
+    if (n * (int64_t)n_labels >= ((int64_t)1 << 31)) return fail(GSWORD_ELIMIT, "load_graph: |V| * n_labels >= 2^31");
+    if (row_ptr[0] != 0) return fail(GSWORD_EGRAPH, "load_graph: row_ptr[0] != 0");
+    for (int64_t v = 0; v < n; ++v)
+        if (row_ptr[v + 1] < row_ptr[v]) return fail(GSWORD_EGRAPH, "load_graph: row_ptr decreasing at %lld", (long long)v);
+    const int64_t nnz = row_ptr[n];
+    if (nnz >= ((int64_t)1 << 31) - 1) return fail(GSWORD_ELIMIT, "load_graph: 2|E| >= 2^31");
+    if (nnz > 0 && !col) return fail(GSWORD_EINVAL, "load_graph: col NULL");
+    if (labels) {
+        for (int64_t v = 0; v < n; ++v)
+            if (labels[v] < 0 || labels[v] >= n_labels)
+                return fail(GSWORD_EINVAL, "load_graph: label of vertex %lld out of range", (long long)v);
+    }
+    std::atomic<int64_t> bad_row{-1};
+    std::atomic<int> bad_kind{0};
+    parallel_for(n, [&](int64_t lo, int64_t hi) {
+        for (int64_t v = lo; v < hi && bad_row.load(std::memory_order_relaxed) < 0; ++v) {
+            for (int64_t i = row_ptr[v]; i < row_ptr[v + 1]; ++i) {
+                const int32_t w = col[i];
+                int kind = 0;
+                if (w < 0 || w >= n) kind = 1;
+                else if (w == v) kind = 2;
+                else if (i > row_ptr[v] && col[i - 1] >= w) kind = 3;
+                else {
+                    const int32_t* b = col + row_ptr[w];
+                    const int32_t* e = col + row_ptr[w + 1];
+                    if (!std::binary_search(b, e, (int32_t)v)) kind = 4;
+                }
+                if (kind) {
+                    int64_t expect = -1;
+                    if (bad_row.compare_exchange_strong(expect, v)) bad_kind = kind;
+                    return;
+                }
+            }
+        }
+    });
+    if (bad_row >= 0) {
+        static const char* what[] = {"", "neighbour id out of range", "self loop", "row not strictly ascending",
+                                     "asymmetric adjacency"};
+        return fail(GSWORD_EGRAPH, "load_graph: %s at vertex %lld", what[bad_kind.load()], (long long)bad_row.load());
+    }
+    return GSWORD_OK;
+}
+
+int plan_query_impl(int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                    const int32_t* order, int32_t n_labels, Plan* plan, gsword_plan_info* info) {
+    if (nq < 1) return fail(GSWORD_EINVAL, "load_query: n_qv < 1");
+    if (nq > GSWORD_MAX_QV) return fail(GSWORD_ELIMIT, "load_query: n_qv > %d", GSWORD_MAX_QV);
+    if (!q_row_ptr || !q_labels || !order) return fail(GSWORD_EINVAL, "load_query: NULL argument");
+    if (q_row_ptr[0] != 0 || (q_row_ptr[nq] > 0 && !q_col)) return fail(GSWORD_EINVAL, "load_query: bad query CSR");
+    bool adj[GSWORD_MAX_QV][GSWORD_MAX_QV] = {};
+    for (int u = 0; u < nq; ++u) {
+        if (q_row_ptr[u + 1] < q_row_ptr[u]) return fail(GSWORD_EINVAL, "load_query: bad query CSR");
+        if (q_labels[u] < 0 || q_labels[u] >= n_labels)
+            return fail(GSWORD_EINVAL, "load_query: label of query vertex %d out of range", u);
+        for (int32_t i = q_row_ptr[u]; i < q_row_ptr[u + 1]; ++i) {
+            const int32_t w = q_col[i];
+            if (w < 0 || w >= nq || w == u) return fail(GSWORD_EINVAL, "load_query: bad query edge (%d,%d)", u, w);
+            adj[u][w] = true;
+        }
+    }
+    for (int u = 0; u < nq; ++u)
+        for (int w = 0; w < nq; ++w)
+            if (adj[u][w] != adj[w][u]) return fail(GSWORD_EINVAL, "load_query: query adjacency not symmetric");
+    bool seen[GSWORD_MAX_QV] = {};
+    for (int d = 0; d < nq; ++d) {
+        if (order[d] < 0 || order[d] >= nq || seen[order[d]])
+            return fail(GSWORD_EORDER, "load_query: order is not a permutation");
+        seen[order[d]] = true;
+    }
+    Plan p;
+    std::memset(&p, 0, sizeof(p));
+    p.nq = nq;
+    for (int d = 0; d < nq; ++d) {
+        const int u = order[d];
+        gsword::PlanStep& s = p.step[d];
+        s.label = q_labels[u];
+        for (int j = 0; j < d; ++j) {
+            if (adj[order[j]][u]) s.back |= 1u << j;
+            if (q_labels[order[j]] == q_labels[u]) s.dup |= 1u << j;
+        }
+        s.nback = __builtin_popcount(s.back);
+        if (d > 0 && s.back == 0)
+            return fail(GSWORD_EORDER, "load_query: order prefix %d is not connected (reading A13)", d);
+    }
+    if (plan) *plan = p;
+    if (info) {
+        std::memset(info, 0, sizeof(*info));
+        info->nq = nq;
+        for (int d = 0; d < nq; ++d) {
+            info->label[d] = p.step[d].label;
+            info->back_mask[d] = p.step[d].back;
+            info->dup_mask[d] = p.step[d].dup;
+        }
+    }
+    return GSWORD_OK;
+}
+
+}  // namespace
+
+struct gsword_ctx {
+    int device = 0;
+    int num_sms = 148;
+    cudaStream_t own_stream = nullptr;
+    cudaStream_t stream = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;    // around a whole estimate
+    cudaEvent_t evk0 = nullptr, evk1 = nullptr;  // around the last sampling-kernel launch
+    // graph
+    bool graph_loaded = false;
+    int32_t* d_col = nullptr;
+    uint32_t* d_seg = nullptr;
+    int32_t* d_bucket = nullptr;
+    int64_t n = 0, nnz = 0;
+    int32_t n_labels = 1;
+    std::vector<int64_t> label_off;
+    // query
+    bool query_loaded = false;
+    Plan plan{};
+    // scratch
+    unsigned long long* d_queue = nullptr;
+    Partial* d_partials = nullptr;
+    int partial_cap = 0;
+    double* d_out4 = nullptr;
+    double* d_sectors = nullptr;
+    // options
+    int opt_blocks_per_sm = 0;
+    int opt_threads = 256;
+    int opt_chunk = 256;
+    int opt_l2 = 0;
+    int opt_coop = 32;
+    // last launch
+    int last_grid = 0, last_threads = 0;
+
+    void free_graph() {
+        if (d_col) cudaFree(d_col);
+        if (d_seg) cudaFree(d_seg);
+        if (d_bucket) cudaFree(d_bucket);
+        d_col = nullptr;
+        d_seg = nullptr;
+        d_bucket = nullptr;
+        graph_loaded = false;
+        query_loaded = false;
+    }
+};
+
+namespace {
+
+int ensure_ready(gsword_ctx* ctx, int method) {
+    if (!ctx) return fail(GSWORD_EINVAL, "NULL context");
+    if (method != GSWORD_WJ && method != GSWORD_ALLEY) return fail(GSWORD_EINVAL, "unknown method %d", method);
+    if (!ctx->graph_loaded) return fail(GSWORD_ENOGRAPH, "no graph loaded");
+    if (!ctx->query_loaded) return fail(GSWORD_ENOQUERY, "no query loaded");
+    cudaError_t e = cudaSetDevice(ctx->device);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
+    return GSWORD_OK;
+}
+
+int apply_l2_window(gsword_ctx* ctx) {
+    if (!ctx->graph_loaded) return GSWORD_OK;
+    cudaStreamAttrValue attr;
+    std::memset(&attr, 0, sizeof(attr));
+    if (ctx->opt_l2) {
+        int max_persist = 0, max_window = 0;
+        CUDA_TRY(cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, ctx->device));
+        CUDA_TRY(cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, ctx->device));
+        const size_t bytes = (size_t)ctx->nnz * sizeof(int32_t);
+        const size_t window = std::min(bytes, (size_t)max_window);
+        const size_t persist = std::min((size_t)max_persist, window);
+        CUDA_TRY(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, persist));
+        attr.accessPolicyWindow.base_ptr = ctx->d_col;
+        attr.accessPolicyWindow.num_bytes = window;
+        attr.accessPolicyWindow.hitRatio = window ? (float)std::min(1.0, (double)persist / (double)window) : 0.f;
+        attr.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        attr.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    } else {
+        attr.accessPolicyWindow.num_bytes = 0;
+        attr.accessPolicyWindow.hitRatio = 0.f;
+        attr.accessPolicyWindow.hitProp = cudaAccessPropertyNormal;
+        attr.accessPolicyWindow.missProp = cudaAccessPropertyNormal;
+    }
+    CUDA_TRY(cudaStreamSetAttribute(ctx->stream, cudaStreamAttributeAccessPolicyWindow, &attr));
+    return GSWORD_OK;
+}
+
+int launch_config(gsword_ctx* ctx, int method, int mode, LaunchCfg* cfg) {
+    size_t smem = 0;
+    const int occ = gsword::max_blocks_per_sm(method, mode, ctx->opt_threads, &smem);
+    if (occ <= 0) return fail(GSWORD_ECUDA, "kernel does not fit on the device (threads=%d)", ctx->opt_threads);
+    const int bps = ctx->opt_blocks_per_sm > 0 ? std::min(ctx->opt_blocks_per_sm, occ) : occ;
+    cfg->grid = ctx->num_sms * bps;
+    cfg->threads = ctx->opt_threads;
+    cfg->chunk = ctx->opt_chunk;
+    cfg->coop_threshold = ctx->opt_coop;
+    if (cfg->grid > ctx->partial_cap) {
+        if (ctx->d_partials) cudaFree(ctx->d_partials);
+        ctx->d_partials = nullptr;
+        CUDA_TRY(cudaMalloc(&ctx->d_partials, sizeof(Partial) * (size_t)cfg->grid));
+        ctx->partial_cap = cfg->grid;
+    }
+    ctx->last_grid = cfg->grid;
+    ctx->last_threads = cfg->threads;
+    return GSWORD_OK;
+}
+
+DeviceGraph device_graph(const gsword_ctx* ctx) {
+    DeviceGraph g;
+    g.col = ctx->d_col;
+    g.seg = ctx->d_seg;
+    g.bucket = ctx->d_bucket;
+    g.n = ctx->n;
+    g.nnz = ctx->nnz;
+    g.n_labels = ctx->n_labels;
+    return g;
+}
+
+int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, uint64_t seed, double* d_out4,
+        gsword_sample_record* d_records, double* d_sectors) {
+    LaunchCfg cfg;
+    int rc = launch_config(ctx, method, mode, &cfg);
+    if (rc) return rc;
+    CUDA_TRY(cudaEventRecord(ctx->evk0, ctx->stream));
+    cudaError_t e = gsword::launch_sample(method, mode, device_graph(ctx), ctx->plan, cfg, first, count, seed,
+                                          ctx->d_queue, ctx->d_partials, d_records, ctx->stream);
+    if (e != cudaSuccess) return cuda_fail(e, "launch sample kernel");
+    CUDA_TRY(cudaEventRecord(ctx->evk1, ctx->stream));
+    e = gsword::launch_reduce(ctx->d_partials, cfg.grid, d_out4, d_sectors, ctx->stream);
+    if (e != cudaSuccess) return cuda_fail(e, "launch reduce kernel");
+    return GSWORD_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int gsword_version(void) { return 100; }
+
+const char* gsword_last_error(void) { return g_last_error.c_str(); }
+
+int gsword_create(int cuda_device, gsword_ctx** out) {
+    if (!out) return fail(GSWORD_EINVAL, "create: out NULL");
+    *out = nullptr;
+    int count = 0;
+    cudaError_t e = cudaGetDeviceCount(&count);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceCount");
+    if (cuda_device < 0 || cuda_device >= count) return fail(GSWORD_ECUDA, "create: no CUDA device %d", cuda_device);
+    CUDA_TRY(cudaSetDevice(cuda_device));
+    gsword_ctx* ctx = new (std::nothrow) gsword_ctx();
+    if (!ctx) return fail(GSWORD_ENOMEM, "create: host allocation failed");
+    ctx->device = cuda_device;
+    cudaDeviceProp prop;
+    e = cudaGetDeviceProperties(&prop, cuda_device);
+    if (e == cudaSuccess) ctx->num_sms = prop.multiProcessorCount;
+    if ((e = cudaStreamCreateWithFlags(&ctx->own_stream, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaEventCreate(&ctx->ev0)) != cudaSuccess || (e = cudaEventCreate(&ctx->ev1)) != cudaSuccess ||
+        (e = cudaEventCreate(&ctx->evk0)) != cudaSuccess || (e = cudaEventCreate(&ctx->evk1)) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_queue, sizeof(unsigned long long))) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_out4, 4 * sizeof(double))) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_sectors, sizeof(double))) != cudaSuccess) {
+        gsword_destroy(ctx);
+        return cuda_fail(e, "create");
+    }
+    ctx->stream = ctx->own_stream;
+    *out = ctx;
+    return GSWORD_OK;
+}
+
+int gsword_destroy(gsword_ctx* ctx) {
+    if (!ctx) return GSWORD_OK;
+    cudaSetDevice(ctx->device);
+    if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+    ctx->free_graph();
+    if (ctx->d_queue) cudaFree(ctx->d_queue);
+    if (ctx->d_partials) cudaFree(ctx->d_partials);
+    if (ctx->d_out4) cudaFree(ctx->d_out4);
+    if (ctx->d_sectors) cudaFree(ctx->d_sectors);
+    if (ctx->ev0) cudaEventDestroy(ctx->ev0);
+    if (ctx->ev1) cudaEventDestroy(ctx->ev1);
+    if (ctx->evk0) cudaEventDestroy(ctx->evk0);
+    if (ctx->evk1) cudaEventDestroy(ctx->evk1);
+    if (ctx->own_stream) cudaStreamDestroy(ctx->own_stream);
+    delete ctx;
+    return GSWORD_OK;
+}
+
+int gsword_set_stream(gsword_ctx* ctx, void* cuda_stream) {
+    if (!ctx) return fail(GSWORD_EINVAL, "set_stream: NULL context");
+    ctx->stream = cuda_stream ? (cudaStream_t)cuda_stream : ctx->own_stream;
+    return apply_l2_window(ctx);
+}
+
+int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
+    if (!ctx) return fail(GSWORD_EINVAL, "set_option: NULL context");
+    switch (option) {
+        case GSWORD_OPT_BLOCKS_PER_SM:
+            if (value < 0 || value > 32) return fail(GSWORD_EINVAL, "blocks_per_sm out of range");
+            ctx->opt_blocks_per_sm = (int)value;
+            return GSWORD_OK;
+        case GSWORD_OPT_THREADS:
+            if (value < 64 || value > 256 || value % 32) return fail(GSWORD_EINVAL, "threads must be 64..256, /32");
+            ctx->opt_threads = (int)value;
+            return GSWORD_OK;
+        case GSWORD_OPT_CHUNK:
+            if (value < 1 || value > (1 << 20)) return fail(GSWORD_EINVAL, "chunk out of range");
+            ctx->opt_chunk = (int)value;
+            return GSWORD_OK;
+        case GSWORD_OPT_L2_PERSIST:
+            ctx->opt_l2 = value ? 1 : 0;
+            return apply_l2_window(ctx);
+        case GSWORD_OPT_COOP_THRESHOLD:
+            if (value < 0 || value > 64) return fail(GSWORD_EINVAL, "coop threshold must be 0..64");
+            ctx->opt_coop = (int)value;
+            return GSWORD_OK;
+        default:
+            return fail(GSWORD_EINVAL, "unknown option %d", option);
+    }
+}
+
+int gsword_check_graph(int64_t n_vertices, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                       int32_t n_labels) {
+    return check_graph_impl(n_vertices, row_ptr, col, labels, n_labels);
+}
+
+int gsword_plan_query(int32_t n_qv, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                      const int32_t* order, int32_t n_labels, gsword_plan_info* out) {
+    return plan_query_impl(n_qv, q_row_ptr, q_col, q_labels, order, n_labels, nullptr, out);
+}
+
+int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                      int32_t n_labels) {
+    if (!ctx) return fail(GSWORD_EINVAL, "load_graph: NULL context");
+    int rc = check_graph_impl(n, row_ptr, col, labels, n_labels);
+    if (rc) return rc;
+    CUDA_TRY(cudaSetDevice(ctx->device));
+    CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    ctx->free_graph();
+    const int64_t nnz = row_ptr[n];
+    const int32_t L = n_labels;
+    // label buckets: vertices sorted by (label, id)
+    std::vector<int64_t> off((size_t)L + 1, 0);
+    for (int64_t v = 0; v < n; ++v) off[(size_t)(labels ? labels[v] : 0) + 1] += 1;
+    for (int32_t l = 0; l < L; ++l) off[(size_t)l + 1] += off[(size_t)l];
+    // adjacency sorted by (label, id) and segment offsets seg[v*L + l]
+    std::vector<int32_t> col2;
+    std::vector<uint32_t> seg((size_t)n * (size_t)L + 1);
+    const int32_t* col_up = col;
+    if (L == 1) {
+        for (int64_t v = 0; v <= n; ++v) seg[(size_t)v] = (uint32_t)row_ptr[v];
+    } else {
+        col2.resize((size_t)nnz);
+        parallel_for(n, [&](int64_t lo, int64_t hi) {
+            std::vector<uint32_t> cnt((size_t)L + 1);
+            for (int64_t v = lo; v < hi; ++v) {
+                std::fill(cnt.begin(), cnt.end(), 0u);
+                for (int64_t i = row_ptr[v]; i < row_ptr[v + 1]; ++i) cnt[(size_t)labels[col[i]] + 1] += 1;
+                for (int32_t l = 0; l < L; ++l) cnt[(size_t)l + 1] += cnt[(size_t)l];
+                for (int32_t l = 0; l < L; ++l) seg[(size_t)v * L + l] = (uint32_t)(row_ptr[v] + cnt[(size_t)l]);
+                for (int64_t i = row_ptr[v]; i < row_ptr[v + 1]; ++i) {  // stable: ascending id per label
+                    const int32_t w = col[i];
+                    col2[(size_t)(row_ptr[v] + cnt[(size_t)labels[w]]++)] = w;
+                }
+            }
+        });
+        seg[(size_t)n * L] = (uint32_t)nnz;
+        col_up = col2.data();
+    }
+    std::vector<int32_t> bucket;
+    if (L > 1) {
+        bucket.resize((size_t)n);
+        std::vector<int64_t> pos(off.begin(), off.end() - 1);
+        for (int64_t v = 0; v < n; ++v) bucket[(size_t)pos[(size_t)labels[v]]++] = (int32_t)v;
+    }
+    cudaError_t e;
+    if ((e = cudaMalloc(&ctx->d_col, sizeof(int32_t) * (size_t)std::max<int64_t>(nnz, 1))) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_seg, sizeof(uint32_t) * seg.size())) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_bucket, sizeof(int32_t) * (size_t)std::max<int64_t>(n, 1))) != cudaSuccess) {
+        ctx->free_graph();
+        return fail(e == cudaErrorMemoryAllocation ? GSWORD_ENOMEM : GSWORD_ECUDA, "load_graph: cudaMalloc: %s",
+                    cudaGetErrorString(e));
+    }
+    if (nnz > 0) CUDA_TRY(cudaMemcpy(ctx->d_col, col_up, sizeof(int32_t) * (size_t)nnz, cudaMemcpyHostToDevice));
+    CUDA_TRY(cudaMemcpy(ctx->d_seg, seg.data(), sizeof(uint32_t) * seg.size(), cudaMemcpyHostToDevice));
+    if (L > 1) {
+        if (n > 0) CUDA_TRY(cudaMemcpy(ctx->d_bucket, bucket.data(), sizeof(int32_t) * (size_t)n, cudaMemcpyHostToDevice));
+    } else if (n > 0) {
+        CUDA_TRY(gsword::launch_build_bucket_identity(ctx->d_bucket, n, ctx->stream));
+        CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    }
+    ctx->n = n;
+    ctx->nnz = nnz;
+    ctx->n_labels = L;
+    ctx->label_off = off;
+    ctx->graph_loaded = true;
+    ctx->query_loaded = false;
+    return apply_l2_window(ctx);
+}
+
+int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, const int32_t* q_col,
+                      const int32_t* q_labels, const int32_t* order) {
+    if (!ctx) return fail(GSWORD_EINVAL, "load_query: NULL context");
+    if (!ctx->graph_loaded) return fail(GSWORD_ENOGRAPH, "load_query: no graph loaded");
+    Plan p;
+    int rc = plan_query_impl(n_qv, q_row_ptr, q_col, q_labels, order, ctx->n_labels, &p, nullptr);
+    if (rc) return rc;
+    const int32_t l0 = p.step[0].label;
+    p.seed_lo = (uint32_t)ctx->label_off[(size_t)l0];
+    p.seed_len = (uint32_t)(ctx->label_off[(size_t)l0 + 1] - ctx->label_off[(size_t)l0]);
+    p.seed_identity = (ctx->n_labels == 1) ? 1 : 0;
+    ctx->plan = p;
+    ctx->query_loaded = true;
+    return GSWORD_OK;
+}
+
+int gsword_estimate_async(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_t n_samples, uint64_t seed,
+                          double* d_out4) {
+    int rc = ensure_ready(ctx, (int)m);
+    if (rc) return rc;
+    if (!d_out4) return fail(GSWORD_EINVAL, "estimate_async: d_out4 NULL");
+    if (n_samples == 0) return fail(GSWORD_EINVAL, "estimate: n_samples must be >= 1");
+    if (first + n_samples < first) return fail(GSWORD_EINVAL, "estimate: sample-id range overflows u64");
+    return run(ctx, (int)m, gsword::kModeEstimate, first, n_samples, seed, d_out4, nullptr, nullptr);
+}
+
+int gsword_finalize(const double* h, gsword_result* out) {
+    if (!h || !out) return fail(GSWORD_EINVAL, "finalize: NULL argument");
+    const double sum = h[0], sq = h[1], valid = h[2], n = h[3];
+    out->sum = sum;
+    out->sumsq = sq;
+    out->n_valid = (uint64_t)valid;
+    out->n_samples = (uint64_t)n;
+    out->estimate = n > 0 ? sum / n : std::numeric_limits<double>::quiet_NaN();
+    out->variance = n >= 2 ? (sq - sum * sum / n) / (n * (n - 1.0)) : std::numeric_limits<double>::quiet_NaN();
+    out->seconds = 0.0;
+    return GSWORD_OK;
+}
+
+int gsword_estimate_range(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_t n_samples, uint64_t seed,
+                          gsword_result* out) {
+    if (!out) return fail(GSWORD_EINVAL, "estimate: out NULL");
+    int rc = ensure_ready(ctx, (int)m);
+    if (rc) return rc;
+    CUDA_TRY(cudaEventRecord(ctx->ev0, ctx->stream));
+    rc = gsword_estimate_async(ctx, m, first, n_samples, seed, ctx->d_out4);
+    if (rc) return rc;
+    CUDA_TRY(cudaEventRecord(ctx->ev1, ctx->stream));
+    double h[4];
+    CUDA_TRY(cudaMemcpyAsync(h, ctx->d_out4, sizeof(h), cudaMemcpyDeviceToHost, ctx->stream));
+    CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    float ms = 0.f;
+    CUDA_TRY(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
+    gsword_finalize(h, out);
+    out->seconds = ms * 1e-3;
+    return GSWORD_OK;
+}
+
+int gsword_estimate(gsword_ctx* ctx, gsword_method m, uint64_t n_samples, uint64_t seed, gsword_result* out) {
+    return gsword_estimate_range(ctx, m, 0, n_samples, seed, out);
+}
+
+int gsword_trace_samples(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_t n_samples, uint64_t seed,
+                         gsword_sample_record* host_out) {
+    int rc = ensure_ready(ctx, (int)m);
+    if (rc) return rc;
+    if (!host_out) return fail(GSWORD_EINVAL, "trace: host_out NULL");
+    if (n_samples == 0) return GSWORD_OK;
+    gsword_sample_record* d_rec = nullptr;
+    const size_t bytes = sizeof(gsword_sample_record) * (size_t)n_samples;
+    cudaError_t e = cudaMalloc(&d_rec, bytes);
+    if (e != cudaSuccess) return fail(GSWORD_ENOMEM, "trace: cudaMalloc(%zu): %s", bytes, cudaGetErrorString(e));
+    CUDA_TRY(cudaMemsetAsync(d_rec, 0, bytes, ctx->stream));
+    rc = run(ctx, (int)m, gsword::kModeTrace, first, n_samples, seed, ctx->d_out4, d_rec, nullptr);
+    if (rc == GSWORD_OK) {
+        e = cudaMemcpyAsync(host_out, d_rec, bytes, cudaMemcpyDeviceToHost, ctx->stream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+        if (e != cudaSuccess) rc = cuda_fail(e, "trace: copy back");
+    }
+    cudaFree(d_rec);
+    return rc;
+}
+
+int gsword_count_sectors(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_t n_samples, uint64_t seed,
+                         double* sectors_out) {
+    int rc = ensure_ready(ctx, (int)m);
+    if (rc) return rc;
+    if (!sectors_out) return fail(GSWORD_EINVAL, "count_sectors: NULL output");
+    if (n_samples == 0) return fail(GSWORD_EINVAL, "count_sectors: n_samples must be >= 1");
+    rc = run(ctx, (int)m, gsword::kModeCount, first, n_samples, seed, ctx->d_out4, nullptr, ctx->d_sectors);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(sectors_out, ctx->d_sectors, sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+    CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    return GSWORD_OK;
+}
+
+int gsword_last_kernel_seconds(gsword_ctx* ctx, double* seconds) {
+    if (!ctx || !seconds) return fail(GSWORD_EINVAL, "last_kernel_seconds: NULL argument");
+    CUDA_TRY(cudaSetDevice(ctx->device));
+    CUDA_TRY(cudaEventSynchronize(ctx->evk1));
+    float ms = 0.f;
+    CUDA_TRY(cudaEventElapsedTime(&ms, ctx->evk0, ctx->evk1));
+    *seconds = (double)ms * 1e-3;
+    return GSWORD_OK;
+}
+
+int gsword_launch_info(gsword_ctx* ctx, int* grid, int* threads, int* launches) {
+    if (!ctx) return fail(GSWORD_EINVAL, "launch_info: NULL context");
+    if (grid) *grid = ctx->last_grid;
+    if (threads) *threads = ctx->last_threads;
+    if (launches) *launches = 2;  // sampling kernel + grid reduction
+    return GSWORD_OK;
+}
+
+}  // extern "C"

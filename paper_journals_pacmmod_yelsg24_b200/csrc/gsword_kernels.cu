@@ -1,0 +1,604 @@
+// gsword_kernels.cu — sm_100a kernels of the gSWORD hot path.
+//
+// One persistent kernel per method (WanderJoin P:L538 / Alley P:L540) runs the
+// Refine-Sample-Validate loop of Alg. 1 for many samples per lane:
+//
+//   * lanes are refilled from a global u64 sample queue as soon as their sample ends
+//     (ballot -> one atomicAdd per warp chunk -> popc rank), so a warp never idles on
+//     dead samples (the "validate imbalance" of P:L379, solved without inheritance);
+//   * every random choice is k = mulhi64(Philox4x32-10(seed; sid, d), |C_d|), so each
+//     sample's path is a pure function of (seed, sample id) (reading A6);
+//   * Alley intersections with a long driver list are done by the whole warp over
+//     coalesced 32-element chunks with ballot/popc/find-nth (the deterministic
+//     replacement of warp streaming), short ones per lane in a 64-bit
+//     register bitmask (the "refine array" of Fig. 19);
+//   * the HT value Y = prod |C_d| (Eq. 1) is accumulated per lane in
+//     compensated fp64, reduced warp -> CTA -> grid in a fixed order.
+//
+// The graph is read through the read-only path; candidate order is ascending vertex
+// id everywhere, so results are bit-identical to the CPU oracle.
+#include <cstdint>
+
+#include "internal.h"
+
+namespace gsword {
+namespace {
+
+constexpr unsigned kFull = 0xffffffffu;
+// Alley drivers longer than the coop threshold (<= 64) are refined by the whole warp.
+
+// ---------------------------------------------------------------- Philox4x32-10 (A6)
+__device__ __forceinline__ uint64_t philox_r(uint64_t seed, uint64_t sid, uint32_t d) {
+    uint32_t c0 = (uint32_t)sid, c1 = (uint32_t)(sid >> 32), c2 = d, c3 = 0u;
+    uint32_t k0 = (uint32_t)seed, k1 = (uint32_t)(seed >> 32);
+#pragma unroll
+    for (int i = 0; i < 10; ++i) {
+        const uint32_t hi0 = __umulhi(0xD2511F53u, c0), lo0 = 0xD2511F53u * c0;
+        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c2), lo1 = 0xCD9E8D57u * c2;
+        const uint32_t n0 = hi1 ^ c1 ^ k0;
+        const uint32_t n2 = hi0 ^ c3 ^ k1;
+        c0 = n0;
+        c1 = lo1;
+        c2 = n2;
+        c3 = lo0;
+        k0 += 0x9E3779B9u;
+        k1 += 0xBB67AE85u;
+    }
+    return ((uint64_t)c1 << 32) | (uint64_t)c0;
+}
+
+__device__ __forceinline__ int32_t ldg_i32(const int32_t* p) { return __ldg(p); }
+__device__ __forceinline__ uint32_t ldg_u32(const uint32_t* p) { return __ldg(p); }
+
+// first index i in [lo, hi) with col[i] >= x (hi if none); *found = (col[i] == x)
+__device__ __forceinline__ uint32_t lower_bound(const int32_t* __restrict__ col, uint32_t lo, uint32_t hi,
+                                                int32_t x, bool* found) {
+    uint32_t n = hi - lo;
+    while (n > 0) {
+        const uint32_t half = n >> 1;
+        const int32_t y = ldg_i32(col + lo + half);
+        if (y < x) {
+            lo += half + 1;
+            n -= half + 1;
+        } else {
+            n = half;
+        }
+    }
+    *found = (lo < hi) && (ldg_i32(col + lo) == x);
+    return lo;
+}
+
+__device__ __forceinline__ bool contains(const int32_t* __restrict__ col, uint32_t lo, uint32_t hi, int32_t x) {
+    bool f;
+    lower_bound(col, lo, hi, x, &f);
+    return f;
+}
+
+// position of the k-th (0-based) set bit of m (k < popc(m))
+__device__ __forceinline__ uint32_t fns32(uint32_t m, uint32_t k) {
+    uint32_t pos = 0, c;
+    c = __popc(m & 0xFFFFu); if (k >= c) { k -= c; m >>= 16; pos += 16; }
+    c = __popc(m & 0xFFu);   if (k >= c) { k -= c; m >>= 8;  pos += 8; }
+    c = __popc(m & 0xFu);    if (k >= c) { k -= c; m >>= 4;  pos += 4; }
+    c = __popc(m & 0x3u);    if (k >= c) { k -= c; m >>= 2;  pos += 2; }
+    c = m & 1u;              if (k >= c) { pos += 1; }
+    return pos;
+}
+
+__device__ __forceinline__ uint32_t fns64(uint64_t m, uint32_t k) {
+    const uint32_t lo = (uint32_t)m;
+    const uint32_t c = __popc(lo);
+    return k < c ? fns32(lo, k) : 32u + fns32((uint32_t)(m >> 32), k - c);
+}
+
+// algorithmic sectors of a binary search over a sorted run of `len` 4-byte ids
+__device__ __forceinline__ uint32_t bs_sectors(uint32_t len) {
+    if (len == 0) return 0;
+    const uint32_t c = (len + 7) / 8;
+    return 1 + (c > 1 ? 32 - __clz(c - 1) : 0);
+}
+
+__device__ __forceinline__ uint32_t scan_sectors(uint32_t len) { return (4 * len + 31) / 32; }
+
+// Neumaier-compensated accumulation
+__device__ __forceinline__ void nsum(double& s, double& c, double x) {
+    const double t = __dadd_rn(s, x);
+    if (fabs(s) >= fabs(x)) c = __dadd_rn(c, __dadd_rn(__dsub_rn(s, t), x));
+    else c = __dadd_rn(c, __dadd_rn(__dsub_rn(x, t), s));
+    s = t;
+}
+
+// double-double addition (a_hi, a_lo) += (b_hi, b_lo)
+__device__ __forceinline__ void dd_add(double& ah, double& al, double bh, double bl) {
+    const double s = __dadd_rn(ah, bh);
+    const double v = __dsub_rn(s, ah);
+    double e = __dadd_rn(__dsub_rn(ah, __dsub_rn(s, v)), __dsub_rn(bh, v));
+    e = __dadd_rn(e, __dadd_rn(al, bl));
+    ah = __dadd_rn(s, e);
+    al = __dsub_rn(e, __dsub_rn(ah, s));
+}
+
+__device__ __forceinline__ double shfl_xor_d(double x, int m) { return __shfl_xor_sync(kFull, x, m); }
+
+// segment of N_l(v): [seg[v*nL + l], seg[v*nL + l + 1])
+__device__ __forceinline__ void segment(const DeviceGraph& g, uint32_t v, int32_t l, uint32_t* a, uint32_t* b) {
+    const size_t i = (size_t)v * (size_t)g.n_labels + (size_t)l;
+    *a = ldg_u32(g.seg + i);
+    *b = ldg_u32(g.seg + i + 1);
+}
+
+// Is x in every N_l(M[j]) for j in `mask`?  M column `col_of` in shared memory.
+__device__ __forceinline__ bool member_all(const DeviceGraph& g, const uint32_t* Ms, int stride, int col_of,
+                                           uint32_t mask, int32_t l, int32_t x) {
+    while (mask) {
+        const int j = __ffs(mask) - 1;
+        mask &= mask - 1;
+        uint32_t a, b;
+        segment(g, Ms[j * stride + col_of], l, &a, &b);
+        if (!contains(g.col, a, b, x)) return false;
+    }
+    return true;
+}
+
+__device__ __forceinline__ bool not_matched(const uint32_t* Ms, int stride, int col_of, uint32_t dup, int32_t x) {
+    while (dup) {
+        const int j = __ffs(dup) - 1;
+        dup &= dup - 1;
+        if ((int32_t)Ms[j * stride + col_of] == x) return false;
+    }
+    return true;
+}
+
+template <int METHOD, int MODE>
+__global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
+                                                     const uint64_t count, const uint64_t seed, const int chunk,
+                                                     const uint32_t coop_threshold,
+                                                     unsigned long long* __restrict__ queue,
+                                                     Partial* __restrict__ partials,
+                                                     gsword_sample_record* __restrict__ records) {
+    __shared__ PlanStep plan_s[kMaxQV];
+    __shared__ Partial warp_part[32];
+    extern __shared__ uint32_t Ms[];  // Ms[j * blockDim.x + tid] = M[j] of this lane
+
+    const int tid = threadIdx.x;
+    const int T = blockDim.x;
+    const int lane = tid & 31;
+    const int wbase = tid - lane;
+    const unsigned lt_mask = (1u << lane) - 1u;
+    if (tid < kMaxQV) plan_s[tid] = plan_in.step[tid];
+    __syncthreads();
+
+    const int nq = plan_in.nq;
+
+    // lane state
+    bool has = false;
+    uint64_t sid = 0;
+    int d = 0;
+    double W = 0.0;
+    // lane accumulators
+    double s_sum = 0.0, c_sum = 0.0, s_sq = 0.0, c_sq = 0.0;
+    unsigned long long n_valid = 0, n_done = 0;
+    double sectors = 0.0;
+
+    // warp chunk of the queue (warp-uniform)
+    uint64_t q_next = 0, q_end = 0;
+    bool exhausted = false;
+
+    while (true) {
+        // ---------------- A1: refill free lanes from the sample queue ----------------
+        unsigned need = __ballot_sync(kFull, !has);
+        while (need && !exhausted) {
+            if (q_next == q_end) {
+                unsigned long long base = 0;
+                if (lane == 0) base = atomicAdd(queue, (unsigned long long)chunk);
+                base = __shfl_sync(kFull, base, 0);
+                if (base >= count) {
+                    exhausted = true;
+                    break;
+                }
+                q_next = base;
+                q_end = ((uint64_t)base + (uint64_t)chunk < count) ? (uint64_t)base + (uint64_t)chunk : count;
+            }
+            const uint32_t avail = (q_end - q_next) < 32 ? (uint32_t)(q_end - q_next) : 32u;
+            const uint32_t rank = __popc(need & lt_mask);
+            if (!has && rank < avail) {
+                has = true;
+                sid = first + q_next + rank;
+                d = 0;
+                W = 1.0;
+                if (MODE == kModeTrace) {
+                    gsword_sample_record* rec = records + (sid - first);
+                    rec->sample_id = sid;
+#pragma unroll
+                    for (int i = 0; i < kMaxQV; ++i) {
+                        rec->path[i] = -1;
+                        rec->csize[i] = 0;
+                    }
+                }
+            }
+            q_next += min((uint32_t)__popc(need), avail);
+            need = __ballot_sync(kFull, !has);
+        }
+        if (!__any_sync(kFull, has)) break;
+        __syncwarp();
+
+        // ---------------- per-lane prologue: draw + GetMinCandidate -----------------
+        PlanStep ps = {0, 0u, 0u, 0};
+        uint64_t r = 0;
+        uint32_t lo_p = 0, len_p = 0;
+        int p = -1;
+        if (has) {
+            ps = plan_s[d];
+            r = philox_r(seed, sid, (uint32_t)d);
+            if (d == 0) {
+                lo_p = plan_in.seed_lo;
+                len_p = plan_in.seed_len;
+                if (MODE == kModeCount) sectors += plan_in.seed_identity ? 0.0 : 1.0;
+            } else {
+                // GetMinCandidate (Alg. 1 l.8): the smallest N_l(M[j]) over j in B(d)
+                uint32_t bm = ps.back;
+                len_p = 0xFFFFFFFFu;
+                while (bm) {
+                    const int j = __ffs(bm) - 1;
+                    bm &= bm - 1;
+                    uint32_t a, b;
+                    segment(g, Ms[j * T + tid], ps.label, &a, &b);
+                    if (b - a < len_p) {
+                        len_p = b - a;
+                        lo_p = a;
+                        p = j;
+                    }
+                }
+                if (MODE == kModeCount) sectors += (double)ps.nback;
+            }
+        }
+
+        uint32_t cnt = 0;     // |C_d|
+        int32_t v = -1;       // drawn vertex
+        bool reject = false;  // WJ Validate failure
+        if (METHOD == GSWORD_WJ) {
+            if (has) {
+                cnt = len_p;
+                if (cnt > 0) {
+                    const uint64_t k = __umul64hi(r, (uint64_t)cnt);
+                    if (d == 0) {
+                        v = plan_in.seed_identity ? (int32_t)(lo_p + k) : ldg_i32(g.bucket + lo_p + k);
+                    } else {
+                        v = ldg_i32(g.col + lo_p + k);
+                        if (MODE == kModeCount) sectors += 1.0;
+                        // Validate: DupCheck, then IsEdge for the other matched neighbours
+                        reject = !not_matched(Ms + tid, T, 0, ps.dup, v);
+                        uint32_t bm = ps.back & ~(1u << p);
+                        while (bm && !reject) {
+                            const int j = __ffs(bm) - 1;
+                            bm &= bm - 1;
+                            uint32_t a, b;
+                            segment(g, Ms[j * T + tid], ps.label, &a, &b);
+                            reject = !contains(g.col, a, b, v);
+                            if (MODE == kModeCount) sectors += (double)bs_sectors(b - a);
+                        }
+                    }
+                }
+            }
+        } else {
+            // ---------------- Alley Refine + Sample ----------------
+            bool coop = has && d > 0 && ps.nback >= 2 && len_p > coop_threshold;
+            if (has && !coop) {
+                if (d == 0) {
+                    cnt = len_p;
+                    if (cnt > 0) {
+                        const uint64_t k = __umul64hi(r, (uint64_t)cnt);
+                        v = plan_in.seed_identity ? (int32_t)(lo_p + k) : ldg_i32(g.bucket + lo_p + k);
+                    }
+                } else if (len_p == 0) {
+                    cnt = 0;
+                } else if (ps.nback == 1) {
+                    // C_d = S_p minus matched vertices lying in S_p (reading A5)
+                    uint32_t in_sp = 0;  // bit j: M[j] (same label) is an element of S_p
+                    uint32_t dm = ps.dup;
+                    while (dm) {
+                        const int j = __ffs(dm) - 1;
+                        dm &= dm - 1;
+                        if (contains(g.col, lo_p, lo_p + len_p, (int32_t)Ms[j * T + tid])) in_sp |= 1u << j;
+                        if (MODE == kModeCount) sectors += (double)bs_sectors(len_p);
+                    }
+                    cnt = len_p - __popc(in_sp);
+                    if (cnt > 0) {
+                        const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
+                        // smallest idx with idx = k + #{x in X : x <= S_p[idx]}
+                        uint32_t idx = k;
+                        while (true) {
+                            v = ldg_i32(g.col + lo_p + idx);
+                            uint32_t c = 0, xm = in_sp;
+                            while (xm) {
+                                const int j = __ffs(xm) - 1;
+                                xm &= xm - 1;
+                                c += ((int32_t)Ms[j * T + tid] <= v) ? 1u : 0u;
+                            }
+                            if (idx == k + c) break;
+                            idx = k + c;
+                        }
+                        if (MODE == kModeCount) sectors += 1.0;
+                    }
+                } else {
+                    // short driver: per-lane 64-bit refine bitmask over S_p
+                    uint64_t mask = (len_p >= 64) ? ~0ull : ((1ull << len_p) - 1ull);
+                    uint32_t bm = ps.back & ~(1u << p);
+                    while (bm && mask) {
+                        const int j = __ffs(bm) - 1;
+                        bm &= bm - 1;
+                        uint32_t a, b;
+                        segment(g, Ms[j * T + tid], ps.label, &a, &b);
+                        if (MODE == kModeCount)
+                            sectors += (double)min(len_p * bs_sectors(b - a), scan_sectors(b - a));
+                        uint64_t mm = mask;
+                        uint32_t cur = a;
+                        while (mm) {
+                            const int i = __ffsll((long long)mm) - 1;
+                            mm &= mm - 1;
+                            const int32_t x = ldg_i32(g.col + lo_p + i);
+                            bool f;
+                            cur = lower_bound(g.col, cur, b, x, &f);
+                            if (!f) mask &= ~(1ull << i);
+                        }
+                    }
+                    if (MODE == kModeCount) sectors += (double)scan_sectors(len_p);
+                    uint32_t dm = ps.dup;
+                    while (dm && mask) {
+                        const int j = __ffs(dm) - 1;
+                        dm &= dm - 1;
+                        bool f;
+                        const uint32_t pos = lower_bound(g.col, lo_p, lo_p + len_p, (int32_t)Ms[j * T + tid], &f);
+                        if (f) mask &= ~(1ull << (pos - lo_p));
+                    }
+                    cnt = __popcll(mask);
+                    if (cnt > 0) {
+                        const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
+                        v = ldg_i32(g.col + lo_p + fns64(mask, k));
+                    }
+                }
+            }
+            // ---------------- warp-cooperative refine for long drivers ----------------
+            unsigned cm = __ballot_sync(kFull, coop);
+            while (cm) {
+                const int L = __ffs(cm) - 1;
+                cm &= cm - 1;
+                const uint32_t Llo = __shfl_sync(kFull, lo_p, L);
+                const uint32_t Llen = __shfl_sync(kFull, len_p, L);
+                const int Lp = __shfl_sync(kFull, p, L);
+                const int Ld = __shfl_sync(kFull, d, L);
+                const uint32_t Lr_lo = __shfl_sync(kFull, (uint32_t)r, L);
+                const uint32_t Lr_hi = __shfl_sync(kFull, (uint32_t)(r >> 32), L);
+                const PlanStep Lps = plan_s[Ld];
+                const uint32_t others = Lps.back & ~(1u << Lp);
+                const int colL = wbase + L;
+                uint32_t total = 0, my_bal = 0;
+                for (uint32_t base = 0; base < Llen; base += 32) {
+                    const uint32_t i = base + lane;
+                    bool keep = i < Llen;
+                    int32_t x = 0;
+                    if (keep) {
+                        x = ldg_i32(g.col + Llo + i);
+                        keep = member_all(g, Ms, T, colL, others, Lps.label, x) &&
+                               not_matched(Ms, T, colL, Lps.dup, x);
+                    }
+                    const unsigned bal = __ballot_sync(kFull, keep);
+                    if ((base >> 5) == (uint32_t)lane) my_bal = bal;
+                    total += __popc(bal);
+                }
+                int32_t chosen = -1;
+                if (total > 0) {
+                    const uint64_t Lr = ((uint64_t)Lr_hi << 32) | Lr_lo;
+                    const uint32_t k = (uint32_t)__umul64hi(Lr, (uint64_t)total);
+                    if (Llen <= 32u * 32u) {
+                        // lane c holds the ballot of chunk c: warp scan of popcounts
+                        const uint32_t pc = __popc(my_bal);
+                        uint32_t incl = pc;
+#pragma unroll
+                        for (int o = 1; o < 32; o <<= 1) {
+                            const uint32_t y = __shfl_up_sync(kFull, incl, o);
+                            if (lane >= o) incl += y;
+                        }
+                        const uint32_t excl = incl - pc;
+                        const bool here = (k >= excl) && (k < incl);
+                        const unsigned hm = __ballot_sync(kFull, here);
+                        const int c = __ffs(hm) - 1;
+                        int32_t val = 0;
+                        if (lane == c) val = ldg_i32(g.col + Llo + (uint32_t)c * 32u + fns32(my_bal, k - excl));
+                        chosen = __shfl_sync(kFull, val, c);
+                    } else {
+                        uint32_t run = 0;
+                        for (uint32_t base = 0; base < Llen; base += 32) {
+                            const uint32_t i = base + lane;
+                            bool keep = i < Llen;
+                            int32_t x = 0;
+                            if (keep) {
+                                x = ldg_i32(g.col + Llo + i);
+                                keep = member_all(g, Ms, T, colL, others, Lps.label, x) &&
+                                       not_matched(Ms, T, colL, Lps.dup, x);
+                            }
+                            const unsigned bal = __ballot_sync(kFull, keep);
+                            const uint32_t c = __popc(bal);
+                            if (run + c > k) {
+                                chosen = __shfl_sync(kFull, x, (int)fns32(bal, k - run));
+                                break;
+                            }
+                            run += c;
+                        }
+                    }
+                }
+                if (lane == L) {
+                    cnt = total;
+                    v = chosen;
+                    if (MODE == kModeCount) {
+                        double s = (double)scan_sectors(Llen);
+                        uint32_t om = others;
+                        while (om) {
+                            const int j = __ffs(om) - 1;
+                            om &= om - 1;
+                            uint32_t a, b;
+                            segment(g, Ms[j * T + colL], Lps.label, &a, &b);
+                            s += (double)min(Llen * bs_sectors(b - a), scan_sectors(b - a));
+                        }
+                        sectors += s;
+                    }
+                }
+            }
+        }
+
+        // ---------------- common epilogue: HT weight, record, terminate ----------------
+        if (has) {
+            W = (d == 0) ? (double)cnt : __dmul_rn(W, (double)cnt);
+            if (MODE == kModeTrace) {
+                gsword_sample_record* rec = records + (sid - first);
+                rec->csize[d] = cnt;
+                rec->path[d] = (cnt > 0) ? v : -1;
+            }
+            bool dead = (cnt == 0) || reject;
+            bool complete = false;
+            if (!dead) {
+                Ms[d * T + tid] = (uint32_t)v;
+                if (d + 1 == nq) complete = true;
+            }
+            if (dead || complete) {
+                n_done += 1;
+                if (complete) {
+                    n_valid += 1;
+                    nsum(s_sum, c_sum, W);
+                    nsum(s_sq, c_sq, __dmul_rn(W, W));
+                }
+                if (MODE == kModeTrace) {
+                    gsword_sample_record* rec = records + (sid - first);
+                    rec->valid = complete ? 1 : 0;
+                    rec->depth_reached = (uint8_t)d;
+                    rec->weight = W;
+                }
+                has = false;
+            } else {
+                d += 1;
+            }
+        }
+    }
+
+    // ---------------- A10: warp -> CTA partial, fixed order ----------------
+    double sh = __dadd_rn(s_sum, c_sum), sl = __dsub_rn(c_sum, __dsub_rn(sh, s_sum));
+    double qh = __dadd_rn(s_sq, c_sq), ql = __dsub_rn(c_sq, __dsub_rn(qh, s_sq));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const double bh = shfl_xor_d(sh, o), bl = shfl_xor_d(sl, o);
+        const double ch = shfl_xor_d(qh, o), cl = shfl_xor_d(ql, o);
+        dd_add(sh, sl, bh, bl);
+        dd_add(qh, ql, ch, cl);
+        n_valid += __shfl_xor_sync(kFull, n_valid, o);
+        n_done += __shfl_xor_sync(kFull, n_done, o);
+        sectors += shfl_xor_d(sectors, o);
+    }
+    const int warp = tid >> 5;
+    if (lane == 0) {
+        warp_part[warp] = Partial{sh, sl, qh, ql, n_valid, n_done, sectors, 0.0};
+    }
+    __syncthreads();
+    if (tid == 0) {
+        Partial acc = warp_part[0];
+        for (int w = 1; w < (T >> 5); ++w) {
+            const Partial& o = warp_part[w];
+            dd_add(acc.sum_hi, acc.sum_lo, o.sum_hi, o.sum_lo);
+            dd_add(acc.sq_hi, acc.sq_lo, o.sq_hi, o.sq_lo);
+            acc.valid += o.valid;
+            acc.n += o.n;
+            acc.sectors += o.sectors;
+        }
+        partials[blockIdx.x] = acc;
+    }
+}
+
+// Grid reduction in CTA order (one warp; lane-strided then a fixed butterfly).
+__global__ void reduce_kernel(const Partial* __restrict__ partials, int n, double* __restrict__ out4,
+                              double* __restrict__ sectors_out) {
+    const int lane = threadIdx.x;
+    double sh = 0, sl = 0, qh = 0, ql = 0, sec = 0;
+    unsigned long long valid = 0, cnt = 0;
+    for (int i = lane; i < n; i += 32) {
+        const Partial p = partials[i];
+        dd_add(sh, sl, p.sum_hi, p.sum_lo);
+        dd_add(qh, ql, p.sq_hi, p.sq_lo);
+        valid += p.valid;
+        cnt += p.n;
+        sec += p.sectors;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const double bh = shfl_xor_d(sh, o), bl = shfl_xor_d(sl, o);
+        const double ch = shfl_xor_d(qh, o), cl = shfl_xor_d(ql, o);
+        dd_add(sh, sl, bh, bl);
+        dd_add(qh, ql, ch, cl);
+        valid += __shfl_xor_sync(kFull, valid, o);
+        cnt += __shfl_xor_sync(kFull, cnt, o);
+        sec += shfl_xor_d(sec, o);
+    }
+    if (lane == 0) {
+        out4[0] = __dadd_rn(sh, sl);
+        out4[1] = __dadd_rn(qh, ql);
+        out4[2] = (double)valid;
+        out4[3] = (double)cnt;
+        if (sectors_out) *sectors_out = sec;
+    }
+}
+
+__global__ void iota_kernel(int32_t* out, int64_t n) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = (int32_t)i;
+}
+
+template <int METHOD, int MODE>
+const void* kernel_ptr() {
+    return reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE>);
+}
+
+const void* select_kernel(int method, int mode) {
+    if (method == GSWORD_WJ) {
+        if (mode == kModeTrace) return kernel_ptr<GSWORD_WJ, kModeTrace>();
+        if (mode == kModeCount) return kernel_ptr<GSWORD_WJ, kModeCount>();
+        return kernel_ptr<GSWORD_WJ, kModeEstimate>();
+    }
+    if (mode == kModeTrace) return kernel_ptr<GSWORD_ALLEY, kModeTrace>();
+    if (mode == kModeCount) return kernel_ptr<GSWORD_ALLEY, kModeCount>();
+    return kernel_ptr<GSWORD_ALLEY, kModeEstimate>();
+}
+
+}  // namespace
+
+int max_blocks_per_sm(int method, int mode, int threads, size_t* smem_bytes) {
+    const size_t smem = (size_t)kMaxQV * (size_t)threads * sizeof(uint32_t);
+    if (smem_bytes) *smem_bytes = smem;
+    int blocks = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, select_kernel(method, mode), threads, smem) !=
+        cudaSuccess)
+        return 0;
+    return blocks;
+}
+
+cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan& plan, const LaunchCfg& cfg,
+                          uint64_t first, uint64_t count, uint64_t seed, unsigned long long* d_queue,
+                          Partial* d_partials, gsword_sample_record* d_records, cudaStream_t stream) {
+    cudaError_t e = cudaMemsetAsync(d_queue, 0, sizeof(unsigned long long), stream);
+    if (e != cudaSuccess) return e;
+    const size_t smem = (size_t)kMaxQV * (size_t)cfg.threads * sizeof(uint32_t);
+    const uint32_t thr = (uint32_t)cfg.coop_threshold;
+    void* args[] = {(void*)&g,      (void*)&plan,  (void*)&first,   (void*)&count,     (void*)&seed,
+                    (void*)&cfg.chunk, (void*)&thr, (void*)&d_queue, (void*)&d_partials, (void*)&d_records};
+    return cudaLaunchKernel(select_kernel(method, mode), dim3(cfg.grid), dim3(cfg.threads), args, smem, stream);
+}
+
+cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_out4, double* d_sectors,
+                          cudaStream_t stream) {
+    reduce_kernel<<<1, 32, 0, stream>>>(d_partials, n_partials, d_out4, d_sectors);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream) {
+    iota_kernel<<<148 * 4, 256, 0, stream>>>(bucket, n);
+    return cudaGetLastError();
+}
+
+}  // namespace gsword

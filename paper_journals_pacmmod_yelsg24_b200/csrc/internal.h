@@ -1,0 +1,76 @@
+// internal.h — structures shared by the host library (gsword_host.cpp) and the
+// sm_100a kernels (gsword_kernels.cu).  Not part of the public ABI.
+#pragma once
+
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+#include "../../include/gsword.h"
+
+namespace gsword {
+
+constexpr int kMaxQV = GSWORD_MAX_QV;
+
+// One matching-order position, staged into shared memory (16 B => one LDS.128).
+//   label : L_q(phi[d])
+//   back  : bitmask of backward positions B(d) (j < d, query edge to phi[d])
+//   dup   : bitmask of j < d with the same label (injectivity candidates, SURVEY R5')
+struct alignas(16) PlanStep {
+    int32_t label;
+    uint32_t back;
+    uint32_t dup;
+    int32_t nback;
+};
+
+struct Plan {
+    int32_t nq;
+    int32_t seed_identity;  // 1: seed set C(phi[0]) is 0..n-1 (unlabelled) -> no bucket gather
+    uint32_t seed_lo;       // C(phi[0]) = bucket[seed_lo, seed_lo + seed_len)
+    uint32_t seed_len;
+    PlanStep step[kMaxQV];
+};
+
+// Device-resident data graph, relaid out for the sampler:
+//   col[ seg[v*nL + l] .. seg[v*nL + l + 1] )  = N_l(v), ascending id
+//   seg has n*nL + 1 entries; for nL == 1 it is exactly row_ptr (as u32)
+//   bucket[ label_off[l] .. label_off[l+1] ) = {v : L(v) = l}, ascending id
+struct DeviceGraph {
+    const int32_t* col;
+    const uint32_t* seg;
+    const int32_t* bucket;
+    int64_t n;
+    int64_t nnz;
+    int32_t n_labels;
+};
+
+// Launch parameters of one estimate.
+struct LaunchCfg {
+    int grid;
+    int threads;
+    int chunk;
+    int coop_threshold;
+};
+
+// Per-CTA partial aggregate (written by the sampling kernel, reduced in CTA order).
+struct Partial {
+    double sum_hi, sum_lo;      // double-double sum of Y
+    double sq_hi, sq_lo;        // double-double sum of Y*Y
+    unsigned long long valid;   // complete instances
+    unsigned long long n;       // samples
+    double sectors;             // algorithmic sectors (counting build only)
+    double pad;
+};
+
+// Kernel entry points (gsword_kernels.cu).  All enqueue on `stream`.
+cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan& plan, const LaunchCfg& cfg,
+                          uint64_t first, uint64_t count, uint64_t seed, unsigned long long* d_queue,
+                          Partial* d_partials, gsword_sample_record* d_records, cudaStream_t stream);
+cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_out4, double* d_sectors,
+                          cudaStream_t stream);
+cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream);
+int max_blocks_per_sm(int method, int mode, int threads, size_t* smem_bytes);
+
+enum Mode { kModeEstimate = 0, kModeTrace = 1, kModeCount = 2 };
+
+}  // namespace gsword

@@ -1,0 +1,89 @@
+"""Multi-GPU layer (BASELINE.json north_star (4)).
+
+G is replicated on every rank (each rank loads the same canonical CSR), the global
+sample-id range is split contiguously, each rank runs the sampling +
+reduction kernels on its slice, and ONE all_reduce(SUM) of the 4 fp64 values
+{sum, sumsq, n_valid, n} combines them.  Counter-based Philox makes the union of the
+slices bit-identical, sample by sample, to a single-GPU run of the whole range.
+"""
+from __future__ import annotations
+
+from typing import Dict, Optional, Tuple
+
+from .gsword import Context, finalize
+
+
+def rank_range(n_total: int, rank: int, world: int, first: int = 0) -> Tuple[int, int]:
+    """Rank r of P takes [first + floor(r n / P), first + floor((r+1) n / P)).
+    Returns (first_sample_id, count)."""
+    if world < 1 or not 0 <= rank < world:
+        raise ValueError("bad rank/world")
+    a = (n_total * rank) // world
+    b = (n_total * (rank + 1)) // world
+    return first + a, b - a
+
+
+def allreduce_sum4(t4, group=None):
+    """The one collective of the path: SUM over ranks of the 4-vector (in place)."""
+    import torch.distributed as dist
+    dist.all_reduce(t4, op=dist.ReduceOp.SUM, group=group)
+    return t4
+
+
+def estimate_distributed(ctx: Context, method: int, n_total: int, seed: int, first: int = 0, group=None,
+                         out4=None) -> Dict[str, float]:
+    """Every rank calls this with the same arguments; every rank gets the combined
+    result.  The kernels and the NCCL all_reduce run on torch's current stream, so no
+    host synchronisation sits between them."""
+    import torch
+    import torch.distributed as dist
+
+    rank = dist.get_rank(group) if dist.is_initialized() else 0
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    f, cnt = rank_range(n_total, rank, world, first)
+    dev = torch.device("cuda", ctx.device)
+    stream = torch.cuda.current_stream(dev)
+    ctx.set_stream(stream)
+    if out4 is None:
+        out4 = torch.zeros(4, dtype=torch.float64, device=dev)
+    else:
+        out4.zero_()
+    if cnt > 0:
+        ctx.estimate_async(method, f, cnt, seed, out4)
+    if world > 1:
+        allreduce_sum4(out4, group)
+    return finalize(out4.cpu().numpy())
+
+
+def combine_host(values4_per_rank) -> Dict[str, float]:
+    """Host-side equivalent of the all_reduce + finalize (for checkpoint/resume of
+    partial ranges): element-wise sum of {sum, sumsq, n_valid, n} then finalize."""
+    import numpy as np
+    acc = np.zeros(4, np.float64)
+    for v in values4_per_rank:
+        acc += np.asarray(v, np.float64).reshape(4)
+    return finalize(acc)
+
+
+def init_from_env(backend: Optional[str] = None):
+    """torchrun plumbing: init the process group from RANK/WORLD_SIZE/MASTER_* and bind
+    LOCAL_RANK's GPU.  Returns (rank, world, local_rank)."""
+    import os
+
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1 and not dist.is_initialized():
+        if backend is None:
+            backend = "nccl" if torch.cuda.is_available() else "gloo"
+        if backend == "nccl":
+            torch.cuda.set_device(local)
+            dist.init_process_group(backend, device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    elif torch.cuda.is_available():
+        torch.cuda.set_device(local)
+    return rank, world, local

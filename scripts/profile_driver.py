@@ -1,0 +1,31 @@
+"""Short, fixed launch sequence for ncu captures (one GPU, never multi-rank):
+2 warm-up estimates (WanderJoin, Alley; 1e6 samples), then WanderJoin and Alley at
+--samples each on the bench workload.  Use `ncu -k regex:sample_kernel -s 2 -c 2`."""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import paper_journals_pacmmod_yelsg24_b200 as G  # noqa: E402
+from workloads import gen  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--samples", type=float, default=1e7)
+ap.add_argument("--config", default="C1")
+ap.add_argument("--query", type=int, default=1)
+ap.add_argument("--l2", type=int, default=0)
+args = ap.parse_args()
+
+g, qs = gen.CONFIGS[args.config]()
+q = qs[args.query]
+with G.Context(0) as ctx:
+    ctx.set_option(G.OPT_L2_PERSIST, args.l2)
+    ctx.load_graph_obj(g)
+    ctx.load_query_obj(q)
+    for m in (G.WJ, G.ALLEY):
+        ctx.estimate(m, 1_000_000, 42)
+    for m in (G.WJ, G.ALLEY):
+        r = ctx.estimate(m, int(args.samples), 42)
+        print(f"method={m} samples={int(args.samples)} seconds={r['seconds']:.4f} "
+              f"rate={args.samples / r['seconds']:.3e}/s est={r['estimate']:.4e} valid={r['n_valid']}")

@@ -1,0 +1,260 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Per sample: bit-exact records (path, csize, validity, fp64 weight) for every sample
+id compared.  Aggregates: sum and sumsq within a relative 1e-12 (BASELINE.json
+north_star), n and n_valid exact, variance within the cancellation-aware bound of
+DESIGN.md §4.  Inputs are the seeded workloads of workloads/gen.py.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+from workloads import gen
+
+pytestmark = pytest.mark.gpu
+
+REL = 1e-12
+
+
+@pytest.fixture(scope="module")
+def G():
+    import paper_journals_pacmmod_yelsg24_b200 as G
+    return G
+
+
+@pytest.fixture(scope="module")
+def ctx(G):
+    c = G.Context(0)
+    yield c
+    c.close()
+
+
+def _records_equal(gpu, ref, what=""):
+    assert gpu.shape == ref.shape
+    if gpu.tobytes() == ref.tobytes():
+        return
+    for f in ("sample_id", "valid", "depth_reached", "path", "csize", "weight"):
+        bad = np.nonzero(np.any((gpu[f] != ref[f]).reshape(gpu.shape[0], -1), axis=1))[0]
+        if bad.size:
+            i = int(bad[0])
+            raise AssertionError(f"{what}: field {f} differs at {bad.size} samples; first sid "
+                                 f"{int(ref['sample_id'][i])}: gpu={gpu[i]} oracle={ref[i]}")
+    raise AssertionError(f"{what}: records differ in padding")
+
+
+def _agg_close(gpu, ref, G):
+    assert gpu["n"] == ref["n"]
+    assert gpu["n_valid"] == ref["n_valid"]
+    for k in ("sum", "sumsq", "estimate"):
+        assert gpu[k] == pytest.approx(ref[k], rel=REL, abs=0.0), k
+    if gpu["n"] >= 2:
+        assert abs(gpu["variance"] - ref["variance"]) <= G.variance_tolerance(ref) + REL * abs(ref["variance"])
+
+
+def _parity(ctx, G, g, q, method, seed, first, count, threads=8, loaded=False):
+    if not loaded:
+        ctx.load_graph_obj(g)
+    ctx.load_query_obj(q)
+    rec = ctx.trace_samples(method, first, count, seed)
+    y, ref = oracle.sample_range(g, q, method, seed, first, count, records=True, threads=threads)
+    _records_equal(rec, ref, f"{g.name}/{q.name}/m{method}")
+    agg = ctx.estimate(method, count, seed, first=first)
+    _agg_close(agg, oracle.aggregate(y), G)
+    return rec
+
+
+# ------------------------------------------------------------------ C0 (BASELINE configs[0])
+@pytest.mark.parametrize("method", [0, 1])
+def test_c0_full_parity(ctx, G, c0, method):
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    for qi, q in enumerate(qs):
+        _parity(ctx, G, g, q, method, seed=1 + qi, first=0, count=100_000, loaded=True)
+
+
+def test_c0_estimate_near_exact(ctx, G, c0):
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    for q in qs[:6]:
+        truth = oracle.count_embeddings(g, q)
+        ctx.load_query_obj(q)
+        for m in (G.WJ, G.ALLEY):
+            r = ctx.estimate(m, 1_000_000, seed=7)
+            assert abs(r["estimate"] - truth) <= 5 * math.sqrt(max(r["variance"], 0.0)) + 1e-9
+
+
+# ------------------------------------------------------------------ fuzz: tiny random inputs
+@pytest.mark.parametrize("seed", range(16))
+def test_fuzz_small(ctx, G, seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(5, 40))
+    nl = int(rng.integers(1, 5))
+    g = gen.random_small_graph(n, float(rng.uniform(0.15, 0.7)), nl, seed=1000 + seed)
+    nq = int(rng.integers(1, min(n, 9) + 1))
+    if seed % 2 == 0:
+        q = gen.random_connected_query(nq, float(rng.uniform(0, 0.6)), nl, 2000 + seed)
+    else:
+        try:
+            q = gen.extract_query(g, nq, 3000 + seed, dense=bool(seed % 4 == 1))
+            q = q.with_order(gen.random_connected_order(q, seed))
+        except RuntimeError:
+            q = gen.random_connected_query(nq, 0.3, nl, 2000 + seed)
+    ctx.load_graph_obj(g)
+    for m in (0, 1):
+        _parity(ctx, G, g, q, m, seed=seed, first=int(rng.integers(0, 2**40)), count=3000, loaded=True)
+
+
+# ------------------------------------------------------------------ closed forms on the GPU
+def test_alley_zero_variance_on_gpu(ctx, G):
+    for n, k in ((9, 4), (80, 3), (100, 5)):  # n-1 >= 64 exercises the warp-cooperative refine
+        g = gen.complete_graph(n)
+        ctx.load_graph_obj(g)
+        ctx.load_query_obj(gen.clique_query(k))
+        r = ctx.estimate(G.ALLEY, 20_000, seed=3)
+        want = float(math.factorial(n) // math.factorial(n - k))
+        assert r["n_valid"] == 20_000 and r["estimate"] == want and abs(r["variance"]) <= G.variance_tolerance(r)
+
+
+@pytest.mark.parametrize("coop", [0, 1, 17, 32, 64])
+def test_coop_threshold_invariance(ctx, G, coop):
+    """The warp-cooperative and per-lane refine paths give identical samples."""
+    g = gen.chung_lu(3000, 60_000, gamma=2.2, max_over_mean=40.0, seed=5, labels=gen.uniform_labels(3000, 2, 6),
+                     n_labels=2)
+    q = gen.extract_query(g, 6, seed=8, dense=True)
+    ctx.set_option(G.OPT_COOP_THRESHOLD, coop)
+    try:
+        _parity(ctx, G, g, q, G.ALLEY, seed=4, first=0, count=20_000)
+    finally:
+        ctx.set_option(G.OPT_COOP_THRESHOLD, 32)
+
+
+def test_edge_cases(ctx, G):
+    g = gen.random_small_graph(30, 0.3, 3, seed=9)
+    ctx.load_graph_obj(g)
+    # single-vertex query: every sample valid with W = |C(u)|
+    q1 = gen.query_from_edges(1, [], labels=[1], order=[0])
+    ctx.load_query_obj(q1)
+    r = ctx.estimate(G.WJ, 1000, seed=1)
+    assert r["n_valid"] == 1000 and r["estimate"] == float(np.sum(g.labels == 1))
+    # one sample
+    q = gen.extract_query(g, 3, seed=2, dense=True)
+    _parity(ctx, G, g, q, G.ALLEY, seed=5, first=123, count=1, loaded=True)
+    # a query label that no data vertex has: every sample dead, estimate 0
+    lab = np.asarray(g.labels).copy()
+    lab[lab == 2] = 0
+    g2 = gen.Graph(g.row_ptr, g.col, lab, 3)
+    q2 = gen.query_from_edges(2, [(0, 1)], labels=[2, 0], order=[0, 1])
+    for m in (0, 1):
+        _parity(ctx, G, g2, q2, m, seed=1, first=0, count=500)
+    # the largest query: 16-clique in K_20 (W = 20!/4! beyond 2^53: fp64 rounding order)
+    _parity(ctx, G, gen.complete_graph(20), gen.clique_query(16), G.ALLEY, seed=2, first=0, count=2000)
+    _parity(ctx, G, gen.complete_graph(20), gen.clique_query(16), G.WJ, seed=2, first=0, count=2000)
+
+
+def test_errors(G):
+    c = G.Context(0)
+    with pytest.raises(G.GswordError) as e:
+        c.estimate(G.WJ, 10, 1)
+    assert e.value.status == -2
+    g = gen.ring_graph(10)
+    c.load_graph_obj(g)
+    with pytest.raises(G.GswordError) as e:
+        c.estimate(G.WJ, 10, 1)
+    assert e.value.status == -3
+    q = gen.path_query(3)
+    with pytest.raises(G.GswordError) as e:
+        c.load_query(*q.csr(), q.labels, [0, 2, 1])
+    assert e.value.status == -4
+    bad_col = g.col.copy()
+    bad_col[0], bad_col[1] = bad_col[1], bad_col[0]
+    with pytest.raises(G.GswordError) as e:
+        c.load_graph(g.row_ptr, bad_col)
+    assert e.value.status == -5
+    c.close()
+
+
+# ------------------------------------------------------------------ C2 / C1 (paper-shaped)
+def test_c2_parity(ctx, G):
+    g, qs = gen.config_c2()
+    ctx.load_graph_obj(g)
+    for i, q in enumerate(qs):
+        for m in (0, 1):
+            _parity(ctx, G, g, q, m, seed=10 + i, first=0, count=50_000, loaded=True)
+
+
+@pytest.fixture(scope="module")
+def c1():
+    return gen.config_c1()
+
+
+def test_c1_parity_prefix(ctx, G, c1):
+    g, qs = c1
+    ctx.load_graph_obj(g)
+    for q in qs:
+        for m in (0, 1):
+            _parity(ctx, G, g, q, m, seed=42, first=0, count=20_000, loaded=True)
+
+
+def test_c1_full_size_sampled_and_split(ctx, G, c1):
+    """BASELINE configs[1] at its full budget (1e8 samples, the bench launch config):
+    sampled sample ids against the oracle, plus split-range invariance of the whole."""
+    g, qs = c1
+    ctx.load_graph_obj(g)
+    n = 100_000_000
+    for q in qs:
+        ctx.load_query_obj(q)
+        for m in (0, 1):
+            for first in (0, 31_415_926, n - 1500):
+                rec = ctx.trace_samples(m, first, 1500, 42)
+                _, ref = oracle.sample_range(g, q, m, 42, first, 1500, records=True, threads=8)
+                _records_equal(rec, ref, f"C1/{q.name}/m{m}@{first}")
+            full = ctx.estimate(m, n, 42)
+            a = ctx.estimate(m, 37_000_000, 42, first=0)
+            b = ctx.estimate(m, n - 37_000_000, 42, first=37_000_000)
+            assert full["n"] == n and a["n"] + b["n"] == n
+            assert full["n_valid"] == a["n_valid"] + b["n_valid"]
+            assert full["sum"] == pytest.approx(a["sum"] + b["sum"], rel=REL)
+            assert full["sumsq"] == pytest.approx(a["sumsq"] + b["sumsq"], rel=REL)
+
+
+def test_scheduling_invariance(ctx, G, c0):
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    q = qs[3]
+    ctx.load_query_obj(q)
+    base = {m: ctx.estimate(m, 400_000, 9) for m in (0, 1)}
+    try:
+        for opt, val in ((G.OPT_CHUNK, 1), (G.OPT_CHUNK, 4096), (G.OPT_BLOCKS_PER_SM, 1),
+                         (G.OPT_THREADS, 64), (G.OPT_L2_PERSIST, 1)):
+            ctx.set_option(opt, val)
+            for m in (0, 1):
+                r = ctx.estimate(m, 400_000, 9)
+                assert r["n_valid"] == base[m]["n_valid"]
+                assert r["sum"] == pytest.approx(base[m]["sum"], rel=REL)
+                assert r["sumsq"] == pytest.approx(base[m]["sumsq"], rel=REL)
+    finally:
+        ctx.set_option(G.OPT_CHUNK, 256)
+        ctx.set_option(G.OPT_BLOCKS_PER_SM, 0)
+        ctx.set_option(G.OPT_THREADS, 256)
+        ctx.set_option(G.OPT_L2_PERSIST, 0)
+
+
+def test_async_matches_sync_on_torch_stream(ctx, G, c0):
+    import torch
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    ctx.load_query_obj(qs[0])
+    s = torch.cuda.Stream()
+    ctx.set_stream(s)
+    try:
+        out = torch.zeros(4, dtype=torch.float64, device="cuda")
+        with torch.cuda.stream(s):
+            ctx.estimate_async(G.ALLEY, 0, 50_000, 3, out)
+        s.synchronize()
+        r = G.finalize(out.cpu().numpy())
+        ref = ctx.estimate(G.ALLEY, 50_000, 3)
+        assert r["sum"] == ref["sum"] and r["n_valid"] == ref["n_valid"]
+    finally:
+        ctx.set_stream(None)
