@@ -321,8 +321,9 @@ def run_ours(args):
         with open(args.traffic_file) as f:
             tf = json.load(f)
         key = "wj" if dom == G.WJ else "alley"
-        if tf.get("workload") == WORKLOAD and key in tf.get("dram_bytes_per_launch", {}):
-            traffic = float(tf["dram_bytes_per_launch"][key])
+        if tf.get("workload") == WORKLOAD and key in tf.get("dram_bytes_per_sample", {}):
+            # ncu capture (cold cache, serialised) scaled to this launch's samples
+            traffic = float(tf["dram_bytes_per_sample"][key]) * cnt
     except Exception:
         traffic = None
 
