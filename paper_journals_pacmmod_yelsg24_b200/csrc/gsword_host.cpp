@@ -155,6 +155,8 @@ int plan_query_impl(int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, 
             if (q_labels[order[j]] == q_labels[u]) s.dup |= 1u << j;
         }
         s.nback = __builtin_popcount(s.back);
+        for (int j = 0; j < nq; ++j)
+            if (j != d && adj[order[j]][u]) p.qadj[d] |= 1u << j;
         if (d > 0 && s.back == 0)
             return fail(GSWORD_EORDER, "load_query: order prefix %d is not connected (reading A13)", d);
     }
@@ -202,7 +204,7 @@ struct gsword_ctx {
     int opt_threads = 256;
     int opt_chunk = 256;
     int opt_l2 = 0;
-    int opt_coop = 32;
+    int opt_coop = 64;
     // last launch
     int last_grid = 0, last_threads = 0;
 

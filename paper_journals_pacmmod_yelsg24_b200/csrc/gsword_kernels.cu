@@ -50,28 +50,49 @@ __device__ __forceinline__ uint64_t philox_r(uint64_t seed, uint64_t sid, uint32
 __device__ __forceinline__ int32_t ldg_i32(const int32_t* p) { return __ldg(p); }
 __device__ __forceinline__ uint32_t ldg_u32(const uint32_t* p) { return __ldg(p); }
 
-// first index i in [lo, hi) with col[i] >= x (hi if none); *found = (col[i] == x)
-__device__ __forceinline__ uint32_t lower_bound(const int32_t* __restrict__ col, uint32_t lo, uint32_t hi,
-                                                int32_t x, bool* found) {
-    uint32_t n = hi - lo;
-    while (n > 0) {
-        const uint32_t half = n >> 1;
-        const int32_t y = ldg_i32(col + lo + half);
-        if (y < x) {
-            lo += half + 1;
-            n -= half + 1;
-        } else {
-            n = half;
-        }
+// Branchless search over the ascending run col[lo, lo+n): the trip count depends on
+// n only (no data-dependent branches).  Returns the index of the last element <= x
+// (lo if none) and whether it equals x.
+__device__ __forceinline__ uint32_t search_last_le(const int32_t* __restrict__ col, uint32_t lo, uint32_t n,
+                                                   int32_t x, bool* found) {
+    if (n == 0) {
+        *found = false;
+        return lo;
     }
-    *found = (lo < hi) && (ldg_i32(col + lo) == x);
+    while (n > 1) {
+        const uint32_t half = n >> 1;
+        lo = (ldg_i32(col + lo + half) <= x) ? lo + half : lo;
+        n -= half;
+    }
+    *found = ldg_i32(col + lo) == x;
     return lo;
 }
 
-__device__ __forceinline__ bool contains(const int32_t* __restrict__ col, uint32_t lo, uint32_t hi, int32_t x) {
+__device__ __forceinline__ bool in_run(const int32_t* __restrict__ col, uint32_t lo, uint32_t hi, int32_t x) {
     bool f;
-    lower_bound(col, lo, hi, x, &f);
+    search_last_le(col, lo, hi - lo, x, &f);
     return f;
+}
+
+// Up to 4 keys searched in lock step over the same run (independent loads in flight;
+// the first probes coincide and hit L1).  Bit t of the result: key t is present.
+__device__ __forceinline__ uint32_t has4(const int32_t* __restrict__ col, uint32_t lo, uint32_t n, int nk,
+                                         int32_t x0, int32_t x1, int32_t x2, int32_t x3) {
+    if (n == 0) return 0u;
+    uint32_t b0 = lo, b1 = lo, b2 = lo, b3 = lo;
+    while (n > 1) {
+        const uint32_t half = n >> 1;
+        b0 = (ldg_i32(col + b0 + half) <= x0) ? b0 + half : b0;
+        if (nk > 1) b1 = (ldg_i32(col + b1 + half) <= x1) ? b1 + half : b1;
+        if (nk > 2) b2 = (ldg_i32(col + b2 + half) <= x2) ? b2 + half : b2;
+        if (nk > 3) b3 = (ldg_i32(col + b3 + half) <= x3) ? b3 + half : b3;
+        n -= half;
+    }
+    uint32_t r = (ldg_i32(col + b0) == x0) ? 1u : 0u;
+    if (nk > 1 && ldg_i32(col + b1) == x1) r |= 2u;
+    if (nk > 2 && ldg_i32(col + b2) == x2) r |= 4u;
+    if (nk > 3 && ldg_i32(col + b3) == x3) r |= 8u;
+    return r;
 }
 
 // position of the k-th (0-based) set bit of m (k < popc(m))
@@ -135,7 +156,7 @@ __device__ __forceinline__ bool member_all(const DeviceGraph& g, const uint32_t*
         mask &= mask - 1;
         uint32_t a, b;
         segment(g, Ms[j * stride + col_of], l, &a, &b);
-        if (!contains(g.col, a, b, x)) return false;
+        if (!in_run(g.col, a, b, x)) return false;
     }
     return true;
 }
@@ -157,6 +178,10 @@ __global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const 
                                                      Partial* __restrict__ partials,
                                                      gsword_sample_record* __restrict__ records) {
     __shared__ PlanStep plan_s[kMaxQV];
+    __shared__ uint32_t qadj_s[kMaxQV];
+    __shared__ uint32_t res_s[256];   // Alley task-pool results per lane (adjacent matched vertices)
+    __shared__ uint32_t rmlo_s[256];  // Alley task-pool results per lane (refine-mask removals)
+    __shared__ uint32_t rmhi_s[256];
     __shared__ Partial warp_part[32];
     extern __shared__ uint32_t Ms[];  // Ms[j * blockDim.x + tid] = M[j] of this lane
 
@@ -165,7 +190,10 @@ __global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const 
     const int lane = tid & 31;
     const int wbase = tid - lane;
     const unsigned lt_mask = (1u << lane) - 1u;
-    if (tid < kMaxQV) plan_s[tid] = plan_in.step[tid];
+    if (tid < kMaxQV) {
+        plan_s[tid] = plan_in.step[tid];
+        qadj_s[tid] = plan_in.qadj[tid];
+    }
     __syncthreads();
 
     const int nq = plan_in.nq;
@@ -266,98 +294,156 @@ __global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const 
                     } else {
                         v = ldg_i32(g.col + lo_p + k);
                         if (MODE == kModeCount) sectors += 1.0;
-                        // Validate: DupCheck, then IsEdge for the other matched neighbours
+                        // Validate: DupCheck, then IsEdge for the other matched neighbours.
+                        // v in N_l(M[j]) <=> M[j] in N_{L(phi[j])}(v): search the shorter run.
                         reject = !not_matched(Ms + tid, T, 0, ps.dup, v);
                         uint32_t bm = ps.back & ~(1u << p);
                         while (bm && !reject) {
                             const int j = __ffs(bm) - 1;
                             bm &= bm - 1;
-                            uint32_t a, b;
-                            segment(g, Ms[j * T + tid], ps.label, &a, &b);
-                            reject = !contains(g.col, a, b, v);
-                            if (MODE == kModeCount) sectors += (double)bs_sectors(b - a);
+                            const uint32_t mj = Ms[j * T + tid];
+                            uint32_t a, b, a2, b2;
+                            segment(g, mj, ps.label, &a, &b);
+                            segment(g, (uint32_t)v, plan_s[j].label, &a2, &b2);
+                            if (b2 - a2 < b - a) reject = !in_run(g.col, a2, b2, (int32_t)mj);
+                            else reject = !in_run(g.col, a, b, v);
+                            if (MODE == kModeCount) sectors += 1.0 + (double)bs_sectors(min(b - a, b2 - a2));
                         }
                     }
                 }
             }
         } else {
-            // ---------------- Alley Refine + Sample ----------------
-            bool coop = has && d > 0 && ps.nback >= 2 && len_p > coop_threshold;
-            if (has && !coop) {
+            // ---------------- Alley Refine + Sample (Fig. 19 AL) ----------------
+            // kind 1: |B(d)| = 1 -> C_d = S_p minus matched same-label vertices in S_p
+            // kind 2: |B(d)| >= 2, |S_p| <= threshold -> refine bitmask over S_p, membership
+            //         tests pooled across the warp
+            // kind 3: |B(d)| >= 2, |S_p| > threshold -> warp-cooperative chunks (below)
+            int kind = 0;
+            uint32_t unk = 0, known = 0, others = 0;
+            if (has) {
                 if (d == 0) {
                     cnt = len_p;
                     if (cnt > 0) {
                         const uint64_t k = __umul64hi(r, (uint64_t)cnt);
                         v = plan_in.seed_identity ? (int32_t)(lo_p + k) : ldg_i32(g.bucket + lo_p + k);
                     }
-                } else if (len_p == 0) {
-                    cnt = 0;
-                } else if (ps.nback == 1) {
-                    // C_d = S_p minus matched vertices lying in S_p (reading A5)
-                    uint32_t in_sp = 0;  // bit j: M[j] (same label) is an element of S_p
-                    uint32_t dm = ps.dup;
-                    while (dm) {
-                        const int j = __ffs(dm) - 1;
-                        dm &= dm - 1;
-                        if (contains(g.col, lo_p, lo_p + len_p, (int32_t)Ms[j * T + tid])) in_sp |= 1u << j;
-                        if (MODE == kModeCount) sectors += (double)bs_sectors(len_p);
-                    }
-                    cnt = len_p - __popc(in_sp);
-                    if (cnt > 0) {
-                        const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
-                        // smallest idx with idx = k + #{x in X : x <= S_p[idx]}
-                        uint32_t idx = k;
-                        while (true) {
-                            v = ldg_i32(g.col + lo_p + idx);
-                            uint32_t c = 0, xm = in_sp;
-                            while (xm) {
-                                const int j = __ffs(xm) - 1;
-                                xm &= xm - 1;
-                                c += ((int32_t)Ms[j * T + tid] <= v) ? 1u : 0u;
-                            }
-                            if (idx == k + c) break;
-                            idx = k + c;
-                        }
-                        if (MODE == kModeCount) sectors += 1.0;
-                    }
-                } else {
-                    // short driver: per-lane 64-bit refine bitmask over S_p
-                    uint64_t mask = (len_p >= 64) ? ~0ull : ((1ull << len_p) - 1ull);
-                    uint32_t bm = ps.back & ~(1u << p);
-                    while (bm && mask) {
-                        const int j = __ffs(bm) - 1;
-                        bm &= bm - 1;
-                        uint32_t a, b;
-                        segment(g, Ms[j * T + tid], ps.label, &a, &b);
-                        if (MODE == kModeCount)
-                            sectors += (double)min(len_p * bs_sectors(b - a), scan_sectors(b - a));
-                        uint64_t mm = mask;
-                        uint32_t cur = a;
-                        while (mm) {
-                            const int i = __ffsll((long long)mm) - 1;
-                            mm &= mm - 1;
-                            const int32_t x = ldg_i32(g.col + lo_p + i);
-                            bool f;
-                            cur = lower_bound(g.col, cur, b, x, &f);
-                            if (!f) mask &= ~(1ull << i);
-                        }
-                    }
-                    if (MODE == kModeCount) sectors += (double)scan_sectors(len_p);
-                    uint32_t dm = ps.dup;
-                    while (dm && mask) {
-                        const int j = __ffs(dm) - 1;
-                        dm &= dm - 1;
-                        bool f;
-                        const uint32_t pos = lower_bound(g.col, lo_p, lo_p + len_p, (int32_t)Ms[j * T + tid], &f);
-                        if (f) mask &= ~(1ull << (pos - lo_p));
-                    }
-                    cnt = __popcll(mask);
-                    if (cnt > 0) {
-                        const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
-                        v = ldg_i32(g.col + lo_p + fns64(mask, k));
+                } else if (len_p > 0) {
+                    if (ps.nback == 1) {
+                        // M[j] (same label) with (phi[j], phi[p]) a query edge lies in S_p by the
+                        // Alley invariant (every drawn prefix is a partial instance); M[p] never
+                        // does (no self loops); the rest need an adjacency test.
+                        const uint32_t qa = qadj_s[p];
+                        kind = 1;
+                        known = ps.dup & qa;
+                        unk = ps.dup & ~qa & ~(1u << p);
+                    } else if (len_p <= coop_threshold) {
+                        kind = 2;
+                        others = ps.back & ~(1u << p);
+                        if (MODE == kModeCount) sectors += (double)scan_sectors(len_p);
+                    } else {
+                        kind = 3;
                     }
                 }
             }
+
+            // ---- warp task pool: every lane executes one adjacency test per round ----
+            const uint32_t ntask = (kind == 1) ? (uint32_t)__popc(unk)
+                                 : (kind == 2) ? len_p * (uint32_t)__popc(others) : 0u;
+            res_s[tid] = 0u;
+            rmlo_s[tid] = 0u;
+            rmhi_s[tid] = 0u;
+            uint32_t incl = ntask;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, incl, o);
+                if (lane >= o) incl += y;
+            }
+            const uint32_t total = __shfl_sync(kFull, incl, 31);
+            const uint32_t excl = incl - ntask;
+            __syncwarp();
+            for (uint32_t base = 0; base < total; base += 32) {
+                const uint32_t t = base + (uint32_t)lane;
+                const uint32_t tt = t < total ? t : total - 1;
+                int o = 0;  // owner lane: number of lanes whose inclusive count <= tt
+#pragma unroll
+                for (int s = 16; s >= 1; s >>= 1) {
+                    const uint32_t y = __shfl_sync(kFull, incl, o + s - 1);
+                    if (y <= tt) o += s;
+                }
+                const uint32_t k = tt - __shfl_sync(kFull, excl, o);
+                const int okind = __shfl_sync(kFull, kind, o);
+                const uint32_t olo = __shfl_sync(kFull, lo_p, o);
+                const uint32_t olen = __shfl_sync(kFull, len_p, o);
+                const int op = __shfl_sync(kFull, p, o);
+                const uint32_t omask = __shfl_sync(kFull, (kind == 1) ? unk : others, o);
+                const int32_t olab = __shfl_sync(kFull, ps.label, o);
+                if (t < total) {
+                    const int ocol = wbase + o;
+                    if (okind == 1) {
+                        // is M[j] adjacent to M[p]?  search the shorter of N_l(M[p]) = S_p and
+                        // N_{L(phi[p])}(M[j])
+                        const int j = (int)fns32(omask, k);
+                        const uint32_t key = Ms[j * T + ocol];
+                        const uint32_t mp = Ms[op * T + ocol];
+                        uint32_t a, b;
+                        segment(g, key, plan_s[op].label, &a, &b);
+                        const bool adj = (b - a < olen) ? in_run(g.col, a, b, (int32_t)mp)
+                                                        : in_run(g.col, olo, olo + olen, (int32_t)key);
+                        if (adj) atomicOr(&res_s[ocol], 1u << j);
+                        if (MODE == kModeCount) sectors += 1.0 + (double)bs_sectors(min(b - a, olen));
+                    } else {
+                        // is S_p[i] in N_l(M[j])?
+                        const uint32_t nth = k / olen;
+                        const uint32_t i = k - nth * olen;
+                        const int j = (int)fns32(omask, nth);
+                        const int32_t x = ldg_i32(g.col + olo + i);
+                        uint32_t a, b;
+                        segment(g, Ms[j * T + ocol], olab, &a, &b);
+                        if (!in_run(g.col, a, b, x)) atomicOr(i < 32 ? &rmlo_s[ocol] : &rmhi_s[ocol], 1u << (i & 31));
+                        if (MODE == kModeCount) sectors += (double)bs_sectors(b - a);
+                    }
+                }
+            }
+            __syncwarp();
+            if (kind == 1) {
+                const uint32_t in_sp = known | res_s[tid];  // matched vertices inside S_p
+                cnt = len_p - __popc(in_sp);
+                if (cnt > 0) {
+                    const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
+                    // smallest idx with idx = k + #{x in X : x <= S_p[idx]}: the k-th survivor
+                    uint32_t idx = k;
+                    while (true) {
+                        v = ldg_i32(g.col + lo_p + idx);
+                        uint32_t c = 0, xm = in_sp;
+                        while (xm) {
+                            const int j = __ffs(xm) - 1;
+                            xm &= xm - 1;
+                            c += ((int32_t)Ms[j * T + tid] <= v) ? 1u : 0u;
+                        }
+                        if (idx == k + c) break;
+                        idx = k + c;
+                    }
+                    if (MODE == kModeCount) sectors += 1.0;
+                }
+            } else if (kind == 2) {
+                uint64_t mask = (len_p >= 64) ? ~0ull : ((1ull << len_p) - 1ull);
+                mask &= ~(((uint64_t)rmhi_s[tid] << 32) | (uint64_t)rmlo_s[tid]);
+                // injectivity: drop survivors equal to a matched same-label vertex
+                uint64_t mm = mask;
+                const uint32_t dup = ps.dup & ~(1u << p);
+                while (mm && dup) {
+                    const int i = __ffsll((long long)mm) - 1;
+                    mm &= mm - 1;
+                    if (!not_matched(Ms + tid, T, 0, dup, ldg_i32(g.col + lo_p + i))) mask &= ~(1ull << i);
+                }
+                cnt = __popcll(mask);
+                if (cnt > 0) {
+                    const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
+                    v = ldg_i32(g.col + lo_p + fns64(mask, k));
+                }
+            }
+            const bool coop = (kind == 3);
+
             // ---------------- warp-cooperative refine for long drivers ----------------
             unsigned cm = __ballot_sync(kFull, coop);
             while (cm) {

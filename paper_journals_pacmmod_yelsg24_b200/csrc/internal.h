@@ -29,6 +29,7 @@ struct Plan {
     uint32_t seed_lo;       // C(phi[0]) = bucket[seed_lo, seed_lo + seed_len)
     uint32_t seed_len;
     PlanStep step[kMaxQV];
+    uint32_t qadj[kMaxQV];  // bit j: (phi[j], phi[d]) is a query edge, any j != d
 };
 
 // Device-resident data graph, relaid out for the sampler:

@@ -15,12 +15,24 @@ ap.add_argument("--samples", type=float, default=1e7)
 ap.add_argument("--config", default="C1")
 ap.add_argument("--query", type=int, default=1)
 ap.add_argument("--l2", type=int, default=0)
+ap.add_argument("--coop", type=int, default=-1)
+ap.add_argument("--threads", type=int, default=0)
+ap.add_argument("--chunk", type=int, default=0)
+ap.add_argument("--bps", type=int, default=0)
 args = ap.parse_args()
 
 g, qs = gen.CONFIGS[args.config]()
 q = qs[args.query]
 with G.Context(0) as ctx:
     ctx.set_option(G.OPT_L2_PERSIST, args.l2)
+    if args.coop >= 0:
+        ctx.set_option(G.OPT_COOP_THRESHOLD, args.coop)
+    if args.threads:
+        ctx.set_option(G.OPT_THREADS, args.threads)
+    if args.chunk:
+        ctx.set_option(G.OPT_CHUNK, args.chunk)
+    if args.bps:
+        ctx.set_option(G.OPT_BLOCKS_PER_SM, args.bps)
     ctx.load_graph_obj(g)
     ctx.load_query_obj(q)
     for m in (G.WJ, G.ALLEY):

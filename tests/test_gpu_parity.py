@@ -127,7 +127,7 @@ def test_coop_threshold_invariance(ctx, G, coop):
     try:
         _parity(ctx, G, g, q, G.ALLEY, seed=4, first=0, count=20_000)
     finally:
-        ctx.set_option(G.OPT_COOP_THRESHOLD, 32)
+        ctx.set_option(G.OPT_COOP_THRESHOLD, 64)
 
 
 def test_edge_cases(ctx, G):
