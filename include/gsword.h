@@ -99,7 +99,9 @@ typedef enum {
     GSWORD_OPT_THREADS = 1,        /* threads per CTA (multiple of 32, 64..256)       */
     GSWORD_OPT_CHUNK = 2,          /* sample ids a warp takes from the queue at once  */
     GSWORD_OPT_L2_PERSIST = 3,     /* 1 = L2 access-policy window over the adjacency  */
-    GSWORD_OPT_COOP_THRESHOLD = 4  /* Alley driver length at which a warp cooperates  */
+    GSWORD_OPT_COOP_THRESHOLD = 4, /* Alley |S_p| above which the warp refines it in   */
+                                   /* 32-element chunks (0..64; below: task pool)     */
+    GSWORD_OPT_BLOOM = 5           /* 1 = edge Bloom pre-test before exact searches   */
 } gsword_option;
 
 /* ---- context -------------------------------------------------------------------- */

@@ -187,6 +187,8 @@ struct gsword_ctx {
     int32_t* d_col = nullptr;
     uint32_t* d_seg = nullptr;
     int32_t* d_bucket = nullptr;
+    unsigned long long* d_bloom = nullptr;
+    uint64_t bloom_words = 0;
     int64_t n = 0, nnz = 0;
     int32_t n_labels = 1;
     std::vector<int64_t> label_off;
@@ -205,6 +207,7 @@ struct gsword_ctx {
     int opt_chunk = 256;
     int opt_l2 = 0;
     int opt_coop = 64;
+    int opt_bloom = 1;
     // last launch
     int last_grid = 0, last_threads = 0;
 
@@ -212,6 +215,9 @@ struct gsword_ctx {
         if (d_col) cudaFree(d_col);
         if (d_seg) cudaFree(d_seg);
         if (d_bucket) cudaFree(d_bucket);
+        if (d_bloom) cudaFree(d_bloom);
+        d_bloom = nullptr;
+        bloom_words = 0;
         d_col = nullptr;
         d_seg = nullptr;
         d_bucket = nullptr;
@@ -284,6 +290,8 @@ DeviceGraph device_graph(const gsword_ctx* ctx) {
     g.col = ctx->d_col;
     g.seg = ctx->d_seg;
     g.bucket = ctx->d_bucket;
+    g.bloom = ctx->opt_bloom ? ctx->d_bloom : nullptr;
+    g.bloom_mask = ctx->bloom_words ? ctx->bloom_words - 1 : 0;
     g.n = ctx->n;
     g.nnz = ctx->nnz;
     g.n_labels = ctx->n_labels;
@@ -383,6 +391,9 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
         case GSWORD_OPT_L2_PERSIST:
             ctx->opt_l2 = value ? 1 : 0;
             return apply_l2_window(ctx);
+        case GSWORD_OPT_BLOOM:
+            ctx->opt_bloom = value ? 1 : 0;
+            return GSWORD_OK;
         case GSWORD_OPT_COOP_THRESHOLD:
             if (value < 0 || value > 64) return fail(GSWORD_EINVAL, "coop threshold must be 0..64");
             ctx->opt_coop = (int)value;
@@ -461,6 +472,25 @@ int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const 
     } else if (n > 0) {
         CUDA_TRY(gsword::launch_build_bucket_identity(ctx->d_bucket, n, ctx->stream));
         CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    }
+    // blocked Bloom filter over the edge set: ~16 bits per undirected edge, power-of-two words
+    {
+        const uint64_t want = std::max<uint64_t>(1, (uint64_t)(nnz / 2) * 16 / 64);
+        uint64_t words = 1;
+        while (words < want) words <<= 1;
+        int64_t* d_rp = nullptr;
+        if ((e = cudaMalloc(&ctx->d_bloom, words * sizeof(unsigned long long))) != cudaSuccess ||
+            (e = cudaMalloc(&d_rp, sizeof(int64_t) * (size_t)(n + 1))) != cudaSuccess) {
+            if (d_rp) cudaFree(d_rp);
+            ctx->free_graph();
+            return fail(GSWORD_ENOMEM, "load_graph: cudaMalloc(bloom): %s", cudaGetErrorString(e));
+        }
+        ctx->bloom_words = words;
+        CUDA_TRY(cudaMemsetAsync(ctx->d_bloom, 0, words * sizeof(unsigned long long), ctx->stream));
+        CUDA_TRY(cudaMemcpyAsync(d_rp, row_ptr, sizeof(int64_t) * (size_t)(n + 1), cudaMemcpyHostToDevice, ctx->stream));
+        CUDA_TRY(gsword::launch_build_bloom(d_rp, ctx->d_col, n, ctx->d_bloom, words - 1, ctx->stream));
+        CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+        cudaFree(d_rp);
     }
     ctx->n = n;
     ctx->nnz = nnz;

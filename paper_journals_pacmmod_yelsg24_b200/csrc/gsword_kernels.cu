@@ -148,14 +148,24 @@ __device__ __forceinline__ void segment(const DeviceGraph& g, uint32_t v, int32_
     *b = ldg_u32(g.seg + i + 1);
 }
 
+// Edge-existence pre-test: false means "certainly not an edge" (no false negatives).
+__device__ __forceinline__ bool maybe_edge(const DeviceGraph& g, uint32_t a, uint32_t b) {
+    if (!g.bloom) return true;
+    const uint64_t h = edge_hash(a, b);
+    const uint64_t m = bloom_bits(h);
+    return (__ldg(g.bloom + (h & g.bloom_mask)) & m) == m;
+}
+
 // Is x in every N_l(M[j]) for j in `mask`?  M column `col_of` in shared memory.
 __device__ __forceinline__ bool member_all(const DeviceGraph& g, const uint32_t* Ms, int stride, int col_of,
                                            uint32_t mask, int32_t l, int32_t x) {
     while (mask) {
         const int j = __ffs(mask) - 1;
         mask &= mask - 1;
+        const uint32_t mj = Ms[j * stride + col_of];
+        if (!maybe_edge(g, mj, (uint32_t)x)) return false;
         uint32_t a, b;
-        segment(g, Ms[j * stride + col_of], l, &a, &b);
+        segment(g, mj, l, &a, &b);
         if (!in_run(g.col, a, b, x)) return false;
     }
     return true;
@@ -302,6 +312,11 @@ __global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const 
                             const int j = __ffs(bm) - 1;
                             bm &= bm - 1;
                             const uint32_t mj = Ms[j * T + tid];
+                            if (MODE == kModeCount && g.bloom) sectors += 1.0;
+                            if (!maybe_edge(g, mj, (uint32_t)v)) {
+                                reject = true;
+                                break;
+                            }
                             uint32_t a, b, a2, b2;
                             segment(g, mj, ps.label, &a, &b);
                             segment(g, (uint32_t)v, plan_s[j].label, &a2, &b2);
@@ -385,22 +400,31 @@ __global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const 
                         const int j = (int)fns32(omask, k);
                         const uint32_t key = Ms[j * T + ocol];
                         const uint32_t mp = Ms[op * T + ocol];
-                        uint32_t a, b;
-                        segment(g, key, plan_s[op].label, &a, &b);
-                        const bool adj = (b - a < olen) ? in_run(g.col, a, b, (int32_t)mp)
-                                                        : in_run(g.col, olo, olo + olen, (int32_t)key);
-                        if (adj) atomicOr(&res_s[ocol], 1u << j);
-                        if (MODE == kModeCount) sectors += 1.0 + (double)bs_sectors(min(b - a, olen));
+                        if (MODE == kModeCount && g.bloom) sectors += 1.0;
+                        if (maybe_edge(g, key, mp)) {
+                            uint32_t a, b;
+                            segment(g, key, plan_s[op].label, &a, &b);
+                            const bool adj = (b - a < olen) ? in_run(g.col, a, b, (int32_t)mp)
+                                                            : in_run(g.col, olo, olo + olen, (int32_t)key);
+                            if (adj) atomicOr(&res_s[ocol], 1u << j);
+                            if (MODE == kModeCount) sectors += 1.0 + (double)bs_sectors(min(b - a, olen));
+                        }
                     } else {
                         // is S_p[i] in N_l(M[j])?
                         const uint32_t nth = k / olen;
                         const uint32_t i = k - nth * olen;
                         const int j = (int)fns32(omask, nth);
                         const int32_t x = ldg_i32(g.col + olo + i);
-                        uint32_t a, b;
-                        segment(g, Ms[j * T + ocol], olab, &a, &b);
-                        if (!in_run(g.col, a, b, x)) atomicOr(i < 32 ? &rmlo_s[ocol] : &rmhi_s[ocol], 1u << (i & 31));
-                        if (MODE == kModeCount) sectors += (double)bs_sectors(b - a);
+                        const uint32_t mj = Ms[j * T + ocol];
+                        bool member = maybe_edge(g, mj, (uint32_t)x);
+                        if (MODE == kModeCount && g.bloom) sectors += 1.0;
+                        if (member) {
+                            uint32_t a, b;
+                            segment(g, mj, olab, &a, &b);
+                            member = in_run(g.col, a, b, x);
+                            if (MODE == kModeCount) sectors += 1.0 + (double)bs_sectors(b - a);
+                        }
+                        if (!member) atomicOr(i < 32 ? &rmlo_s[ocol] : &rmhi_s[ocol], 1u << (i & 31));
                     }
                 }
             }
@@ -636,6 +660,19 @@ __global__ void iota_kernel(int32_t* out, int64_t n) {
         out[i] = (int32_t)i;
 }
 
+// One thread per vertex v: set the filter bits of every edge {v, w} with w > v.
+__global__ void bloom_kernel(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col, int64_t n,
+                             unsigned long long* __restrict__ bloom, uint64_t mask) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        for (int64_t i = row_ptr[v]; i < row_ptr[v + 1]; ++i) {
+            const int32_t w = col[i];
+            if (w <= v) continue;
+            const uint64_t h = edge_hash((uint32_t)v, (uint32_t)w);
+            atomicOr(bloom + (h & mask), (unsigned long long)bloom_bits(h));
+        }
+    }
+}
+
 template <int METHOD, int MODE>
 const void* kernel_ptr() {
     return reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE>);
@@ -679,6 +716,12 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
 cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_out4, double* d_sectors,
                           cudaStream_t stream) {
     reduce_kernel<<<1, 32, 0, stream>>>(d_partials, n_partials, d_out4, d_sectors);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* bloom,
+                               uint64_t mask, cudaStream_t stream) {
+    bloom_kernel<<<148 * 8, 256, 0, stream>>>(d_row_ptr, col, n, bloom, mask);
     return cudaGetLastError();
 }
 

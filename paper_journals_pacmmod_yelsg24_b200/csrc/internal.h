@@ -36,14 +36,33 @@ struct Plan {
 //   col[ seg[v*nL + l] .. seg[v*nL + l + 1] )  = N_l(v), ascending id
 //   seg has n*nL + 1 entries; for nL == 1 it is exactly row_ptr (as u32)
 //   bucket[ label_off[l] .. label_off[l+1] ) = {v : L(v) = l}, ascending id
+//   bloom: blocked Bloom filter over the undirected edge set (one 64-bit word per
+//   test, 3 bits, ~16 bits per edge): "no" is exact, "maybe" falls back to the
+//   binary search.  NULL = disabled.
 struct DeviceGraph {
     const int32_t* col;
     const uint32_t* seg;
     const int32_t* bucket;
+    const unsigned long long* bloom;
+    uint64_t bloom_mask;  // words - 1 (words is a power of two)
     int64_t n;
     int64_t nnz;
     int32_t n_labels;
 };
+
+// 64-bit mix of an undirected edge {a, b} (splitmix64 finaliser); shared by the
+// host-side filter build and the device-side test.
+__host__ __device__ inline uint64_t edge_hash(uint32_t a, uint32_t b) {
+    const uint64_t key = a < b ? (((uint64_t)a << 32) | b) : (((uint64_t)b << 32) | a);
+    uint64_t z = key + 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+__host__ __device__ inline uint64_t bloom_bits(uint64_t h) {
+    return (1ull << ((h >> 40) & 63)) | (1ull << ((h >> 46) & 63)) | (1ull << ((h >> 52) & 63));
+}
 
 // Launch parameters of one estimate.
 struct LaunchCfg {
@@ -70,6 +89,8 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
 cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_out4, double* d_sectors,
                           cudaStream_t stream);
 cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream);
+cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* bloom,
+                               uint64_t mask, cudaStream_t stream);
 int max_blocks_per_sm(int method, int mode, int threads, size_t* smem_bytes);
 
 enum Mode { kModeEstimate = 0, kModeTrace = 1, kModeCount = 2 };

@@ -130,6 +130,20 @@ def test_coop_threshold_invariance(ctx, G, coop):
         ctx.set_option(G.OPT_COOP_THRESHOLD, 64)
 
 
+@pytest.mark.parametrize("bloom", [0, 1])
+def test_bloom_invariance(ctx, G, bloom):
+    """The edge Bloom pre-test only skips searches that would fail: identical samples."""
+    g = gen.chung_lu(5000, 150_000, gamma=2.1, max_over_mean=60.0, seed=11)
+    ctx.set_option(G.OPT_BLOOM, bloom)
+    try:
+        for dense, qs in ((True, 12), (False, 13)):
+            q = gen.extract_query(g, 7, seed=qs, dense=dense)
+            for m in (0, 1):
+                _parity(ctx, G, g, q, m, seed=6, first=0, count=20_000)
+    finally:
+        ctx.set_option(G.OPT_BLOOM, 1)
+
+
 def test_edge_cases(ctx, G):
     g = gen.random_small_graph(30, 0.3, 3, seed=9)
     ctx.load_graph_obj(g)
@@ -227,7 +241,7 @@ def test_scheduling_invariance(ctx, G, c0):
     base = {m: ctx.estimate(m, 400_000, 9) for m in (0, 1)}
     try:
         for opt, val in ((G.OPT_CHUNK, 1), (G.OPT_CHUNK, 4096), (G.OPT_BLOCKS_PER_SM, 1),
-                         (G.OPT_THREADS, 64), (G.OPT_L2_PERSIST, 1)):
+                         (G.OPT_THREADS, 64), (G.OPT_L2_PERSIST, 1), (G.OPT_BLOOM, 0)):
             ctx.set_option(opt, val)
             for m in (0, 1):
                 r = ctx.estimate(m, 400_000, 9)
@@ -239,6 +253,7 @@ def test_scheduling_invariance(ctx, G, c0):
         ctx.set_option(G.OPT_BLOCKS_PER_SM, 0)
         ctx.set_option(G.OPT_THREADS, 256)
         ctx.set_option(G.OPT_L2_PERSIST, 0)
+        ctx.set_option(G.OPT_BLOOM, 1)
 
 
 def test_async_matches_sync_on_torch_stream(ctx, G, c0):
