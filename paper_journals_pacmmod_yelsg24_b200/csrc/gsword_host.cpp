@@ -189,6 +189,8 @@ struct gsword_ctx {
     int32_t* d_bucket = nullptr;
     unsigned long long* d_bloom = nullptr;
     uint64_t bloom_words = 0;
+    unsigned long long* d_eset = nullptr;
+    uint64_t eset_buckets = 0;
     int64_t n = 0, nnz = 0;
     int32_t n_labels = 1;
     std::vector<int64_t> label_off;
@@ -208,6 +210,7 @@ struct gsword_ctx {
     int opt_l2 = 0;
     int opt_coop = 64;
     int opt_bloom = 1;
+    int opt_eset = 1;
     // last launch
     int last_grid = 0, last_threads = 0;
 
@@ -216,8 +219,11 @@ struct gsword_ctx {
         if (d_seg) cudaFree(d_seg);
         if (d_bucket) cudaFree(d_bucket);
         if (d_bloom) cudaFree(d_bloom);
+        if (d_eset) cudaFree(d_eset);
         d_bloom = nullptr;
         bloom_words = 0;
+        d_eset = nullptr;
+        eset_buckets = 0;
         d_col = nullptr;
         d_seg = nullptr;
         d_bucket = nullptr;
@@ -292,6 +298,8 @@ DeviceGraph device_graph(const gsword_ctx* ctx) {
     g.bucket = ctx->d_bucket;
     g.bloom = ctx->opt_bloom ? ctx->d_bloom : nullptr;
     g.bloom_mask = ctx->bloom_words ? ctx->bloom_words - 1 : 0;
+    g.eset = ctx->opt_eset ? ctx->d_eset : nullptr;
+    g.eset_mask = ctx->eset_buckets ? ctx->eset_buckets - 1 : 0;
     g.n = ctx->n;
     g.nnz = ctx->nnz;
     g.n_labels = ctx->n_labels;
@@ -394,6 +402,9 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
         case GSWORD_OPT_BLOOM:
             ctx->opt_bloom = value ? 1 : 0;
             return GSWORD_OK;
+        case GSWORD_OPT_EDGE_SET:
+            ctx->opt_eset = value ? 1 : 0;
+            return GSWORD_OK;
         case GSWORD_OPT_COOP_THRESHOLD:
             if (value < 0 || value > 64) return fail(GSWORD_EINVAL, "coop threshold must be 0..64");
             ctx->opt_coop = (int)value;
@@ -478,17 +489,25 @@ int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const 
         const uint64_t want = std::max<uint64_t>(1, (uint64_t)(nnz / 2) * 16 / 64);
         uint64_t words = 1;
         while (words < want) words <<= 1;
+        // exact edge set: 4-key buckets, load factor <= 1/2
+        const uint64_t want_b = std::max<uint64_t>(1, ((uint64_t)(nnz / 2) + 1) / 2);
+        uint64_t buckets = 1;
+        while (buckets < want_b) buckets <<= 1;
         int64_t* d_rp = nullptr;
         if ((e = cudaMalloc(&ctx->d_bloom, words * sizeof(unsigned long long))) != cudaSuccess ||
+            (e = cudaMalloc(&ctx->d_eset, buckets * 4 * sizeof(unsigned long long))) != cudaSuccess ||
             (e = cudaMalloc(&d_rp, sizeof(int64_t) * (size_t)(n + 1))) != cudaSuccess) {
             if (d_rp) cudaFree(d_rp);
             ctx->free_graph();
-            return fail(GSWORD_ENOMEM, "load_graph: cudaMalloc(bloom): %s", cudaGetErrorString(e));
+            return fail(GSWORD_ENOMEM, "load_graph: cudaMalloc(edge index): %s", cudaGetErrorString(e));
         }
         ctx->bloom_words = words;
+        ctx->eset_buckets = buckets;
         CUDA_TRY(cudaMemsetAsync(ctx->d_bloom, 0, words * sizeof(unsigned long long), ctx->stream));
+        CUDA_TRY(cudaMemsetAsync(ctx->d_eset, 0xFF, buckets * 4 * sizeof(unsigned long long), ctx->stream));
         CUDA_TRY(cudaMemcpyAsync(d_rp, row_ptr, sizeof(int64_t) * (size_t)(n + 1), cudaMemcpyHostToDevice, ctx->stream));
         CUDA_TRY(gsword::launch_build_bloom(d_rp, ctx->d_col, n, ctx->d_bloom, words - 1, ctx->stream));
+        CUDA_TRY(gsword::launch_build_eset(d_rp, ctx->d_col, n, ctx->d_eset, buckets - 1, ctx->stream));
         CUDA_TRY(cudaStreamSynchronize(ctx->stream));
         cudaFree(d_rp);
     }

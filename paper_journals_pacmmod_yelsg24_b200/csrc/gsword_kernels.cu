@@ -148,25 +148,43 @@ __device__ __forceinline__ void segment(const DeviceGraph& g, uint32_t v, int32_
     *b = ldg_u32(g.seg + i + 1);
 }
 
-// Edge-existence pre-test: false means "certainly not an edge" (no false negatives).
-__device__ __forceinline__ bool maybe_edge(const DeviceGraph& g, uint32_t a, uint32_t b) {
-    if (!g.bloom) return true;
+// Is {a, b} an edge of G?  Exact.  (1) blocked Bloom filter (L2-resident): "no" is
+// final; (2) exact edge set (one 32-byte bucket per probe); without the edge set, a
+// binary search of b in N_lb(a) (lb = L(b)).  `sec` accumulates the sectors touched.
+template <bool COUNT>
+__device__ __forceinline__ bool is_edge(const DeviceGraph& g, uint32_t a, uint32_t b, int32_t lb, double& sec) {
     const uint64_t h = edge_hash(a, b);
-    const uint64_t m = bloom_bits(h);
-    return (__ldg(g.bloom + (h & g.bloom_mask)) & m) == m;
+    if (g.bloom) {
+        if (COUNT) sec += 1.0;
+        const uint64_t m = bloom_bits(h);
+        if ((__ldg(g.bloom + (h & g.bloom_mask)) & m) != m) return false;
+    }
+    if (g.eset) {
+        const unsigned long long key = edge_key(a, b);
+        uint64_t bk = h & g.eset_mask;
+        while (true) {
+            if (COUNT) sec += 1.0;
+            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(g.eset + 4 * bk);
+            const ulonglong2 x0 = __ldg(p), x1 = __ldg(p + 1);
+            if (x0.x == key || x0.y == key || x1.x == key || x1.y == key) return true;
+            if (x0.x == kEmptyKey || x0.y == kEmptyKey || x1.x == kEmptyKey || x1.y == kEmptyKey) return false;
+            bk = (bk + 1) & g.eset_mask;
+        }
+    }
+    uint32_t lo, hi;
+    segment(g, a, lb, &lo, &hi);
+    if (COUNT) sec += 1.0 + (double)bs_sectors(hi - lo);
+    return in_run(g.col, lo, hi, (int32_t)b);
 }
 
 // Is x in every N_l(M[j]) for j in `mask`?  M column `col_of` in shared memory.
+template <bool COUNT>
 __device__ __forceinline__ bool member_all(const DeviceGraph& g, const uint32_t* Ms, int stride, int col_of,
-                                           uint32_t mask, int32_t l, int32_t x) {
+                                           uint32_t mask, int32_t l, int32_t x, double& sec) {
     while (mask) {
         const int j = __ffs(mask) - 1;
         mask &= mask - 1;
-        const uint32_t mj = Ms[j * stride + col_of];
-        if (!maybe_edge(g, mj, (uint32_t)x)) return false;
-        uint32_t a, b;
-        segment(g, mj, l, &a, &b);
-        if (!in_run(g.col, a, b, x)) return false;
+        if (!is_edge<COUNT>(g, Ms[j * stride + col_of], (uint32_t)x, l, sec)) return false;
     }
     return true;
 }
@@ -311,18 +329,7 @@ __global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const 
                         while (bm && !reject) {
                             const int j = __ffs(bm) - 1;
                             bm &= bm - 1;
-                            const uint32_t mj = Ms[j * T + tid];
-                            if (MODE == kModeCount && g.bloom) sectors += 1.0;
-                            if (!maybe_edge(g, mj, (uint32_t)v)) {
-                                reject = true;
-                                break;
-                            }
-                            uint32_t a, b, a2, b2;
-                            segment(g, mj, ps.label, &a, &b);
-                            segment(g, (uint32_t)v, plan_s[j].label, &a2, &b2);
-                            if (b2 - a2 < b - a) reject = !in_run(g.col, a2, b2, (int32_t)mj);
-                            else reject = !in_run(g.col, a, b, v);
-                            if (MODE == kModeCount) sectors += 1.0 + (double)bs_sectors(min(b - a, b2 - a2));
+                            reject = !is_edge<MODE == kModeCount>(g, Ms[j * T + tid], (uint32_t)v, ps.label, sectors);
                         }
                     }
                 }
@@ -398,33 +405,18 @@ __global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const 
                         // is M[j] adjacent to M[p]?  search the shorter of N_l(M[p]) = S_p and
                         // N_{L(phi[p])}(M[j])
                         const int j = (int)fns32(omask, k);
-                        const uint32_t key = Ms[j * T + ocol];
-                        const uint32_t mp = Ms[op * T + ocol];
-                        if (MODE == kModeCount && g.bloom) sectors += 1.0;
-                        if (maybe_edge(g, key, mp)) {
-                            uint32_t a, b;
-                            segment(g, key, plan_s[op].label, &a, &b);
-                            const bool adj = (b - a < olen) ? in_run(g.col, a, b, (int32_t)mp)
-                                                            : in_run(g.col, olo, olo + olen, (int32_t)key);
-                            if (adj) atomicOr(&res_s[ocol], 1u << j);
-                            if (MODE == kModeCount) sectors += 1.0 + (double)bs_sectors(min(b - a, olen));
-                        }
+                        // M[j] has the owner's label l_d: M[j] in S_p  <=>  {M[p], M[j]} is an edge
+                        if (is_edge<MODE == kModeCount>(g, Ms[op * T + ocol], Ms[j * T + ocol], olab, sectors))
+                            atomicOr(&res_s[ocol], 1u << j);
                     } else {
                         // is S_p[i] in N_l(M[j])?
                         const uint32_t nth = k / olen;
                         const uint32_t i = k - nth * olen;
                         const int j = (int)fns32(omask, nth);
                         const int32_t x = ldg_i32(g.col + olo + i);
-                        const uint32_t mj = Ms[j * T + ocol];
-                        bool member = maybe_edge(g, mj, (uint32_t)x);
-                        if (MODE == kModeCount && g.bloom) sectors += 1.0;
-                        if (member) {
-                            uint32_t a, b;
-                            segment(g, mj, olab, &a, &b);
-                            member = in_run(g.col, a, b, x);
-                            if (MODE == kModeCount) sectors += 1.0 + (double)bs_sectors(b - a);
-                        }
-                        if (!member) atomicOr(i < 32 ? &rmlo_s[ocol] : &rmhi_s[ocol], 1u << (i & 31));
+                        // x has label l_d: x in N_l(M[j])  <=>  {M[j], x} is an edge
+                        if (!is_edge<MODE == kModeCount>(g, Ms[j * T + ocol], (uint32_t)x, olab, sectors))
+                            atomicOr(i < 32 ? &rmlo_s[ocol] : &rmhi_s[ocol], 1u << (i & 31));
                     }
                 }
             }
@@ -489,7 +481,7 @@ __global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const 
                     int32_t x = 0;
                     if (keep) {
                         x = ldg_i32(g.col + Llo + i);
-                        keep = member_all(g, Ms, T, colL, others, Lps.label, x) &&
+                        keep = member_all<MODE == kModeCount>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
                                not_matched(Ms, T, colL, Lps.dup, x);
                     }
                     const unsigned bal = __ballot_sync(kFull, keep);
@@ -524,7 +516,7 @@ __global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const 
                             int32_t x = 0;
                             if (keep) {
                                 x = ldg_i32(g.col + Llo + i);
-                                keep = member_all(g, Ms, T, colL, others, Lps.label, x) &&
+                                keep = member_all<MODE == kModeCount>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
                                        not_matched(Ms, T, colL, Lps.dup, x);
                             }
                             const unsigned bal = __ballot_sync(kFull, keep);
@@ -540,18 +532,7 @@ __global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const 
                 if (lane == L) {
                     cnt = total;
                     v = chosen;
-                    if (MODE == kModeCount) {
-                        double s = (double)scan_sectors(Llen);
-                        uint32_t om = others;
-                        while (om) {
-                            const int j = __ffs(om) - 1;
-                            om &= om - 1;
-                            uint32_t a, b;
-                            segment(g, Ms[j * T + colL], Lps.label, &a, &b);
-                            s += (double)min(Llen * bs_sectors(b - a), scan_sectors(b - a));
-                        }
-                        sectors += s;
-                    }
+                    if (MODE == kModeCount) sectors += (double)scan_sectors(Llen);  // driver chunks
                 }
             }
         }
@@ -660,6 +641,27 @@ __global__ void iota_kernel(int32_t* out, int64_t n) {
         out[i] = (int32_t)i;
 }
 
+// One thread per vertex v: insert every edge {v, w}, w > v, into the edge set.
+__global__ void eset_kernel(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col, int64_t n,
+                            unsigned long long* __restrict__ keys, uint64_t mask) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        for (int64_t i = row_ptr[v]; i < row_ptr[v + 1]; ++i) {
+            const int32_t w = col[i];
+            if (w <= v) continue;
+            const unsigned long long key = edge_key((uint32_t)v, (uint32_t)w);
+            uint64_t bk = edge_hash((uint32_t)v, (uint32_t)w) & mask;
+            bool done = false;
+            while (!done) {
+                for (int s = 0; s < 4 && !done; ++s) {
+                    const unsigned long long prev = atomicCAS(keys + 4 * bk + s, kEmptyKey, key);
+                    done = (prev == kEmptyKey) || (prev == key);
+                }
+                bk = (bk + 1) & mask;
+            }
+        }
+    }
+}
+
 // One thread per vertex v: set the filter bits of every edge {v, w} with w > v.
 __global__ void bloom_kernel(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col, int64_t n,
                              unsigned long long* __restrict__ bloom, uint64_t mask) {
@@ -722,6 +724,12 @@ cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_o
 cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* bloom,
                                uint64_t mask, cudaStream_t stream) {
     bloom_kernel<<<148 * 8, 256, 0, stream>>>(d_row_ptr, col, n, bloom, mask);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_build_eset(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* keys,
+                              uint64_t mask, cudaStream_t stream) {
+    eset_kernel<<<148 * 8, 256, 0, stream>>>(d_row_ptr, col, n, keys, mask);
     return cudaGetLastError();
 }
 

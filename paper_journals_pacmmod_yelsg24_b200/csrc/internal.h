@@ -45,16 +45,23 @@ struct DeviceGraph {
     const int32_t* bucket;
     const unsigned long long* bloom;
     uint64_t bloom_mask;  // words - 1 (words is a power of two)
+    // exact edge set: open addressing, 32-byte buckets of 4 keys (min<<32 | max),
+    // linear probing over buckets, load <= 1/2.  NULL = use binary search instead.
+    const unsigned long long* eset;
+    uint64_t eset_mask;   // buckets - 1
     int64_t n;
     int64_t nnz;
     int32_t n_labels;
 };
 
+__host__ __device__ inline uint64_t edge_key(uint32_t a, uint32_t b) {
+    return a < b ? (((uint64_t)a << 32) | b) : (((uint64_t)b << 32) | a);
+}
+
 // 64-bit mix of an undirected edge {a, b} (splitmix64 finaliser); shared by the
 // host-side filter build and the device-side test.
 __host__ __device__ inline uint64_t edge_hash(uint32_t a, uint32_t b) {
-    const uint64_t key = a < b ? (((uint64_t)a << 32) | b) : (((uint64_t)b << 32) | a);
-    uint64_t z = key + 0x9E3779B97F4A7C15ull;
+    uint64_t z = edge_key(a, b) + 0x9E3779B97F4A7C15ull;
     z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
     z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
     return z ^ (z >> 31);
@@ -89,6 +96,9 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
 cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_out4, double* d_sectors,
                           cudaStream_t stream);
 cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream);
+constexpr unsigned long long kEmptyKey = ~0ull;
+cudaError_t launch_build_eset(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* keys,
+                              uint64_t mask, cudaStream_t stream);
 cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* bloom,
                                uint64_t mask, cudaStream_t stream);
 int max_blocks_per_sm(int method, int mode, int threads, size_t* smem_bytes);

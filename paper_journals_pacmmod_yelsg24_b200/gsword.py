@@ -27,6 +27,7 @@ OPT_CHUNK = 2
 OPT_L2_PERSIST = 3
 OPT_COOP_THRESHOLD = 4
 OPT_BLOOM = 5
+OPT_EDGE_SET = 6
 CUDA_STREAM_LEGACY = 0x1  # cudaStreamLegacy
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOGRAPH", -3: "ENOQUERY", -4: "EORDER", -5: "EGRAPH",

@@ -130,11 +130,14 @@ def test_coop_threshold_invariance(ctx, G, coop):
         ctx.set_option(G.OPT_COOP_THRESHOLD, 64)
 
 
-@pytest.mark.parametrize("bloom", [0, 1])
-def test_bloom_invariance(ctx, G, bloom):
-    """The edge Bloom pre-test only skips searches that would fail: identical samples."""
-    g = gen.chung_lu(5000, 150_000, gamma=2.1, max_over_mean=60.0, seed=11)
+@pytest.mark.parametrize("bloom,eset", [(0, 0), (1, 0), (0, 1), (1, 1)])
+def test_edge_index_invariance(ctx, G, bloom, eset):
+    """Bloom pre-test / exact edge set / binary search answer the same adjacency
+    questions: identical samples with every combination."""
+    g = gen.chung_lu(5000, 150_000, gamma=2.1, max_over_mean=60.0, seed=11,
+                     labels=gen.uniform_labels(5000, 2, 12) if bloom != eset else None, n_labels=2 if bloom != eset else 1)
     ctx.set_option(G.OPT_BLOOM, bloom)
+    ctx.set_option(G.OPT_EDGE_SET, eset)
     try:
         for dense, qs in ((True, 12), (False, 13)):
             q = gen.extract_query(g, 7, seed=qs, dense=dense)
@@ -142,6 +145,8 @@ def test_bloom_invariance(ctx, G, bloom):
                 _parity(ctx, G, g, q, m, seed=6, first=0, count=20_000)
     finally:
         ctx.set_option(G.OPT_BLOOM, 1)
+        ctx.set_option(G.OPT_EDGE_SET, 1)
+        ctx.set_option(G.OPT_EDGE_SET, 1)
 
 
 def test_edge_cases(ctx, G):
@@ -241,7 +246,7 @@ def test_scheduling_invariance(ctx, G, c0):
     base = {m: ctx.estimate(m, 400_000, 9) for m in (0, 1)}
     try:
         for opt, val in ((G.OPT_CHUNK, 1), (G.OPT_CHUNK, 4096), (G.OPT_BLOCKS_PER_SM, 1),
-                         (G.OPT_THREADS, 64), (G.OPT_L2_PERSIST, 1), (G.OPT_BLOOM, 0)):
+                         (G.OPT_THREADS, 64), (G.OPT_L2_PERSIST, 1), (G.OPT_BLOOM, 0), (G.OPT_EDGE_SET, 0)):
             ctx.set_option(opt, val)
             for m in (0, 1):
                 r = ctx.estimate(m, 400_000, 9)
@@ -254,6 +259,7 @@ def test_scheduling_invariance(ctx, G, c0):
         ctx.set_option(G.OPT_THREADS, 256)
         ctx.set_option(G.OPT_L2_PERSIST, 0)
         ctx.set_option(G.OPT_BLOOM, 1)
+        ctx.set_option(G.OPT_EDGE_SET, 1)
 
 
 def test_async_matches_sync_on_torch_stream(ctx, G, c0):
