@@ -208,7 +208,7 @@ struct gsword_ctx {
     int opt_threads = 256;
     int opt_chunk = 256;
     int opt_l2 = 0;
-    int opt_coop = 64;
+    int opt_coop = 32;
     int opt_bloom = 1;
     int opt_eset = 1;
     // last launch

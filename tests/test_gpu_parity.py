@@ -127,7 +127,7 @@ def test_coop_threshold_invariance(ctx, G, coop):
     try:
         _parity(ctx, G, g, q, G.ALLEY, seed=4, first=0, count=20_000)
     finally:
-        ctx.set_option(G.OPT_COOP_THRESHOLD, 64)
+        ctx.set_option(G.OPT_COOP_THRESHOLD, 32)
 
 
 @pytest.mark.parametrize("bloom,eset", [(0, 0), (1, 0), (0, 1), (1, 1)])
