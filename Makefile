@@ -6,9 +6,13 @@ PKG      := paper_journals_pacmmod_yelsg24_b200
 CSRC     := $(PKG)/csrc
 LIB      := $(PKG)/libgsword.so
 ORACLE   := oracle/liboracle.so
-NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-O3,-pthread -Xptxas -v --expt-relaxed-constexpr
+XFLAGS   ?=
+NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-O3,-pthread -Xptxas -v --expt-relaxed-constexpr $(XFLAGS)
 
 all: $(LIB) $(ORACLE)
+
+variant:
+	$(NVCC) $(NVFLAGS) -shared -o $(OUT) $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_host.cpp 2> $(OUT).ptxas.log || (cat $(OUT).ptxas.log; false)
 
 $(LIB): $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_host.cpp $(CSRC)/internal.h include/gsword.h
 	$(NVCC) $(NVFLAGS) -shared -o $@ $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_host.cpp 2> build_ptxas.log || (cat build_ptxas.log; false)
@@ -19,4 +23,4 @@ $(ORACLE): oracle/oracle.c
 clean:
 	rm -f $(LIB) $(ORACLE) build_ptxas.log
 
-.PHONY: all clean
+.PHONY: all clean variant

@@ -198,8 +198,16 @@ __device__ __forceinline__ bool not_matched(const uint32_t* Ms, int stride, int 
     return true;
 }
 
+#ifndef GSWORD_WJ_MIN_BLOCKS
+#define GSWORD_WJ_MIN_BLOCKS 6  // 42 registers: 48 warps per SM (measured best)
+#endif
+#ifndef GSWORD_AL_MIN_BLOCKS
+#define GSWORD_AL_MIN_BLOCKS 5  // 51 registers: 40 warps per SM (measured best)
+#endif
+
 template <int METHOD, int MODE>
-__global__ void __launch_bounds__(256) sample_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
+__global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLOCKS : GSWORD_AL_MIN_BLOCKS)
+    sample_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
                                                      const uint64_t count, const uint64_t seed, const int chunk,
                                                      const uint32_t coop_threshold,
                                                      unsigned long long* __restrict__ queue,

@@ -14,7 +14,8 @@ from typing import Dict, Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgsword.so")
+# GSWORD_LIB overrides the library path (build-variant experiments only)
+LIB_PATH = os.environ.get("GSWORD_LIB") or os.path.join(_HERE, "libgsword.so")
 
 WJ = 0
 ALLEY = 1
