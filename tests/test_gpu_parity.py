@@ -238,6 +238,21 @@ def test_c1_full_size_sampled_and_split(ctx, G, c1):
             assert full["sumsq"] == pytest.approx(a["sumsq"] + b["sumsq"], rel=REL)
 
 
+def test_c3_parity_sampled(ctx, G):
+    """BASELINE configs[3] (LiveJournal shape, 16 labels, 12-vertex queries, a 1e10
+    budget): a prefix and two windows deep in the 1e10 id range, every query/method."""
+    g, qs = gen.config_c3()
+    ctx.load_graph_obj(g)
+    for q in qs:
+        for m in (0, 1):
+            _parity(ctx, G, g, q, m, seed=7, first=0, count=10_000, loaded=True, threads=16)
+            for first in (5_000_000_000, 10_000_000_000 - 2000):
+                ctx.load_query_obj(q)
+                rec = ctx.trace_samples(m, first, 2000, 7)
+                _, ref = oracle.sample_range(g, q, m, 7, first, 2000, records=True, threads=16)
+                _records_equal(rec, ref, f"C3/{q.name}/m{m}@{first}")
+
+
 def test_scheduling_invariance(ctx, G, c0):
     g, qs = c0
     ctx.load_graph_obj(g)

@@ -380,10 +380,13 @@ def random_connected_query(nq: int, extra_edge_p: float, n_labels: int, seed: in
     return q.with_order(random_connected_order(q, seed + 7))
 
 
-def extract_query(g: Graph, k: int, seed: int, dense: bool, max_tries: int = 1000) -> Query:
+def extract_query(g: Graph, k: int, seed: int, dense: bool, max_tries: int = 1000,
+                  require_dense: bool = False) -> Query:
     """Random-walk query extraction.
 
-    dense=True : random walk until k distinct vertices, query = induced subgraph.
+    dense=True : random walk until k distinct vertices, query = induced subgraph;
+                 with require_dense, walks are retried until the query's maximum
+                 degree is >= 3 (the paper's dense/sparse split).
     dense=False: self-avoiding walk of k vertices, query = the walk path
                  (max degree 2 < 3, "sparse" per P:L1055).
     Labels are copied from the data vertices, so the count is >= 1.
@@ -429,6 +432,13 @@ def extract_query(g: Graph, k: int, seed: int, dense: bool, max_tries: int = 100
                 for b in range(a + 1, k):
                     if int(vs[b]) in nb:
                         edges.append((a, b))
+            if require_dense:
+                degs = np.zeros(k, np.int64)
+                for a, b in edges:
+                    degs[a] += 1
+                    degs[b] += 1
+                if degs.max() < 3:
+                    continue
         else:
             edges = tree_edges
         labels = g.labels[np.asarray(verts)]
@@ -454,7 +464,7 @@ def config_c0() -> Tuple[Graph, List[Query]]:
 def config_c1() -> Tuple[Graph, List[Query]]:
     """C1: eu2005-shaped Chung-Lu (|V|=862,664, |E|=16,138,468), unlabelled, 8-vertex queries."""
     g = chung_lu(862_664, 16_138_468, gamma=2.1, max_over_mean=68_963 / 37.4, seed=2005, name="C1_eu2005")
-    qs = [extract_query(g, 8, seed=20, dense=False), extract_query(g, 8, seed=21, dense=True)]
+    qs = [extract_query(g, 8, seed=20, dense=False), extract_query(g, 8, seed=21, dense=True, require_dense=True)]
     return g, qs
 
 
@@ -464,7 +474,7 @@ def config_c2() -> Tuple[Graph, List[Query]]:
     lab = skewed_labels(n, (0.60, 0.20, 0.10, 0.06, 0.04), seed=5)
     g = chung_lu(n, 120_399, gamma=2.5, max_over_mean=300.0, seed=76_853, labels=lab, n_labels=5,
                  name="C2_wordnet")
-    qs = [extract_query(g, 8, seed=s, dense=True) for s in (30, 31, 32)]
+    qs = [extract_query(g, 8, seed=s, dense=True, require_dense=True) for s in (30, 31, 32)]
     return g, qs
 
 
@@ -474,7 +484,8 @@ def config_c3() -> Tuple[Graph, List[Query]]:
     lab = uniform_labels(n, 16, seed=16)
     g = chung_lu(n, 42_851_237, gamma=2.4, max_over_mean=20_000 / 17.7, seed=4847, labels=lab, n_labels=16,
                  name="C3_lj")
-    qs = [extract_query(g, 12, seed=s, dense=d) for s, d in ((40, False), (41, False), (42, True), (43, True))]
+    qs = [extract_query(g, 12, seed=s, dense=d, require_dense=d) for s, d in ((40, False), (41, False), (42, True),
+                                                                             (43, True))]
     return g, qs
 
 
