@@ -183,6 +183,12 @@ int gsword_trace_samples(gsword_ctx* ctx, gsword_method m, uint64_t first_sample
 int gsword_count_sectors(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples,
                          uint64_t seed, double* sectors_out);
 
+/* Profiling aid: warp-cycles per loop phase summed over all warps, recorded by the last
+ * gsword_count_sectors run: [0] refill, [1] draw + GetMinCandidate, [2] WanderJoin step /
+ * Alley path selection, [3] Alley task pool, [4] Alley survivor selection, [5] Alley
+ * cooperative refine, [6] epilogue, [7] exit.  out8 receives 8 doubles. */
+int gsword_phase_cycles(gsword_ctx* ctx, double* out8);
+
 /* Device time (CUDA events on the context stream) of the last sampling-kernel launch
  * alone (without the queue reset and the grid reduction).  Waits for that launch. */
 int gsword_last_kernel_seconds(gsword_ctx* ctx, double* seconds);

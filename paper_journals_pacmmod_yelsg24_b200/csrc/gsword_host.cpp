@@ -186,6 +186,8 @@ struct gsword_ctx {
     bool graph_loaded = false;
     int32_t* d_col = nullptr;
     uint32_t* d_seg = nullptr;
+    void* d_hot = nullptr;     // one allocation: [Bloom filter words][seg] (the L2-window target)
+    size_t hot_bytes = 0;
     int32_t* d_bucket = nullptr;
     unsigned long long* d_bloom = nullptr;
     uint64_t bloom_words = 0;
@@ -203,6 +205,8 @@ struct gsword_ctx {
     int partial_cap = 0;
     double* d_out4 = nullptr;
     double* d_sectors = nullptr;
+    unsigned long long* d_phase = nullptr;  // count build: warp cycles per loop phase
+    double h_phase[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     // options
     int opt_blocks_per_sm = 0;
     int opt_threads = 256;
@@ -216,10 +220,11 @@ struct gsword_ctx {
 
     void free_graph() {
         if (d_col) cudaFree(d_col);
-        if (d_seg) cudaFree(d_seg);
+        if (d_hot) cudaFree(d_hot);
         if (d_bucket) cudaFree(d_bucket);
-        if (d_bloom) cudaFree(d_bloom);
         if (d_eset) cudaFree(d_eset);
+        d_hot = nullptr;
+        hot_bytes = 0;
         d_bloom = nullptr;
         bloom_words = 0;
         d_eset = nullptr;
@@ -252,11 +257,13 @@ int apply_l2_window(gsword_ctx* ctx) {
         int max_persist = 0, max_window = 0;
         CUDA_TRY(cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, ctx->device));
         CUDA_TRY(cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, ctx->device));
-        const size_t bytes = (size_t)ctx->nnz * sizeof(int32_t);
+        // mode 1: the adjacency array; mode 2: the hot buffer (Bloom filter + seg)
+        void* base = ctx->opt_l2 == 1 ? (void*)ctx->d_col : ctx->d_hot;
+        const size_t bytes = ctx->opt_l2 == 1 ? (size_t)ctx->nnz * sizeof(int32_t) : ctx->hot_bytes;
         const size_t window = std::min(bytes, (size_t)max_window);
         const size_t persist = std::min((size_t)max_persist, window);
         CUDA_TRY(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, persist));
-        attr.accessPolicyWindow.base_ptr = ctx->d_col;
+        attr.accessPolicyWindow.base_ptr = base;
         attr.accessPolicyWindow.num_bytes = window;
         attr.accessPolicyWindow.hitRatio = window ? (float)std::min(1.0, (double)persist / (double)window) : 0.f;
         attr.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
@@ -312,8 +319,10 @@ int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, u
     int rc = launch_config(ctx, method, mode, &cfg);
     if (rc) return rc;
     CUDA_TRY(cudaEventRecord(ctx->evk0, ctx->stream));
+    if (mode == gsword::kModeCount) CUDA_TRY(cudaMemsetAsync(ctx->d_phase, 0, 8 * sizeof(unsigned long long), ctx->stream));
     cudaError_t e = gsword::launch_sample(method, mode, device_graph(ctx), ctx->plan, cfg, first, count, seed,
-                                          ctx->d_queue, ctx->d_partials, d_records, ctx->stream);
+                                          ctx->d_queue, ctx->d_partials, d_records,
+                                          mode == gsword::kModeCount ? ctx->d_phase : nullptr, ctx->stream);
     if (e != cudaSuccess) return cuda_fail(e, "launch sample kernel");
     CUDA_TRY(cudaEventRecord(ctx->evk1, ctx->stream));
     e = gsword::launch_reduce(ctx->d_partials, cfg.grid, d_out4, d_sectors, ctx->stream);
@@ -348,7 +357,8 @@ int gsword_create(int cuda_device, gsword_ctx** out) {
         (e = cudaEventCreate(&ctx->evk0)) != cudaSuccess || (e = cudaEventCreate(&ctx->evk1)) != cudaSuccess ||
         (e = cudaMalloc(&ctx->d_queue, sizeof(unsigned long long))) != cudaSuccess ||
         (e = cudaMalloc(&ctx->d_out4, 4 * sizeof(double))) != cudaSuccess ||
-        (e = cudaMalloc(&ctx->d_sectors, sizeof(double))) != cudaSuccess) {
+        (e = cudaMalloc(&ctx->d_sectors, sizeof(double))) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_phase, 8 * sizeof(unsigned long long))) != cudaSuccess) {
         gsword_destroy(ctx);
         return cuda_fail(e, "create");
     }
@@ -366,6 +376,7 @@ int gsword_destroy(gsword_ctx* ctx) {
     if (ctx->d_partials) cudaFree(ctx->d_partials);
     if (ctx->d_out4) cudaFree(ctx->d_out4);
     if (ctx->d_sectors) cudaFree(ctx->d_sectors);
+    if (ctx->d_phase) cudaFree(ctx->d_phase);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
     if (ctx->ev1) cudaEventDestroy(ctx->ev1);
     if (ctx->evk0) cudaEventDestroy(ctx->evk0);
@@ -397,7 +408,8 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
             ctx->opt_chunk = (int)value;
             return GSWORD_OK;
         case GSWORD_OPT_L2_PERSIST:
-            ctx->opt_l2 = value ? 1 : 0;
+            if (value < 0 || value > 2) return fail(GSWORD_EINVAL, "l2 window mode must be 0, 1 or 2");
+            ctx->opt_l2 = (int)value;
             return apply_l2_window(ctx);
         case GSWORD_OPT_BLOOM:
             ctx->opt_bloom = value ? 1 : 0;
@@ -468,14 +480,24 @@ int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const 
         std::vector<int64_t> pos(off.begin(), off.end() - 1);
         for (int64_t v = 0; v < n; ++v) bucket[(size_t)pos[(size_t)labels[v]]++] = (int32_t)v;
     }
+    // blocked Bloom filter over the edge set: ~16 bits per undirected edge, power-of-two words
+    uint64_t words = 1;
+    {
+        const uint64_t want = std::max<uint64_t>(1, (uint64_t)(nnz / 2) * 16 / 64);
+        while (words < want) words <<= 1;
+    }
     cudaError_t e;
+    const size_t hot_bytes = words * sizeof(unsigned long long) + sizeof(uint32_t) * seg.size();
     if ((e = cudaMalloc(&ctx->d_col, sizeof(int32_t) * (size_t)std::max<int64_t>(nnz, 1))) != cudaSuccess ||
-        (e = cudaMalloc(&ctx->d_seg, sizeof(uint32_t) * seg.size())) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_hot, hot_bytes)) != cudaSuccess ||
         (e = cudaMalloc(&ctx->d_bucket, sizeof(int32_t) * (size_t)std::max<int64_t>(n, 1))) != cudaSuccess) {
         ctx->free_graph();
         return fail(e == cudaErrorMemoryAllocation ? GSWORD_ENOMEM : GSWORD_ECUDA, "load_graph: cudaMalloc: %s",
                     cudaGetErrorString(e));
     }
+    ctx->hot_bytes = hot_bytes;
+    ctx->d_bloom = reinterpret_cast<unsigned long long*>(ctx->d_hot);
+    ctx->d_seg = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ctx->d_hot) + words * sizeof(unsigned long long));
     if (nnz > 0) CUDA_TRY(cudaMemcpy(ctx->d_col, col_up, sizeof(int32_t) * (size_t)nnz, cudaMemcpyHostToDevice));
     CUDA_TRY(cudaMemcpy(ctx->d_seg, seg.data(), sizeof(uint32_t) * seg.size(), cudaMemcpyHostToDevice));
     if (L > 1) {
@@ -484,18 +506,14 @@ int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const 
         CUDA_TRY(gsword::launch_build_bucket_identity(ctx->d_bucket, n, ctx->stream));
         CUDA_TRY(cudaStreamSynchronize(ctx->stream));
     }
-    // blocked Bloom filter over the edge set: ~16 bits per undirected edge, power-of-two words
+    // Bloom filter (allocated above) and exact edge set, both built on the device
     {
-        const uint64_t want = std::max<uint64_t>(1, (uint64_t)(nnz / 2) * 16 / 64);
-        uint64_t words = 1;
-        while (words < want) words <<= 1;
         // exact edge set: 4-key buckets, load factor <= 1/2
         const uint64_t want_b = std::max<uint64_t>(1, ((uint64_t)(nnz / 2) + 1) / 2);
         uint64_t buckets = 1;
         while (buckets < want_b) buckets <<= 1;
         int64_t* d_rp = nullptr;
-        if ((e = cudaMalloc(&ctx->d_bloom, words * sizeof(unsigned long long))) != cudaSuccess ||
-            (e = cudaMalloc(&ctx->d_eset, buckets * 4 * sizeof(unsigned long long))) != cudaSuccess ||
+        if ((e = cudaMalloc(&ctx->d_eset, buckets * 4 * sizeof(unsigned long long))) != cudaSuccess ||
             (e = cudaMalloc(&d_rp, sizeof(int64_t) * (size_t)(n + 1))) != cudaSuccess) {
             if (d_rp) cudaFree(d_rp);
             ctx->free_graph();
@@ -612,7 +630,16 @@ int gsword_count_sectors(gsword_ctx* ctx, gsword_method m, uint64_t first, uint6
     rc = run(ctx, (int)m, gsword::kModeCount, first, n_samples, seed, ctx->d_out4, nullptr, ctx->d_sectors);
     if (rc) return rc;
     CUDA_TRY(cudaMemcpyAsync(sectors_out, ctx->d_sectors, sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+    unsigned long long ph[8];
+    CUDA_TRY(cudaMemcpyAsync(ph, ctx->d_phase, sizeof(ph), cudaMemcpyDeviceToHost, ctx->stream));
     CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    for (int i = 0; i < 8; ++i) ctx->h_phase[i] = (double)ph[i];
+    return GSWORD_OK;
+}
+
+int gsword_phase_cycles(gsword_ctx* ctx, double* out8) {
+    if (!ctx || !out8) return fail(GSWORD_EINVAL, "phase_cycles: NULL argument");
+    for (int i = 0; i < 8; ++i) out8[i] = ctx->h_phase[i];
     return GSWORD_OK;
 }
 

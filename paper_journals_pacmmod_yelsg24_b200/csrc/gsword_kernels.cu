@@ -212,7 +212,8 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                                                      const uint32_t coop_threshold,
                                                      unsigned long long* __restrict__ queue,
                                                      Partial* __restrict__ partials,
-                                                     gsword_sample_record* __restrict__ records) {
+                                                     gsword_sample_record* __restrict__ records,
+                                                     unsigned long long* __restrict__ phase_out) {
     __shared__ PlanStep plan_s[kMaxQV];
     __shared__ uint32_t qadj_s[kMaxQV];
     __shared__ uint32_t res_s[256];   // Alley task-pool results per lane (adjacent matched vertices)
@@ -248,7 +249,22 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
     uint64_t q_next = 0, q_end = 0;
     bool exhausted = false;
 
+    // count build only: warp-level cycle split of the loop (lane 0 of every warp)
+    unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    long long ph_t = clock64();
+    int ph_cur = 0;
+    auto mark = [&](int next) {
+        if (MODE == kModeCount) {
+            __syncwarp();
+            const long long now = clock64();
+            ph[ph_cur] += (unsigned long long)(now - ph_t);
+            ph_t = now;
+            ph_cur = next;
+        }
+    };
+
     while (true) {
+        mark(0);
         // ---------------- A1: refill free lanes from the sample queue ----------------
         unsigned need = __ballot_sync(kFull, !has);
         while (need && !exhausted) {
@@ -286,11 +302,14 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
         if (!__any_sync(kFull, has)) break;
         __syncwarp();
 
+        mark(1);
         // ---------------- per-lane prologue: draw + GetMinCandidate -----------------
         PlanStep ps = {0, 0u, 0u, 0};
         uint64_t r = 0;
         uint32_t lo_p = 0, len_p = 0;
         int p = -1;
+        uint32_t seg_a = 0, seg_b = 0;
+        bool deferred = false;
         if (has) {
             ps = plan_s[d];
             r = philox_r(seed, sid, (uint32_t)d);
@@ -298,6 +317,13 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 lo_p = plan_in.seed_lo;
                 len_p = plan_in.seed_len;
                 if (MODE == kModeCount) sectors += plan_in.seed_identity ? 0.0 : 1.0;
+            } else if (METHOD == GSWORD_ALLEY && ps.nback == 1) {
+                // one backward neighbour: p is fixed by the plan; the segment load is left
+                // in flight and consumed after the exclusion tests (which need only M)
+                p = __ffs(ps.back) - 1;
+                segment(g, Ms[p * T + tid], ps.label, &seg_a, &seg_b);
+                deferred = true;
+                if (MODE == kModeCount) sectors += 1.0;
             } else {
                 // GetMinCandidate (Alg. 1 l.8): the smallest N_l(M[j]) over j in B(d)
                 uint32_t bm = ps.back;
@@ -317,6 +343,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             }
         }
 
+        mark(2);
         uint32_t cnt = 0;     // |C_d|
         int32_t v = -1;       // drawn vertex
         bool reject = false;  // WJ Validate failure
@@ -348,8 +375,65 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             // kind 2: |B(d)| >= 2, |S_p| <= threshold -> refine bitmask over S_p, membership
             //         tests pooled across the warp
             // kind 3: |B(d)| >= 2, |S_p| > threshold -> warp-cooperative chunks (below)
+            //
+            // Warp task pool: the edge tests of all 32 lanes are dealt out round-robin (an
+            // exclusive scan of per-lane counts, owner found by shuffle bisection), so every
+            // lane is busy whichever lanes generated the work (the refine imbalance).
+            // test(o, k) runs task k of owner lane o; every lane calls it (it shuffles).
+            auto pool = [&](uint32_t ntask, auto&& test) {
+                if (!__any_sync(kFull, ntask != 0u)) return;
+                uint32_t incl = ntask;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(kFull, incl, o);
+                    if (lane >= o) incl += y;
+                }
+                const uint32_t total = __shfl_sync(kFull, incl, 31);
+                const uint32_t excl = incl - ntask;
+                for (uint32_t base = 0; base < total; base += 32) {
+                    const uint32_t t = base + (uint32_t)lane;
+                    const uint32_t tt = t < total ? t : total - 1;
+                    int o = 0;  // owner lane: number of lanes whose inclusive count <= tt
+#pragma unroll
+                    for (int s2 = 16; s2 >= 1; s2 >>= 1) {
+                        const uint32_t y = __shfl_sync(kFull, incl, o + s2 - 1);
+                        if (y <= tt) o += s2;
+                    }
+                    test(o, tt - __shfl_sync(kFull, excl, o), t < total);
+                }
+                __syncwarp();
+            };
             int kind = 0;
             uint32_t unk = 0, known = 0, others = 0;
+            res_s[tid] = 0u;
+            rmlo_s[tid] = 0u;
+            rmhi_s[tid] = 0u;
+            if (has && deferred) {
+                // M[j] (same label) with (phi[j], phi[p]) a query edge lies in S_p by the
+                // Alley invariant (every drawn prefix is a partial instance); M[p] never does
+                // (no self loops); the rest need an edge test {M[p], M[j]}.
+                const uint32_t qa = qadj_s[p];
+                kind = 1;
+                known = ps.dup & qa;
+                unk = ps.dup & ~qa & ~(1u << p);
+            }
+            __syncwarp();
+            // pool 1: exclusion tests, overlapping the in-flight segment loads
+            pool((kind == 1) ? (uint32_t)__popc(unk) : 0u, [&](int o, uint32_t k, bool valid) {
+                const uint32_t omask = __shfl_sync(kFull, unk, o);
+                const int op = __shfl_sync(kFull, p, o);
+                const int32_t olab = __shfl_sync(kFull, ps.label, o);
+                if (valid) {
+                    const int ocol = wbase + o;
+                    const int j = (int)fns32(omask, k);
+                    if (is_edge<MODE == kModeCount>(g, Ms[op * T + ocol], Ms[j * T + ocol], olab, sectors))
+                        atomicOr(&res_s[ocol], 1u << j);
+                }
+            });
+            if (deferred) {
+                lo_p = seg_a;
+                len_p = seg_b - seg_a;
+            }
             if (has) {
                 if (d == 0) {
                     cnt = len_p;
@@ -357,16 +441,10 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                         const uint64_t k = __umul64hi(r, (uint64_t)cnt);
                         v = plan_in.seed_identity ? (int32_t)(lo_p + k) : ldg_i32(g.bucket + lo_p + k);
                     }
-                } else if (len_p > 0) {
-                    if (ps.nback == 1) {
-                        // M[j] (same label) with (phi[j], phi[p]) a query edge lies in S_p by the
-                        // Alley invariant (every drawn prefix is a partial instance); M[p] never
-                        // does (no self loops); the rest need an adjacency test.
-                        const uint32_t qa = qadj_s[p];
-                        kind = 1;
-                        known = ps.dup & qa;
-                        unk = ps.dup & ~qa & ~(1u << p);
-                    } else if (len_p <= coop_threshold) {
+                } else if (len_p == 0) {
+                    kind = 0;
+                } else if (!deferred) {
+                    if (len_p <= coop_threshold) {
                         kind = 2;
                         others = ps.back & ~(1u << p);
                         if (MODE == kModeCount) sectors += (double)scan_sectors(len_p);
@@ -375,60 +453,25 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     }
                 }
             }
-
-            // ---- warp task pool: every lane executes one adjacency test per round ----
-            const uint32_t ntask = (kind == 1) ? (uint32_t)__popc(unk)
-                                 : (kind == 2) ? len_p * (uint32_t)__popc(others) : 0u;
-            res_s[tid] = 0u;
-            rmlo_s[tid] = 0u;
-            rmhi_s[tid] = 0u;
-            uint32_t incl = ntask;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t y = __shfl_up_sync(kFull, incl, o);
-                if (lane >= o) incl += y;
-            }
-            const uint32_t total = __shfl_sync(kFull, incl, 31);
-            const uint32_t excl = incl - ntask;
-            __syncwarp();
-            for (uint32_t base = 0; base < total; base += 32) {
-                const uint32_t t = base + (uint32_t)lane;
-                const uint32_t tt = t < total ? t : total - 1;
-                int o = 0;  // owner lane: number of lanes whose inclusive count <= tt
-#pragma unroll
-                for (int s = 16; s >= 1; s >>= 1) {
-                    const uint32_t y = __shfl_sync(kFull, incl, o + s - 1);
-                    if (y <= tt) o += s;
-                }
-                const uint32_t k = tt - __shfl_sync(kFull, excl, o);
-                const int okind = __shfl_sync(kFull, kind, o);
+            mark(3);
+            // pool 2: membership tests of short refine masks
+            pool((kind == 2) ? len_p * (uint32_t)__popc(others) : 0u, [&](int o, uint32_t k, bool valid) {
+                const uint32_t omask = __shfl_sync(kFull, others, o);
                 const uint32_t olo = __shfl_sync(kFull, lo_p, o);
                 const uint32_t olen = __shfl_sync(kFull, len_p, o);
-                const int op = __shfl_sync(kFull, p, o);
-                const uint32_t omask = __shfl_sync(kFull, (kind == 1) ? unk : others, o);
                 const int32_t olab = __shfl_sync(kFull, ps.label, o);
-                if (t < total) {
+                if (valid) {
                     const int ocol = wbase + o;
-                    if (okind == 1) {
-                        // is M[j] adjacent to M[p]?  search the shorter of N_l(M[p]) = S_p and
-                        // N_{L(phi[p])}(M[j])
-                        const int j = (int)fns32(omask, k);
-                        // M[j] has the owner's label l_d: M[j] in S_p  <=>  {M[p], M[j]} is an edge
-                        if (is_edge<MODE == kModeCount>(g, Ms[op * T + ocol], Ms[j * T + ocol], olab, sectors))
-                            atomicOr(&res_s[ocol], 1u << j);
-                    } else {
-                        // is S_p[i] in N_l(M[j])?
-                        const uint32_t nth = k / olen;
-                        const uint32_t i = k - nth * olen;
-                        const int j = (int)fns32(omask, nth);
-                        const int32_t x = ldg_i32(g.col + olo + i);
-                        // x has label l_d: x in N_l(M[j])  <=>  {M[j], x} is an edge
-                        if (!is_edge<MODE == kModeCount>(g, Ms[j * T + ocol], (uint32_t)x, olab, sectors))
-                            atomicOr(i < 32 ? &rmlo_s[ocol] : &rmhi_s[ocol], 1u << (i & 31));
-                    }
+                    // is S_p[i] (label l_d) in N_l(M[j]), i.e. is {M[j], S_p[i]} an edge?
+                    const uint32_t nth = k / olen;
+                    const uint32_t i = k - nth * olen;
+                    const int j = (int)fns32(omask, nth);
+                    const int32_t x = ldg_i32(g.col + olo + i);
+                    if (!is_edge<MODE == kModeCount>(g, Ms[j * T + ocol], (uint32_t)x, olab, sectors))
+                        atomicOr(i < 32 ? &rmlo_s[ocol] : &rmhi_s[ocol], 1u << (i & 31));
                 }
-            }
-            __syncwarp();
+            });
+            mark(4);
             if (kind == 1) {
                 const uint32_t in_sp = known | res_s[tid];  // matched vertices inside S_p
                 cnt = len_p - __popc(in_sp);
@@ -467,6 +510,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 }
             }
             const bool coop = (kind == 3);
+            mark(5);
 
             // ---------------- warp-cooperative refine for long drivers ----------------
             unsigned cm = __ballot_sync(kFull, coop);
@@ -545,6 +589,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             }
         }
 
+        mark(6);
         // ---------------- common epilogue: HT weight, record, terminate ----------------
         if (has) {
             W = (d == 0) ? (double)cnt : __dmul_rn(W, (double)cnt);
@@ -577,6 +622,12 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 d += 1;
             }
         }
+    }
+
+    mark(7);
+    if (MODE == kModeCount && phase_out && lane == 0) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) atomicAdd(phase_out + i, ph[i]);
     }
 
     // ---------------- A10: warp -> CTA partial, fixed order ----------------
@@ -713,13 +764,15 @@ int max_blocks_per_sm(int method, int mode, int threads, size_t* smem_bytes) {
 
 cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan& plan, const LaunchCfg& cfg,
                           uint64_t first, uint64_t count, uint64_t seed, unsigned long long* d_queue,
-                          Partial* d_partials, gsword_sample_record* d_records, cudaStream_t stream) {
+                          Partial* d_partials, gsword_sample_record* d_records, unsigned long long* d_phase,
+                          cudaStream_t stream) {
     cudaError_t e = cudaMemsetAsync(d_queue, 0, sizeof(unsigned long long), stream);
     if (e != cudaSuccess) return e;
     const size_t smem = (size_t)kMaxQV * (size_t)cfg.threads * sizeof(uint32_t);
     const uint32_t thr = (uint32_t)cfg.coop_threshold;
     void* args[] = {(void*)&g,      (void*)&plan,  (void*)&first,   (void*)&count,     (void*)&seed,
-                    (void*)&cfg.chunk, (void*)&thr, (void*)&d_queue, (void*)&d_partials, (void*)&d_records};
+                    (void*)&cfg.chunk, (void*)&thr, (void*)&d_queue, (void*)&d_partials, (void*)&d_records,
+                    (void*)&d_phase};
     return cudaLaunchKernel(select_kernel(method, mode), dim3(cfg.grid), dim3(cfg.threads), args, smem, stream);
 }
 

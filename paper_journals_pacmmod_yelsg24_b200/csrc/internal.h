@@ -92,7 +92,8 @@ struct Partial {
 // Kernel entry points (gsword_kernels.cu).  All enqueue on `stream`.
 cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan& plan, const LaunchCfg& cfg,
                           uint64_t first, uint64_t count, uint64_t seed, unsigned long long* d_queue,
-                          Partial* d_partials, gsword_sample_record* d_records, cudaStream_t stream);
+                          Partial* d_partials, gsword_sample_record* d_records, unsigned long long* d_phase,
+                          cudaStream_t stream);
 cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_out4, double* d_sectors,
                           cudaStream_t stream);
 cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream);

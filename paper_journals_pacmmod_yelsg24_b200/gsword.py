@@ -81,6 +81,7 @@ def _load_library() -> ctypes.CDLL:
         "gsword_count_sectors": ([P, ctypes.c_int, U64, U64, U64, P], ctypes.c_int),
         "gsword_launch_info": ([P, P, P, P], ctypes.c_int),
         "gsword_last_kernel_seconds": ([P, P], ctypes.c_int),
+        "gsword_phase_cycles": ([P, P], ctypes.c_int),
         "gsword_check_graph": ([I64, P, P, P, I32], ctypes.c_int),
         "gsword_plan_query": ([I32, P, P, P, P, I32, ctypes.POINTER(_PlanInfo)], ctypes.c_int),
         "gsword_last_error": ([], ctypes.c_char_p),
@@ -200,6 +201,11 @@ class Context:
         g, t, l = ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
         _check(_lib.gsword_launch_info(self._h, ctypes.byref(g), ctypes.byref(t), ctypes.byref(l)))
         return {"grid": g.value, "threads": t.value, "launches_per_estimate": l.value}
+
+    def phase_cycles(self) -> list:
+        out = (ctypes.c_double * 8)()
+        _check(_lib.gsword_phase_cycles(self._h, out))
+        return list(out)
 
     def last_kernel_seconds(self) -> float:
         out = ctypes.c_double()

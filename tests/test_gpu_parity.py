@@ -261,7 +261,8 @@ def test_scheduling_invariance(ctx, G, c0):
     base = {m: ctx.estimate(m, 400_000, 9) for m in (0, 1)}
     try:
         for opt, val in ((G.OPT_CHUNK, 1), (G.OPT_CHUNK, 4096), (G.OPT_BLOCKS_PER_SM, 1),
-                         (G.OPT_THREADS, 64), (G.OPT_L2_PERSIST, 1), (G.OPT_BLOOM, 0), (G.OPT_EDGE_SET, 0)):
+                         (G.OPT_THREADS, 64), (G.OPT_L2_PERSIST, 1), (G.OPT_L2_PERSIST, 2), (G.OPT_BLOOM, 0),
+                         (G.OPT_EDGE_SET, 0)):
             ctx.set_option(opt, val)
             for m in (0, 1):
                 r = ctx.estimate(m, 400_000, 9)
