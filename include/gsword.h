@@ -100,7 +100,7 @@ typedef enum {
     GSWORD_OPT_CHUNK = 2,          /* sample ids a warp takes from the queue at once  */
     GSWORD_OPT_L2_PERSIST = 3,     /* 1 = L2 access-policy window over the adjacency  */
     GSWORD_OPT_COOP_THRESHOLD = 4, /* Alley |S_p| above which the warp refines it in   */
-                                   /* 32-element chunks (0..64; below: task pool)     */
+                                   /* 32-element chunks (0..128; below: task pool)    */
     GSWORD_OPT_BLOOM = 5,          /* 1 = edge Bloom pre-test (L2-resident filter)    */
     GSWORD_OPT_EDGE_SET = 6        /* 1 = exact edge hash set for adjacency tests;    */
                                    /* 0 = binary search in the adjacency run          */

@@ -212,7 +212,7 @@ struct gsword_ctx {
     int opt_threads = 256;
     int opt_chunk = 256;
     int opt_l2 = 0;
-    int opt_coop = 32;
+    int opt_coop = 64;
     int opt_bloom = 1;
     int opt_eset = 1;
     // last launch
@@ -418,7 +418,7 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
             ctx->opt_eset = value ? 1 : 0;
             return GSWORD_OK;
         case GSWORD_OPT_COOP_THRESHOLD:
-            if (value < 0 || value > 64) return fail(GSWORD_EINVAL, "coop threshold must be 0..64");
+            if (value < 0 || value > 128) return fail(GSWORD_EINVAL, "coop threshold must be 0..128");
             ctx->opt_coop = (int)value;
             return GSWORD_OK;
         default:

@@ -217,8 +217,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
     __shared__ PlanStep plan_s[kMaxQV];
     __shared__ uint32_t qadj_s[kMaxQV];
     __shared__ uint32_t res_s[256];   // Alley task-pool results per lane (adjacent matched vertices)
-    __shared__ uint32_t rmlo_s[256];  // Alley task-pool results per lane (refine-mask removals)
-    __shared__ uint32_t rmhi_s[256];
+    __shared__ uint32_t rm_s[4][256];  // Alley task-pool results per lane: refine-mask removals (128 bits)
     __shared__ Partial warp_part[32];
     extern __shared__ uint32_t Ms[];  // Ms[j * blockDim.x + tid] = M[j] of this lane
 
@@ -406,8 +405,8 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             int kind = 0;
             uint32_t unk = 0, known = 0, others = 0;
             res_s[tid] = 0u;
-            rmlo_s[tid] = 0u;
-            rmhi_s[tid] = 0u;
+#pragma unroll
+            for (int w = 0; w < 4; ++w) rm_s[w][tid] = 0u;
             if (has && deferred) {
                 // M[j] (same label) with (phi[j], phi[p]) a query edge lies in S_p by the
                 // Alley invariant (every drawn prefix is a partial instance); M[p] never does
@@ -468,7 +467,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     const int j = (int)fns32(omask, nth);
                     const int32_t x = ldg_i32(g.col + olo + i);
                     if (!is_edge<MODE == kModeCount>(g, Ms[j * T + ocol], (uint32_t)x, olab, sectors))
-                        atomicOr(i < 32 ? &rmlo_s[ocol] : &rmhi_s[ocol], 1u << (i & 31));
+                        atomicOr(&rm_s[i >> 5][ocol], 1u << (i & 31));
                 }
             });
             mark(4);
@@ -493,20 +492,35 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     if (MODE == kModeCount) sectors += 1.0;
                 }
             } else if (kind == 2) {
-                uint64_t mask = (len_p >= 64) ? ~0ull : ((1ull << len_p) - 1ull);
-                mask &= ~(((uint64_t)rmhi_s[tid] << 32) | (uint64_t)rmlo_s[tid]);
-                // injectivity: drop survivors equal to a matched same-label vertex
-                uint64_t mm = mask;
+                // refine mask over S_p (<= 128 elements, 4 words): not removed by a membership
+                // test and not a matched same-label vertex (injectivity)
                 const uint32_t dup = ps.dup & ~(1u << p);
-                while (mm && dup) {
-                    const int i = __ffsll((long long)mm) - 1;
-                    mm &= mm - 1;
-                    if (!not_matched(Ms + tid, T, 0, dup, ldg_i32(g.col + lo_p + i))) mask &= ~(1ull << i);
+                uint32_t keep[4];
+                cnt = 0;
+#pragma unroll
+                for (int w = 0; w < 4; ++w) {
+                    const uint32_t n_w = (len_p > 32u * w) ? min(len_p - 32u * w, 32u) : 0u;
+                    uint32_t m = (n_w == 32u) ? 0xFFFFFFFFu : ((1u << n_w) - 1u);
+                    m &= ~rm_s[w][tid];
+                    uint32_t mm = dup ? m : 0u;
+                    while (mm) {
+                        const int i = __ffs(mm) - 1;
+                        mm &= mm - 1;
+                        if (!not_matched(Ms + tid, T, 0, dup, ldg_i32(g.col + lo_p + 32u * w + i))) m &= ~(1u << i);
+                    }
+                    keep[w] = m;
+                    cnt += __popc(m);
                 }
-                cnt = __popcll(mask);
                 if (cnt > 0) {
-                    const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
-                    v = ldg_i32(g.col + lo_p + fns64(mask, k));
+                    uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
+                    uint32_t pos = 0;
+#pragma unroll
+                    for (int w = 0; w < 4; ++w) {
+                        const uint32_t c = __popc(keep[w]);
+                        if (k < c && pos == 0u) pos = 32u * w + fns32(keep[w], k) + 1u;  // +1: found marker
+                        if (pos == 0u) k -= c;
+                    }
+                    v = ldg_i32(g.col + lo_p + pos - 1u);
                 }
             }
             const bool coop = (kind == 3);

@@ -21,7 +21,7 @@ ap.add_argument("--reps", type=int, default=2)
 args = ap.parse_args()
 OPT = {"coop": G.OPT_COOP_THRESHOLD, "threads": G.OPT_THREADS, "chunk": G.OPT_CHUNK, "bps": G.OPT_BLOCKS_PER_SM,
        "l2": G.OPT_L2_PERSIST, "bloom": G.OPT_BLOOM, "eset": G.OPT_EDGE_SET}
-DEF = {"coop": 32, "threads": 256, "chunk": 256, "bps": 0, "l2": 0, "bloom": 1, "eset": 1}
+DEF = {"coop": 64, "threads": 256, "chunk": 256, "bps": 0, "l2": 0, "bloom": 1, "eset": 1}
 grid = json.loads(args.grid)
 g, qs = gen.CONFIGS[args.config]()
 queries = qs if args.query < 0 else [qs[args.query]]

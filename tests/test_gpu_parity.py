@@ -117,7 +117,7 @@ def test_alley_zero_variance_on_gpu(ctx, G):
         assert r["n_valid"] == 20_000 and r["estimate"] == want and abs(r["variance"]) <= G.variance_tolerance(r)
 
 
-@pytest.mark.parametrize("coop", [0, 1, 17, 32, 64])
+@pytest.mark.parametrize("coop", [0, 1, 17, 32, 64, 100, 128])
 def test_coop_threshold_invariance(ctx, G, coop):
     """The warp-cooperative and per-lane refine paths give identical samples."""
     g = gen.chung_lu(3000, 60_000, gamma=2.2, max_over_mean=40.0, seed=5, labels=gen.uniform_labels(3000, 2, 6),
@@ -127,7 +127,7 @@ def test_coop_threshold_invariance(ctx, G, coop):
     try:
         _parity(ctx, G, g, q, G.ALLEY, seed=4, first=0, count=20_000)
     finally:
-        ctx.set_option(G.OPT_COOP_THRESHOLD, 32)
+        ctx.set_option(G.OPT_COOP_THRESHOLD, 64)
 
 
 @pytest.mark.parametrize("bloom,eset", [(0, 0), (1, 0), (0, 1), (1, 1)])
