@@ -1,0 +1,23 @@
+"""Small estimate / trace runs for compute-sanitizer (memcheck, racecheck, synccheck,
+initcheck): both methods, every refine path (coop thresholds 0 and 64), trace mode."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import paper_journals_pacmmod_yelsg24_b200 as G  # noqa: E402
+from workloads import gen  # noqa: E402
+
+g = gen.chung_lu(2000, 30_000, gamma=2.2, max_over_mean=40.0, seed=3, labels=gen.uniform_labels(2000, 2, 4),
+                 n_labels=2)
+q = gen.extract_query(g, 6, seed=5, dense=True, require_dense=True)
+with G.Context(0) as ctx:
+    ctx.load_graph_obj(g)
+    ctx.load_query_obj(q)
+    for coop in (0, 64):
+        ctx.set_option(G.OPT_COOP_THRESHOLD, coop)
+        for m in (G.WJ, G.ALLEY):
+            r = ctx.estimate(m, 20_000, 1)
+            rec = ctx.trace_samples(m, 0, 2000, 1)
+            s = ctx.count_sectors(m, 0, 2000, 1)
+            print(m, coop, r["n_valid"], int(rec["valid"].sum()), s)
