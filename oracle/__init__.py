@@ -67,6 +67,10 @@ def _load():
                                             ctypes.c_int, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64,
                                             P, P]
             lib.or_sample_range.restype = ctypes.c_int
+            lib.or_sample_range_f.argtypes = lib.or_sample_range.argtypes + [ctypes.c_int]
+            lib.or_sample_range_f.restype = ctypes.c_int
+            lib.or_candidate_sets.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, ctypes.c_int, P]
+            lib.or_candidate_sets.restype = ctypes.c_int
             lib.or_count_embeddings.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, P, P]
             lib.or_count_embeddings.restype = ctypes.c_int
             lib.or_record_size.restype = ctypes.c_int
@@ -108,8 +112,25 @@ class _Prepared:
         self.order = np.ascontiguousarray(q.order, np.int32)
 
 
+FILTER_LABEL = 0
+FILTER_LDF = 1
+FILTER_NLF = 2
+
+
+def candidate_sets(g, q, filter: int) -> np.ndarray:
+    """C(u) membership, bool[nq, n] (Def. 4; filter per reading A21)."""
+    lib = _load()
+    pr = _Prepared(g, q)
+    out = np.zeros((pr.nq, pr.n), np.uint8)
+    rc = lib.or_candidate_sets(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq, _ptr(pr.qrp),
+                               _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order), int(filter), _ptr(out))
+    if rc != 0:
+        raise ValueError(f"oracle rejected input (rc={rc})")
+    return out.astype(bool)
+
+
 def sample_range(g, q, method: int, seed: int, first: int, count: int, records: bool = True,
-                 threads: int = 1) -> Tuple[np.ndarray, Optional[np.ndarray]]:
+                 threads: int = 1, filter: int = FILTER_LABEL) -> Tuple[np.ndarray, Optional[np.ndarray]]:
     """Y values (and records) of samples [first, first+count), in sample-id order."""
     lib = _load()
     pr = _Prepared(g, q)
@@ -119,9 +140,9 @@ def sample_range(g, q, method: int, seed: int, first: int, count: int, records: 
     def run(a: int, b: int) -> int:
         yp = ctypes.c_void_p(y.ctypes.data + 8 * a)
         rp = ctypes.c_void_p(rec.ctypes.data + RECORD_DTYPE.itemsize * a) if records else None
-        return lib.or_sample_range(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq,
-                                   _ptr(pr.qrp), _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order),
-                                   int(method), int(seed), int(first + a), int(b - a), yp, rp)
+        return lib.or_sample_range_f(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq,
+                                     _ptr(pr.qrp), _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order),
+                                     int(method), int(seed), int(first + a), int(b - a), yp, rp, int(filter))
 
     if threads <= 1 or count < 2 * threads:
         rc = run(0, count) if count else 0
@@ -151,8 +172,9 @@ def aggregate(y: np.ndarray) -> Dict[str, float]:
     return {"sum": s, "sumsq": sq, "n": n, "n_valid": valid, "estimate": est, "variance": var}
 
 
-def estimate(g, q, method: int, seed: int, n_samples: int, first: int = 0, threads: int = 1) -> Dict[str, float]:
-    y, _ = sample_range(g, q, method, seed, first, n_samples, records=False, threads=threads)
+def estimate(g, q, method: int, seed: int, n_samples: int, first: int = 0, threads: int = 1,
+             filter: int = FILTER_LABEL) -> Dict[str, float]:
+    y, _ = sample_range(g, q, method, seed, first, n_samples, records=False, threads=threads, filter=filter)
     return aggregate(y)
 
 

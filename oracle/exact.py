@@ -38,27 +38,59 @@ def brute_force_count(g, q) -> int:
     return count
 
 
-def tree_walk(g, q, method: int) -> Tuple[Fraction, Fraction, Dict[tuple, Tuple[int, ...]]]:
+def candidate_sets(g, q, filter: int = 0):
+    """Global candidate sets C(u) (Def. 4) written out from their definitions:
+    0 label; 1 + deg(v) >= deg_q(u) (LDF); 2 + |N_l(v)| >= |N_l^q(u)| for every label l
+    (NLF) — DESIGN.md readings A2, A21."""
+    adj = _adjacency_sets(g)
+    lab = [int(x) for x in g.labels]
+    out = []
+    for u in range(q.nq):
+        qn = [w for w in range(q.nq) if q.adj[u, w]]
+        need = {}
+        for w in qn:
+            need[int(q.labels[w])] = need.get(int(q.labels[w]), 0) + 1
+        cu = set()
+        for v in range(g.n):
+            if lab[v] != int(q.labels[u]):
+                continue
+            if filter >= 1 and len(adj[v]) < len(qn):
+                continue
+            if filter >= 2 and any(sum(1 for x in adj[v] if lab[x] == l) < c for l, c in need.items()):
+                continue
+            cu.add(v)
+        out.append(cu)
+    return out
+
+
+def embeddings(g, q):
+    """All embeddings as tuples f[u] (brute force, tiny graphs only)."""
+    adj = _adjacency_sets(g)
+    lab = [int(x) for x in g.labels]
+    edges = q.edges()
+    return [f for f in itertools.permutations(range(g.n), q.nq)
+            if all(lab[f[u]] == int(q.labels[u]) for u in range(q.nq)) and all(f[b] in adj[f[a]] for a, b in edges)]
+
+
+def tree_walk(g, q, method: int, filter: int = 0) -> Tuple[Fraction, Fraction, Dict[tuple, Tuple[int, ...]]]:
     """Returns (E[Y], E[Y^2], cand) where cand[prefix] = the candidate list C_d the
     sampler draws from after matching `prefix` (len(prefix) = d)."""
     adj = _adjacency_sets(g)
-    lab = [int(x) for x in g.labels]
     order = [int(x) for x in q.order]
-    qlab = [int(q.labels[u]) for u in range(q.nq)]
     nq = q.nq
+    csets = candidate_sets(g, q, filter)
     cand: Dict[tuple, Tuple[int, ...]] = {}
 
-    def local(v: int, l: int):
-        return sorted(w for w in adj[v] if lab[w] == l)
+    def local(v: int, u: int):  # C(u', u, v) = N(v) ∩ C(u)
+        return sorted(w for w in adj[v] if w in csets[u])
 
     def candidates(prefix: tuple):
         d = len(prefix)
         u = order[d]
-        l = qlab[u]
         if d == 0:
-            return [v for v in range(g.n) if lab[v] == l], None
+            return sorted(csets[u]), None
         back = [j for j in range(d) if q.adj[order[j], u]]
-        lists = [local(prefix[j], l) for j in back]
+        lists = [local(prefix[j], u) for j in back]
         p = min(range(len(back)), key=lambda b: (len(lists[b]), b))
         if method == 0:  # WanderJoin: the smallest local list, unfiltered
             return lists[p], (back, lists, p)

@@ -104,13 +104,43 @@ static int contains(const int32_t* list, int64_t len, int32_t x) {
     return bsearch(&x, list, (size_t)len, sizeof(int32_t), cmp_i32) != NULL;
 }
 
-/* Local candidate set C(u', u, v) with the label-only filter: N(v) ∩ {w : L(w) = l},
- * ascending id (Def. 4; reading A2/A4).  Returns its size. */
-static int64_t local_candidates(const or_graph* G, int32_t v, int32_t l, int32_t* out) {
+/* Global candidate sets C(u) (Def. 4): inC[u * n + v] = 1 iff v in C(u).
+ * filter 0: label only, C(u) = {v : L(v) = L_q(u)}            (reading A2)
+ * filter 1: + degree, deg(v) >= deg_q(u)                       (LDF, reading A21)
+ * filter 2: + for every label l, |N_l(v)| >= |N_l^q(u)|         (NLF, reading A21)
+ * Each is a superset of the vertices u can map to in an embedding. */
+static void candidate_sets(const or_graph* G, const or_query* Q, int filter, uint8_t* inC) {
+    for (int u = 0; u < Q->nq; ++u) {
+        int deg_q = 0;
+        for (int w = 0; w < Q->nq; ++w) deg_q += Q->adj[u][w] ? 1 : 0;
+        for (int64_t v = 0; v < G->n; ++v) {
+            int ok = G->labels[v] == Q->label[u];
+            if (ok && filter >= 1) ok = (G->row_ptr[v + 1] - G->row_ptr[v]) >= deg_q;
+            if (ok && filter >= 2) {
+                for (int w = 0; w < Q->nq && ok; ++w) {
+                    if (!Q->adj[u][w]) continue;
+                    int32_t l = Q->label[w];
+                    int need = 0;
+                    for (int x = 0; x < Q->nq; ++x)
+                        if (Q->adj[u][x] && Q->label[x] == l) need += 1;
+                    int64_t have = 0;
+                    for (int64_t i = G->row_ptr[v]; i < G->row_ptr[v + 1]; ++i)
+                        if (G->labels[G->col[i]] == l) have += 1;
+                    ok = have >= need;
+                }
+            }
+            inC[(int64_t)u * G->n + v] = (uint8_t)ok;
+        }
+    }
+}
+
+/* Local candidate set C(u', u, v) = N(v) ∩ C(u), ascending id (Def. 4; A2/A4).
+ * `inCu` is the membership row of C(u).  Returns its size. */
+static int64_t local_candidates(const or_graph* G, int32_t v, const uint8_t* inCu, int32_t* out) {
     int64_t len = 0;
     for (int64_t i = G->row_ptr[v]; i < G->row_ptr[v + 1]; ++i) {
         int32_t w = G->col[i];
-        if (G->labels[w] == l) out[len++] = w;
+        if (inCu[w]) out[len++] = w;
     }
     return len;
 }
@@ -118,7 +148,7 @@ static int64_t local_candidates(const or_graph* G, int32_t v, int32_t l, int32_t
 /* ---- one sample (Alg. 1 inner loop) --------------------------------- */
 /* method: 0 = WanderJoin, 1 = Alley.  Returns Y (0 if not a complete instance). */
 static double one_sample(const or_graph* G, const or_query* Q, int method, uint64_t seed, uint64_t sid,
-                         const int32_t* C0, int64_t C0_len, int32_t** S, int32_t* refine,
+                         const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
                          or_record* rec) {
     int32_t M[OR_MAX_QV];
     int nq = Q->nq;
@@ -141,7 +171,6 @@ static double one_sample(const or_graph* G, const or_query* Q, int method, uint6
     for (int d = 1; d < nq; ++d) {
         depth_reached = d;
         int32_t u = Q->order[d];
-        int32_t l = Q->label[u];
         /* backward positions B(d) = { j < d : (phi[j], phi[d]) in E_q } */
         int B[OR_MAX_QV], nb = 0;
         for (int j = 0; j < d; ++j)
@@ -151,7 +180,7 @@ static double one_sample(const or_graph* G, const or_query* Q, int method, uint6
         int64_t len[OR_MAX_QV];
         int p = 0;
         for (int b = 0; b < nb; ++b) {
-            len[b] = local_candidates(G, M[B[b]], l, S[b]);
+            len[b] = local_candidates(G, M[B[b]], inC + (int64_t)u * G->n, S[b]);
             if (len[b] < len[p]) p = b;
         }
         int64_t clen;
@@ -233,10 +262,36 @@ static int load_query(or_query* Q, int32_t nq, const int32_t* q_row_ptr, const i
  * Run samples [first, first + count).  y_out[i] = Y of sample first+i (may be NULL);
  * rec_out[i] = its record (may be NULL).  Returns 0, or -1 on bad input / OOM.
  */
+/* Candidate sets of `filter` for every query vertex: out[u * n + v] (nq * n bytes). */
+int or_candidate_sets(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                      int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                      const int32_t* order, int filter, uint8_t* out) {
+    or_graph G = {n, row_ptr, col, labels};
+    or_query Q;
+    int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
+    if (rc) return rc;
+    candidate_sets(&G, &Q, filter, out);
+    return 0;
+}
+
+int or_sample_range_f(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                      int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                      const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
+                      double* y_out, or_record* rec_out, int filter);
+
 int or_sample_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
                     int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
                     const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
                     double* y_out, or_record* rec_out) {
+    return or_sample_range_f(n, row_ptr, col, labels, nq, q_row_ptr, q_col, q_labels, order, method, seed, first,
+                             count, y_out, rec_out, 0);
+}
+
+/* Run samples [first, first + count) with the candidate sets of `filter`. */
+int or_sample_range_f(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                      int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                      const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
+                      double* y_out, or_record* rec_out, int filter) {
     or_graph G = {n, row_ptr, col, labels};
     or_query Q;
     int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
@@ -244,22 +299,26 @@ int or_sample_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const
     int64_t maxdeg = 0;
     for (int64_t v = 0; v < n; ++v)
         if (row_ptr[v + 1] - row_ptr[v] > maxdeg) maxdeg = row_ptr[v + 1] - row_ptr[v];
-    /* global candidate set of phi[0]: all vertices with its label, ascending (reading A2) */
     int32_t* C0 = (int32_t*)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
     int32_t* buf = (int32_t*)malloc(sizeof(int32_t) * (size_t)(maxdeg + 1) * (OR_MAX_QV + 1));
     if (!C0 || !buf) { free(C0); free(buf); return -1; }
+    uint8_t* inC = (uint8_t*)malloc((size_t)(n > 0 ? n : 1) * (size_t)nq);
+    if (!inC) { free(C0); free(buf); return -1; }
+    candidate_sets(&G, &Q, filter, inC);
+    /* global candidate set of phi[0], ascending */
     int64_t C0_len = 0;
-    int32_t l0 = Q.label[Q.order[0]];
+    const uint8_t* in0 = inC + (int64_t)Q.order[0] * n;
     for (int64_t v = 0; v < n; ++v)
-        if (labels[v] == l0) C0[C0_len++] = (int32_t)v;
+        if (in0[v]) C0[C0_len++] = (int32_t)v;
     int32_t* S[OR_MAX_QV];
     for (int b = 0; b < OR_MAX_QV; ++b) S[b] = buf + (size_t)b * (size_t)(maxdeg + 1);
     int32_t* refine = buf + (size_t)OR_MAX_QV * (size_t)(maxdeg + 1);
     for (uint64_t i = 0; i < count; ++i) {
-        double y = one_sample(&G, &Q, method, seed, first + i, C0, C0_len, S, refine,
+        double y = one_sample(&G, &Q, method, seed, first + i, C0, C0_len, inC, S, refine,
                               rec_out ? &rec_out[i] : NULL);
         if (y_out) y_out[i] = y;
     }
+    free(inC);
     free(C0);
     free(buf);
     return 0;

@@ -255,3 +255,62 @@ def test_bad_order_rejected():
     q = gen.query_from_edges(3, [(0, 1), (1, 2)], order=[0, 2, 1])
     with pytest.raises(ValueError):
         oracle.sample_range(gen.complete_graph(4), q, oracle.WJ, 0, 0, 10)
+
+
+# ---------------------------------------------------------------- candidate filters (NEXT-1)
+def _nlf_example():
+    rows = {r[0]: r[1:] for r in read_golden("nlf_example.txt") if not r[0].isdigit()}
+    sets = [(int(r[0]), int(r[1]), sorted(int(x) for x in r[2:])) for r in read_golden("nlf_example.txt")
+            if r[0].isdigit()]
+    labels = np.array([int(x) for x in rows["labels"]], np.int32)
+    e = [tuple(int(y) for y in x.split("-")) for x in rows["edges"]]
+    g = gen.make_graph(labels.shape[0], [a for a, _ in e], [b for _, b in e], labels, 3)
+    qe = [tuple(int(y) for y in x.split("-")) for x in rows["qedges"]]
+    q = gen.query_from_edges(3, qe, labels=[int(x) for x in rows["qlabels"]], order=[0, 1, 2])
+    return g, q, sets
+
+
+def test_filter_golden_example():
+    g, q, sets = _nlf_example()
+    for f in (0, 1, 2):
+        c = oracle.candidate_sets(g, q, f)
+        py = exact.candidate_sets(g, q, f)
+        for ff, u, members in sets:
+            if ff == f:
+                assert sorted(np.nonzero(c[u])[0].tolist()) == members
+                assert sorted(py[u]) == members
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_filters_sound_and_consistent(seed):
+    g = gen.random_small_graph(8, 0.45, n_labels=1 + seed % 3, seed=500 + seed)
+    q = gen.random_connected_query(2 + seed % 4, 0.5, g.n_labels, 600 + seed)
+    embs = exact.embeddings(g, q)
+    prev = None
+    for f in (0, 1, 2):
+        c = oracle.candidate_sets(g, q, f)
+        py = exact.candidate_sets(g, q, f)
+        assert [set(np.nonzero(c[u])[0].tolist()) for u in range(q.nq)] == py
+        for emb in embs:  # soundness: every embedding survives the filter
+            assert all(c[u][emb[u]] for u in range(q.nq))
+        if prev is not None:  # monotone: each filter refines the previous one
+            assert np.all(c <= prev)
+        prev = c
+
+
+@pytest.mark.parametrize("seed", range(8))
+@pytest.mark.parametrize("method", [oracle.WJ, oracle.ALLEY])
+@pytest.mark.parametrize("filt", [1, 2])
+def test_filtered_tree_walk_and_records(seed, method, filt):
+    g = gen.random_small_graph(8, 0.5, n_labels=1 + seed % 2, seed=700 + seed)
+    try:
+        q = gen.extract_query(g, 3 + seed % 3, seed=800 + seed, dense=bool(seed % 2))
+    except RuntimeError:
+        q = gen.random_connected_query(3, 0.5, g.n_labels, 800 + seed)
+    ey, _, cand = exact.tree_walk(g, q, method, filter=filt)
+    assert ey == exact.brute_force_count(g, q)  # the filtered estimator stays unbiased
+    _, rec = oracle.sample_range(g, q, method, seed=seed, first=0, count=400, filter=filt)
+    for r in rec:
+        for d in range(int(r["depth_reached"]) + 1):
+            prefix = tuple(int(x) for x in r["path"][:d])
+            assert int(r["csize"][d]) == len(cand[prefix])
