@@ -93,6 +93,18 @@ typedef struct {
     uint32_t dup_mask[GSWORD_MAX_QV];
 } gsword_plan_info;
 
+/* Statistics of the loaded query (gsword_query_info).
+ *   candidates[u]  |C(u)| for query vertex u under the filter the query was loaded with
+ *   cg_entries     total local-candidate entries of the candidate graph (0 for filter 0)
+ *   build_seconds  device time of the candidate-graph build (0 for filter 0) */
+typedef struct {
+    int32_t nq;
+    int32_t filter;
+    uint64_t candidates[GSWORD_MAX_QV];
+    uint64_t cg_entries;
+    double build_seconds;
+} gsword_query_stats;
+
 /* Tunables for gsword_set_option (defaults chosen by measurement). */
 typedef enum {
     GSWORD_OPT_BLOCKS_PER_SM = 0,  /* persistent CTAs per SM; 0 = occupancy maximum  */
@@ -102,8 +114,11 @@ typedef enum {
     GSWORD_OPT_COOP_THRESHOLD = 4, /* Alley |S_p| above which the warp refines it in   */
                                    /* 32-element chunks (0..128; below: task pool)    */
     GSWORD_OPT_BLOOM = 5,          /* 1 = edge Bloom pre-test (L2-resident filter)    */
-    GSWORD_OPT_EDGE_SET = 6        /* 1 = exact edge hash set for adjacency tests;    */
+    GSWORD_OPT_EDGE_SET = 6,       /* 1 = exact edge hash set for adjacency tests;    */
                                    /* 0 = binary search in the adjacency run          */
+    GSWORD_OPT_FILTER = 7          /* candidate filter applied by the next            */
+                                   /* gsword_load_query: 0 label only, 1 LDF, 2 NLF   */
+                                   /* (1-2 build the candidate graph, reading A21)    */
 } gsword_option;
 
 /* ---- context -------------------------------------------------------------------- */
@@ -139,13 +154,19 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value);
 int gsword_load_graph(gsword_ctx* ctx, int64_t n_vertices, const int64_t* row_ptr, const int32_t* col,
                       const int32_t* labels, int32_t n_labels);
 
-/* Load the query q and its matching order phi (Def. 2).  Host arrays, copied:
+/* Load the query q and its matching order phi (Def. 2).  Host arrays, copied.
+ * With GSWORD_OPT_FILTER > 0 this also builds the candidate graph on the device
+ * (Def. 5; Fig. 4) and the sampler draws from its local candidate lists:
  *   q_row_ptr int32[n_qv+1], q_col: symmetric query adjacency over vertices 0..n_qv-1
  *   q_labels  int32[n_qv] in [0, n_labels of the loaded graph)
  *   order     int32[n_qv], a permutation of 0..n_qv-1 with every prefix connected
  * Errors: ENOGRAPH, EINVAL, EORDER, ELIMIT (n_qv > GSWORD_MAX_QV). */
 int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, const int32_t* q_col,
                       const int32_t* q_labels, const int32_t* order);
+
+/* Statistics of the loaded query: candidate-set sizes and candidate-graph size/build
+ * time (Tab. 3 analogue).  Errors: EINVAL, ENOQUERY. */
+int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out);
 
 /* ---- estimation ----------------------------------------------------------------------- */
 

@@ -155,11 +155,20 @@ int plan_query_impl(int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, 
             if (q_labels[order[j]] == q_labels[u]) s.dup |= 1u << j;
         }
         s.nback = __builtin_popcount(s.back);
+        p.uq[d] = (uint8_t)u;
         for (int j = 0; j < nq; ++j)
             if (j != d && adj[order[j]][u]) p.qadj[d] |= 1u << j;
         if (d > 0 && s.back == 0)
             return fail(GSWORD_EORDER, "load_query: order prefix %d is not connected (reading A13)", d);
     }
+    // directed query edges (a -> b), enumerated in (a, b) order: candidate-graph rows
+    int eid[GSWORD_MAX_QV][GSWORD_MAX_QV];
+    int ne = 0;
+    for (int a = 0; a < nq; ++a)
+        for (int b = 0; b < nq; ++b) eid[a][b] = adj[a][b] ? ne++ : -1;
+    for (int d = 0; d < nq; ++d)
+        for (int j = 0; j < d; ++j)
+            if (adj[order[j]][order[d]]) p.eidx[d][j] = (uint8_t)eid[order[j]][order[d]];
     if (plan) *plan = p;
     if (info) {
         std::memset(info, 0, sizeof(*info));
@@ -199,6 +208,32 @@ struct gsword_ctx {
     // query
     bool query_loaded = false;
     Plan plan{};
+    int32_t* d_vlabel = nullptr;      // vertex labels (filters need them on the device)
+    // candidate graph of the loaded query (filters 1-2, NEXT-1)
+    int opt_filter = 0;
+    int q_filter = 0;                 // filter the loaded query was built with
+    uint32_t* d_cbits = nullptr;
+    uint32_t* d_cg_off = nullptr;
+    int32_t* d_clist = nullptr;
+    int32_t* d_cand0 = nullptr;
+    uint32_t cwords = 0;
+    uint64_t cg_entries = 0;
+    double cg_seconds = 0.0;
+    uint64_t cand_count[GSWORD_MAX_QV] = {};
+
+    void free_query() {
+        if (d_cbits) cudaFree(d_cbits);
+        if (d_cg_off) cudaFree(d_cg_off);
+        if (d_clist) cudaFree(d_clist);
+        if (d_cand0) cudaFree(d_cand0);
+        d_cbits = nullptr;
+        d_cg_off = nullptr;
+        d_clist = nullptr;
+        d_cand0 = nullptr;
+        cg_entries = 0;
+        q_filter = 0;
+        query_loaded = false;
+    }
     // scratch
     unsigned long long* d_queue = nullptr;
     Partial* d_partials = nullptr;
@@ -219,6 +254,9 @@ struct gsword_ctx {
     int last_grid = 0, last_threads = 0;
 
     void free_graph() {
+        free_query();
+        if (d_vlabel) cudaFree(d_vlabel);
+        d_vlabel = nullptr;
         if (d_col) cudaFree(d_col);
         if (d_hot) cudaFree(d_hot);
         if (d_bucket) cudaFree(d_bucket);
@@ -302,7 +340,11 @@ DeviceGraph device_graph(const gsword_ctx* ctx) {
     DeviceGraph g;
     g.col = ctx->d_col;
     g.seg = ctx->d_seg;
-    g.bucket = ctx->d_bucket;
+    g.bucket = ctx->q_filter ? ctx->d_cand0 : ctx->d_bucket;
+    g.clist = ctx->q_filter ? ctx->d_clist : ctx->d_col;
+    g.cg_off = ctx->q_filter ? ctx->d_cg_off : nullptr;
+    g.cbits = ctx->q_filter ? ctx->d_cbits : nullptr;
+    g.cwords = ctx->cwords;
     g.bloom = ctx->opt_bloom ? ctx->d_bloom : nullptr;
     g.bloom_mask = ctx->bloom_words ? ctx->bloom_words - 1 : 0;
     g.eset = ctx->opt_eset ? ctx->d_eset : nullptr;
@@ -327,6 +369,144 @@ int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, u
     CUDA_TRY(cudaEventRecord(ctx->evk1, ctx->stream));
     e = gsword::launch_reduce(ctx->d_partials, cfg.grid, d_out4, d_sectors, ctx->stream);
     if (e != cudaSuccess) return cuda_fail(e, "launch reduce kernel");
+    return GSWORD_OK;
+}
+
+// Candidate graph of the query (NEXT-1; Def. 4-5, Fig. 4):
+// C(u) by the filter, then one CSR per directed query edge a -> b with rows
+// C(a, b, v) = N(v) ∩ C(b), and the ascending list of C(phi[0]) for the seed.
+int build_candidate_graph(gsword_ctx* ctx, int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col,
+                          const int32_t* q_labels, const int32_t* order, Plan* p) {
+    cudaStream_t st = ctx->stream;
+    const int64_t n = ctx->n;
+    cudaEvent_t e0, e1;
+    CUDA_TRY(cudaEventCreate(&e0));
+    CUDA_TRY(cudaEventCreate(&e1));
+    CUDA_TRY(cudaEventRecord(e0, st));
+    // per-vertex filter data
+    gsword::QFilter qf[GSWORD_MAX_QV];
+    std::memset(qf, 0, sizeof(qf));
+    bool adj[GSWORD_MAX_QV][GSWORD_MAX_QV] = {};
+    for (int u = 0; u < nq; ++u)
+        for (int32_t i = q_row_ptr[u]; i < q_row_ptr[u + 1]; ++i) adj[u][q_col[i]] = true;
+    for (int u = 0; u < nq; ++u) {
+        qf[u].label = q_labels[u];
+        for (int w = 0; w < nq; ++w) {
+            if (!adj[u][w]) continue;
+            qf[u].deg += 1;
+            int k = 0;
+            while (k < qf[u].npairs && qf[u].plabel[k] != q_labels[w]) ++k;
+            if (k == qf[u].npairs) {
+                qf[u].plabel[k] = q_labels[w];
+                qf[u].pcount[k] = 0;
+                qf[u].npairs += 1;
+            }
+            qf[u].pcount[k] += 1;
+        }
+    }
+    int eid[GSWORD_MAX_QV][GSWORD_MAX_QV];
+    int ne = 0;
+    for (int a = 0; a < nq; ++a)
+        for (int b = 0; b < nq; ++b) eid[a][b] = adj[a][b] ? ne++ : -1;
+    ctx->cwords = (uint32_t)((n + 31) / 32) + 1;
+    const size_t row = (size_t)n + 1;
+    gsword::QFilter* d_qf = nullptr;
+    uint32_t* d_tmp = nullptr;
+    unsigned long long* d_tot = nullptr;
+    uint32_t* d_cnt0 = nullptr;
+    const size_t tmpw = gsword::scan_tmp_words((int64_t)row);
+    cudaError_t e;
+    if ((e = cudaMalloc(&ctx->d_cbits, sizeof(uint32_t) * (size_t)nq * ctx->cwords)) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_cg_off, sizeof(uint32_t) * row * (size_t)std::max(ne, 1))) != cudaSuccess ||
+        (e = cudaMalloc(&d_qf, sizeof(qf))) != cudaSuccess ||
+        (e = cudaMalloc(&d_tmp, sizeof(uint32_t) * tmpw)) != cudaSuccess ||
+        (e = cudaMalloc(&d_tot, sizeof(unsigned long long) * (size_t)(ne + 2))) != cudaSuccess ||
+        (e = cudaMalloc(&d_cnt0, sizeof(uint32_t) * row)) != cudaSuccess) {
+        cudaFree(d_qf);
+        cudaFree(d_tmp);
+        cudaFree(d_tot);
+        cudaFree(d_cnt0);
+        return fail(GSWORD_ENOMEM, "load_query: candidate graph allocation: %s", cudaGetErrorString(e));
+    }
+    auto cleanup = [&]() {
+        cudaFree(d_qf);
+        cudaFree(d_tmp);
+        cudaFree(d_tot);
+        cudaFree(d_cnt0);
+        cudaEventDestroy(e0);
+        cudaEventDestroy(e1);
+    };
+#define CG_TRY(expr)                     \
+    do {                                 \
+        cudaError_t _e = (expr);         \
+        if (_e != cudaSuccess) {         \
+            cleanup();                   \
+            return cuda_fail(_e, #expr); \
+        }                                \
+    } while (0)
+    ctx->q_filter = ctx->opt_filter;
+    gsword::DeviceGraph g = device_graph(ctx);
+    g.cbits = ctx->d_cbits;
+    g.cwords = ctx->cwords;
+    CG_TRY(cudaMemcpyAsync(d_qf, qf, sizeof(qf), cudaMemcpyHostToDevice, st));
+    CG_TRY(cudaMemsetAsync(ctx->d_cbits, 0, sizeof(uint32_t) * (size_t)nq * ctx->cwords, st));
+    CG_TRY(gsword::launch_filter(g, d_qf, nq, ctx->q_filter, ctx->d_cbits, ctx->d_vlabel, st));
+    // seed list C(phi[0])
+    CG_TRY(gsword::launch_bits_count(ctx->d_cbits, ctx->cwords, order[0], n, d_cnt0, st));
+    CG_TRY(gsword::launch_scan(d_cnt0, (int64_t)row, nullptr, d_tmp, d_tot + ne + 1, st));
+    // per directed edge a -> b: counts, then offsets chained across edges
+    CG_TRY(cudaMemsetAsync(d_tot, 0, sizeof(unsigned long long), st));
+    for (int a = 0; a < nq; ++a)
+        for (int b = 0; b < nq; ++b) {
+            const int ed = eid[a][b];
+            if (ed < 0) continue;
+            uint32_t* off = ctx->d_cg_off + (size_t)ed * row;
+            CG_TRY(gsword::launch_cg_count(g, ctx->d_cbits, a, b, q_labels[b], off, st));
+            CG_TRY(gsword::launch_scan(off, (int64_t)row, d_tot + ed, d_tmp, d_tot + ed + 1, st));
+        }
+    unsigned long long tot[GSWORD_MAX_QV * GSWORD_MAX_QV + 2];
+    CG_TRY(cudaMemcpyAsync(tot, d_tot, sizeof(unsigned long long) * (size_t)(ne + 2), cudaMemcpyDeviceToHost, st));
+    CG_TRY(cudaStreamSynchronize(st));
+    const uint64_t entries = tot[ne];
+    const uint64_t n0 = tot[ne + 1];
+    if (entries >= (1ull << 32)) {
+        cleanup();
+        return fail(GSWORD_ELIMIT, "load_query: candidate graph has %llu entries (>= 2^32)",
+                    (unsigned long long)entries);
+    }
+    if ((e = cudaMalloc(&ctx->d_clist, sizeof(int32_t) * (size_t)std::max<uint64_t>(entries, 1))) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_cand0, sizeof(int32_t) * (size_t)std::max<uint64_t>(n0, 1))) != cudaSuccess) {
+        cleanup();
+        return fail(GSWORD_ENOMEM, "load_query: candidate graph (%llu entries): %s", (unsigned long long)entries,
+                    cudaGetErrorString(e));
+    }
+    CG_TRY(gsword::launch_bits_fill(ctx->d_cbits, ctx->cwords, order[0], n, d_cnt0, ctx->d_cand0, st));
+    for (int a = 0; a < nq; ++a)
+        for (int b = 0; b < nq; ++b) {
+            const int ed = eid[a][b];
+            if (ed < 0) continue;
+            CG_TRY(gsword::launch_cg_fill(g, ctx->d_cbits, a, b, q_labels[b], ctx->d_cg_off + (size_t)ed * row,
+                                          ctx->d_clist, st));
+        }
+    CG_TRY(cudaEventRecord(e1, st));
+    // candidate counts per query vertex (popcount of the bitmap rows)
+    std::vector<uint32_t> bits((size_t)nq * ctx->cwords);
+    CG_TRY(cudaMemcpyAsync(bits.data(), ctx->d_cbits, sizeof(uint32_t) * bits.size(), cudaMemcpyDeviceToHost, st));
+    CG_TRY(cudaStreamSynchronize(st));
+    float ms = 0.f;
+    CG_TRY(cudaEventElapsedTime(&ms, e0, e1));
+#undef CG_TRY
+    cleanup();
+    for (int u = 0; u < nq; ++u) {
+        uint64_t c = 0;
+        for (uint32_t w = 0; w < ctx->cwords; ++w) c += (uint64_t)__builtin_popcount(bits[(size_t)u * ctx->cwords + w]);
+        ctx->cand_count[u] = c;
+    }
+    ctx->cg_entries = entries;
+    ctx->cg_seconds = ms * 1e-3;
+    p->seed_lo = 0;
+    p->seed_len = (uint32_t)n0;
+    p->seed_identity = 0;
     return GSWORD_OK;
 }
 
@@ -414,6 +594,10 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
         case GSWORD_OPT_BLOOM:
             ctx->opt_bloom = value ? 1 : 0;
             return GSWORD_OK;
+        case GSWORD_OPT_FILTER:
+            if (value < 0 || value > 2) return fail(GSWORD_EINVAL, "filter must be 0 (label), 1 (LDF) or 2 (NLF)");
+            ctx->opt_filter = (int)value;
+            return GSWORD_OK;
         case GSWORD_OPT_EDGE_SET:
             ctx->opt_eset = value ? 1 : 0;
             return GSWORD_OK;
@@ -499,6 +683,14 @@ int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const 
     ctx->d_bloom = reinterpret_cast<unsigned long long*>(ctx->d_hot);
     ctx->d_seg = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ctx->d_hot) + words * sizeof(unsigned long long));
     if (nnz > 0) CUDA_TRY(cudaMemcpy(ctx->d_col, col_up, sizeof(int32_t) * (size_t)nnz, cudaMemcpyHostToDevice));
+    if ((e = cudaMalloc(&ctx->d_vlabel, sizeof(int32_t) * (size_t)std::max<int64_t>(n, 1))) != cudaSuccess) {
+        ctx->free_graph();
+        return fail(GSWORD_ENOMEM, "load_graph: cudaMalloc(labels): %s", cudaGetErrorString(e));
+    }
+    if (labels && n > 0)
+        CUDA_TRY(cudaMemcpy(ctx->d_vlabel, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyHostToDevice));
+    else if (n > 0)
+        CUDA_TRY(cudaMemset(ctx->d_vlabel, 0, sizeof(int32_t) * (size_t)n));
     CUDA_TRY(cudaMemcpy(ctx->d_seg, seg.data(), sizeof(uint32_t) * seg.size(), cudaMemcpyHostToDevice));
     if (L > 1) {
         if (n > 0) CUDA_TRY(cudaMemcpy(ctx->d_bucket, bucket.data(), sizeof(int32_t) * (size_t)n, cudaMemcpyHostToDevice));
@@ -545,12 +737,36 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
     Plan p;
     int rc = plan_query_impl(n_qv, q_row_ptr, q_col, q_labels, order, ctx->n_labels, &p, nullptr);
     if (rc) return rc;
+    CUDA_TRY(cudaSetDevice(ctx->device));
+    CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    ctx->free_query();
     const int32_t l0 = p.step[0].label;
     p.seed_lo = (uint32_t)ctx->label_off[(size_t)l0];
     p.seed_len = (uint32_t)(ctx->label_off[(size_t)l0 + 1] - ctx->label_off[(size_t)l0]);
     p.seed_identity = (ctx->n_labels == 1) ? 1 : 0;
+    for (int u = 0; u < n_qv; ++u)
+        ctx->cand_count[u] = (uint64_t)(ctx->label_off[(size_t)q_labels[u] + 1] - ctx->label_off[(size_t)q_labels[u]]);
+    if (ctx->opt_filter > 0) {
+        rc = build_candidate_graph(ctx, n_qv, q_row_ptr, q_col, q_labels, order, &p);
+        if (rc) {
+            ctx->free_query();
+            return rc;
+        }
+    }
     ctx->plan = p;
     ctx->query_loaded = true;
+    return GSWORD_OK;
+}
+
+int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out) {
+    if (!ctx || !out) return fail(GSWORD_EINVAL, "query_info: NULL argument");
+    if (!ctx->query_loaded) return fail(GSWORD_ENOQUERY, "query_info: no query loaded");
+    std::memset(out, 0, sizeof(*out));
+    out->nq = ctx->plan.nq;
+    out->filter = ctx->q_filter;
+    for (int u = 0; u < ctx->plan.nq; ++u) out->candidates[u] = ctx->cand_count[u];
+    out->cg_entries = ctx->cg_entries;
+    out->build_seconds = ctx->cg_seconds;
     return GSWORD_OK;
 }
 

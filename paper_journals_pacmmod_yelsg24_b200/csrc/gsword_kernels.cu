@@ -148,6 +148,25 @@ __device__ __forceinline__ void segment(const DeviceGraph& g, uint32_t v, int32_
     *b = ldg_u32(g.seg + i + 1);
 }
 
+// Run of the local candidate list C(phi[j], phi[d], v) in clist (Def. 4): the
+// label-filtered adjacency run (filter 0) or the candidate-graph row of directed
+// query edge e (filters 1-2).
+__device__ __forceinline__ void local_run(const DeviceGraph& g, int e, uint32_t v, int32_t l, uint32_t* a,
+                                          uint32_t* b) {
+    if (g.cg_off) {
+        const uint32_t* off = g.cg_off + (size_t)e * (size_t)(g.n + 1) + v;
+        *a = ldg_u32(off);
+        *b = ldg_u32(off + 1);
+    } else {
+        segment(g, v, l, a, b);
+    }
+}
+
+// v in C(u)?  (membership bitmap of the candidate graph; only used under a filter)
+__device__ __forceinline__ bool in_cand(const DeviceGraph& g, int u, uint32_t v) {
+    return (ldg_u32(g.cbits + (size_t)u * g.cwords + (v >> 5)) >> (v & 31u)) & 1u;
+}
+
 // Is {a, b} an edge of G?  Exact.  (1) blocked Bloom filter (L2-resident): "no" is
 // final; (2) exact edge set (one 32-byte bucket per probe); without the edge set, a
 // binary search of b in N_lb(a) (lb = L(b)).  `sec` accumulates the sectors touched.
@@ -216,6 +235,8 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                                                      unsigned long long* __restrict__ phase_out) {
     __shared__ PlanStep plan_s[kMaxQV];
     __shared__ uint32_t qadj_s[kMaxQV];
+    __shared__ uint8_t eidx_s[kMaxQV][kMaxQV];
+    __shared__ uint8_t uq_s[kMaxQV];
     __shared__ uint32_t res_s[256];   // Alley task-pool results per lane (adjacent matched vertices)
     __shared__ uint32_t rm_s[4][256];  // Alley task-pool results per lane: refine-mask removals (128 bits)
     __shared__ Partial warp_part[32];
@@ -229,7 +250,9 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
     if (tid < kMaxQV) {
         plan_s[tid] = plan_in.step[tid];
         qadj_s[tid] = plan_in.qadj[tid];
+        uq_s[tid] = plan_in.uq[tid];
     }
+    if (tid < kMaxQV * kMaxQV) eidx_s[tid / kMaxQV][tid % kMaxQV] = plan_in.eidx[tid / kMaxQV][tid % kMaxQV];
     __syncthreads();
 
     const int nq = plan_in.nq;
@@ -320,7 +343,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 // one backward neighbour: p is fixed by the plan; the segment load is left
                 // in flight and consumed after the exclusion tests (which need only M)
                 p = __ffs(ps.back) - 1;
-                segment(g, Ms[p * T + tid], ps.label, &seg_a, &seg_b);
+                local_run(g, eidx_s[d][p], Ms[p * T + tid], ps.label, &seg_a, &seg_b);
                 deferred = true;
                 if (MODE == kModeCount) sectors += 1.0;
             } else {
@@ -331,7 +354,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     const int j = __ffs(bm) - 1;
                     bm &= bm - 1;
                     uint32_t a, b;
-                    segment(g, Ms[j * T + tid], ps.label, &a, &b);
+                    local_run(g, eidx_s[d][j], Ms[j * T + tid], ps.label, &a, &b);
                     if (b - a < len_p) {
                         len_p = b - a;
                         lo_p = a;
@@ -354,7 +377,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     if (d == 0) {
                         v = plan_in.seed_identity ? (int32_t)(lo_p + k) : ldg_i32(g.bucket + lo_p + k);
                     } else {
-                        v = ldg_i32(g.col + lo_p + k);
+                        v = ldg_i32(g.clist + lo_p + k);
                         if (MODE == kModeCount) sectors += 1.0;
                         // Validate: DupCheck, then IsEdge for the other matched neighbours.
                         // v in N_l(M[j]) <=> M[j] in N_{L(phi[j])}(v): search the shorter run.
@@ -413,8 +436,20 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 // (no self loops); the rest need an edge test {M[p], M[j]}.
                 const uint32_t qa = qadj_s[p];
                 kind = 1;
-                known = ps.dup & qa;
-                unk = ps.dup & ~qa & ~(1u << p);
+                uint32_t cdup = ps.dup & ~(1u << p);
+                if (g.cbits) {
+                    // under a filter S_p lies inside C(phi[d]): matched vertices outside it
+                    // cannot be in S_p
+                    uint32_t m = cdup;
+                    const int ud = uq_s[d];
+                    while (m) {
+                        const int j = __ffs(m) - 1;
+                        m &= m - 1;
+                        if (!in_cand(g, ud, Ms[j * T + tid])) cdup &= ~(1u << j);
+                    }
+                }
+                known = cdup & qa;
+                unk = cdup & ~qa;
             }
             __syncwarp();
             // pool 1: exclusion tests, overlapping the in-flight segment loads
@@ -465,7 +500,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     const uint32_t nth = k / olen;
                     const uint32_t i = k - nth * olen;
                     const int j = (int)fns32(omask, nth);
-                    const int32_t x = ldg_i32(g.col + olo + i);
+                    const int32_t x = ldg_i32(g.clist + olo + i);
                     if (!is_edge<MODE == kModeCount>(g, Ms[j * T + ocol], (uint32_t)x, olab, sectors))
                         atomicOr(&rm_s[i >> 5][ocol], 1u << (i & 31));
                 }
@@ -479,7 +514,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     // smallest idx with idx = k + #{x in X : x <= S_p[idx]}: the k-th survivor
                     uint32_t idx = k;
                     while (true) {
-                        v = ldg_i32(g.col + lo_p + idx);
+                        v = ldg_i32(g.clist + lo_p + idx);
                         uint32_t c = 0, xm = in_sp;
                         while (xm) {
                             const int j = __ffs(xm) - 1;
@@ -506,7 +541,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     while (mm) {
                         const int i = __ffs(mm) - 1;
                         mm &= mm - 1;
-                        if (!not_matched(Ms + tid, T, 0, dup, ldg_i32(g.col + lo_p + 32u * w + i))) m &= ~(1u << i);
+                        if (!not_matched(Ms + tid, T, 0, dup, ldg_i32(g.clist + lo_p + 32u * w + i))) m &= ~(1u << i);
                     }
                     keep[w] = m;
                     cnt += __popc(m);
@@ -520,7 +555,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                         if (k < c && pos == 0u) pos = 32u * w + fns32(keep[w], k) + 1u;  // +1: found marker
                         if (pos == 0u) k -= c;
                     }
-                    v = ldg_i32(g.col + lo_p + pos - 1u);
+                    v = ldg_i32(g.clist + lo_p + pos - 1u);
                 }
             }
             const bool coop = (kind == 3);
@@ -546,7 +581,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     bool keep = i < Llen;
                     int32_t x = 0;
                     if (keep) {
-                        x = ldg_i32(g.col + Llo + i);
+                        x = ldg_i32(g.clist + Llo + i);
                         keep = member_all<MODE == kModeCount>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
                                not_matched(Ms, T, colL, Lps.dup, x);
                     }
@@ -572,7 +607,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                         const unsigned hm = __ballot_sync(kFull, here);
                         const int c = __ffs(hm) - 1;
                         int32_t val = 0;
-                        if (lane == c) val = ldg_i32(g.col + Llo + (uint32_t)c * 32u + fns32(my_bal, k - excl));
+                        if (lane == c) val = ldg_i32(g.clist + Llo + (uint32_t)c * 32u + fns32(my_bal, k - excl));
                         chosen = __shfl_sync(kFull, val, c);
                     } else {
                         uint32_t run = 0;
@@ -581,7 +616,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                             bool keep = i < Llen;
                             int32_t x = 0;
                             if (keep) {
-                                x = ldg_i32(g.col + Llo + i);
+                                x = ldg_i32(g.clist + Llo + i);
                                 keep = member_all<MODE == kModeCount>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
                                        not_matched(Ms, T, colL, Lps.dup, x);
                             }
@@ -748,6 +783,159 @@ __global__ void bloom_kernel(const int64_t* __restrict__ row_ptr, const int32_t*
     }
 }
 
+// ---------------------------------------------------------------- candidate graph build
+// (NEXT-1; Def. 4-5, Fig. 4).  Load-time only.
+__device__ __forceinline__ uint32_t nbr_count(const DeviceGraph& g, uint32_t v, int32_t l) {
+    uint32_t a, b;
+    segment(g, v, l, &a, &b);
+    return b - a;
+}
+
+// cbits[u][v] for every query vertex u (warp-aligned vertex groups -> one word per ballot)
+__global__ void filter_kernel(const DeviceGraph g, const QFilter* __restrict__ qf, int nq, int filter,
+                              uint32_t* __restrict__ cbits, const int32_t* __restrict__ vlabel) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nwarps = (int64_t)gridDim.x * (blockDim.x >> 5);
+    const int64_t warp = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    for (int64_t base = warp * 32; base < g.n; base += nwarps * 32) {
+        const int64_t v = base + lane;
+        const bool in = v < g.n;
+        const int32_t lv = in ? vlabel[v] : -1;
+        uint32_t deg = 0;
+        if (in) {
+            uint32_t a, b, a2, b2;
+            segment(g, (uint32_t)v, 0, &a, &b);
+            segment(g, (uint32_t)v, g.n_labels - 1, &a2, &b2);
+            deg = b2 - a;
+        }
+        for (int u = 0; u < nq; ++u) {
+            bool ok = in && lv == qf[u].label;
+            if (ok && filter >= 1) ok = deg >= (uint32_t)qf[u].deg;
+            if (ok && filter >= 2)
+                for (int i = 0; i < qf[u].npairs && ok; ++i)
+                    ok = nbr_count(g, (uint32_t)v, qf[u].plabel[i]) >= (uint32_t)qf[u].pcount[i];
+            const unsigned word = __ballot_sync(0xffffffffu, ok);
+            if (lane == 0) cbits[(size_t)u * g.cwords + (size_t)(base >> 5)] = word;
+        }
+    }
+}
+
+__device__ __forceinline__ bool bit_of(const uint32_t* cbits, uint32_t cwords, int u, uint32_t v) {
+    return (cbits[(size_t)u * cwords + (v >> 5)] >> (v & 31u)) & 1u;
+}
+
+// counts[v] = |N_{label2}(v) ∩ C(u2)| if v in C(u) else 0;  counts[n] = 0
+__global__ void cg_count_kernel(const DeviceGraph g, const uint32_t* __restrict__ cbits, int u, int u2,
+                                int32_t label2, uint32_t* __restrict__ counts) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= g.n; v += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t c = 0;
+        if (v < g.n && bit_of(cbits, g.cwords, u, (uint32_t)v)) {
+            uint32_t a, b;
+            segment(g, (uint32_t)v, label2, &a, &b);
+            for (uint32_t i = a; i < b; ++i) c += bit_of(cbits, g.cwords, u2, (uint32_t)g.col[i]) ? 1u : 0u;
+        }
+        counts[v] = c;
+    }
+}
+
+__global__ void cg_fill_kernel(const DeviceGraph g, const uint32_t* __restrict__ cbits, int u, int u2,
+                               int32_t label2, const uint32_t* __restrict__ off, int32_t* __restrict__ out) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < g.n; v += (int64_t)gridDim.x * blockDim.x) {
+        if (!bit_of(cbits, g.cwords, u, (uint32_t)v)) continue;
+        uint32_t pos = off[v];
+        uint32_t a, b;
+        segment(g, (uint32_t)v, label2, &a, &b);
+        for (uint32_t i = a; i < b; ++i) {
+            const int32_t w = g.col[i];
+            if (bit_of(cbits, g.cwords, u2, (uint32_t)w)) out[pos++] = w;
+        }
+    }
+}
+
+__global__ void bits_count_kernel(const uint32_t* __restrict__ cbits, uint32_t cwords, int u, int64_t n,
+                                  uint32_t* __restrict__ counts) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= n; v += (int64_t)gridDim.x * blockDim.x)
+        counts[v] = (v < n && bit_of(cbits, cwords, u, (uint32_t)v)) ? 1u : 0u;
+}
+
+__global__ void bits_fill_kernel(const uint32_t* __restrict__ cbits, uint32_t cwords, int u, int64_t n,
+                                 const uint32_t* __restrict__ off, int32_t* __restrict__ out) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        if (bit_of(cbits, cwords, u, (uint32_t)v)) out[off[v]] = (int32_t)v;
+}
+
+// ---- exclusive scan (three phases): 2048 elements per block
+constexpr int kScanThreads = 1024;
+constexpr int kScanPer = 2048;
+
+__device__ __forceinline__ uint32_t block_exclusive(uint32_t x, uint32_t* warp_tot, uint32_t* total) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    uint32_t incl = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += y;
+    }
+    if (lane == 31) warp_tot[w] = incl;
+    __syncthreads();
+    if (w == 0) {
+        uint32_t t = warp_tot[lane];
+        uint32_t ti = t;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, ti, o);
+            if (lane >= o) ti += y;
+        }
+        warp_tot[lane] = ti - t;
+        if (lane == 31) *total = ti;
+    }
+    __syncthreads();
+    const uint32_t r = warp_tot[w] + incl - x;
+    __syncthreads();
+    return r;
+}
+
+__global__ void scan_local_kernel(uint32_t* __restrict__ data, int64_t n, uint32_t* __restrict__ block_sums) {
+    __shared__ uint32_t wt[32];
+    __shared__ uint32_t tot;
+    const int64_t i0 = (int64_t)blockIdx.x * kScanPer + 2 * threadIdx.x;
+    const uint32_t a = i0 < n ? data[i0] : 0u;
+    const uint32_t b = i0 + 1 < n ? data[i0 + 1] : 0u;
+    const uint32_t ex = block_exclusive(a + b, wt, &tot);
+    if (i0 < n) data[i0] = ex;
+    if (i0 + 1 < n) data[i0 + 1] = ex + a;
+    if (threadIdx.x == 0) block_sums[blockIdx.x] = tot;
+}
+
+// one block: exclusive scan of the block sums (in 64-bit, offset by *base_in);
+// total_out[0] = base + sum (64-bit, for the overflow check on the host)
+__global__ void scan_sums_kernel(uint32_t* __restrict__ block_sums, int64_t nb, const unsigned long long* base_in,
+                                 unsigned long long* total_out) {
+    __shared__ unsigned long long carry;
+    __shared__ uint32_t wt[32];
+    __shared__ uint32_t tot;
+    if (threadIdx.x == 0) carry = base_in ? *base_in : 0ull;
+    __syncthreads();
+    for (int64_t b0 = 0; b0 < nb; b0 += kScanThreads) {
+        const int64_t i = b0 + threadIdx.x;
+        const uint32_t x = i < nb ? block_sums[i] : 0u;
+        const uint32_t ex = block_exclusive(x, wt, &tot);
+        const unsigned long long c = carry;
+        if (i < nb) block_sums[i] = (uint32_t)(c + ex);  // absolute offset (checked < 2^32 on host)
+        __syncthreads();
+        if (threadIdx.x == 0) carry = c + tot;
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) *total_out = carry;
+}
+
+__global__ void scan_add_kernel(uint32_t* __restrict__ data, int64_t n, const uint32_t* __restrict__ block_sums) {
+    const int64_t i0 = (int64_t)blockIdx.x * kScanPer + 2 * threadIdx.x;
+    const uint32_t add = block_sums[blockIdx.x];
+    if (i0 < n) data[i0] += add;
+    if (i0 + 1 < n) data[i0 + 1] += add;
+}
+
 template <int METHOD, int MODE>
 const void* kernel_ptr() {
     return reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE>);
@@ -805,6 +993,47 @@ cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int
 cudaError_t launch_build_eset(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* keys,
                               uint64_t mask, cudaStream_t stream) {
     eset_kernel<<<148 * 8, 256, 0, stream>>>(d_row_ptr, col, n, keys, mask);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_filter(const DeviceGraph& g, const QFilter* d_qf, int nq, int filter, uint32_t* cbits,
+                          const int32_t* d_vlabel, cudaStream_t stream) {
+    filter_kernel<<<148 * 4, 256, 0, stream>>>(g, d_qf, nq, filter, cbits, d_vlabel);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_cg_count(const DeviceGraph& g, const uint32_t* cbits, int u, int u2, int32_t label2,
+                            uint32_t* counts, cudaStream_t stream) {
+    cg_count_kernel<<<148 * 8, 256, 0, stream>>>(g, cbits, u, u2, label2, counts);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_cg_fill(const DeviceGraph& g, const uint32_t* cbits, int u, int u2, int32_t label2,
+                           const uint32_t* off, int32_t* out, cudaStream_t stream) {
+    cg_fill_kernel<<<148 * 8, 256, 0, stream>>>(g, cbits, u, u2, label2, off, out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bits_count(const uint32_t* cbits, uint32_t cwords, int u, int64_t n, uint32_t* counts,
+                              cudaStream_t stream) {
+    bits_count_kernel<<<148 * 4, 256, 0, stream>>>(cbits, cwords, u, n, counts);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bits_fill(const uint32_t* cbits, uint32_t cwords, int u, int64_t n, const uint32_t* off,
+                             int32_t* out, cudaStream_t stream) {
+    bits_fill_kernel<<<148 * 4, 256, 0, stream>>>(cbits, cwords, u, n, off, out);
+    return cudaGetLastError();
+}
+
+size_t scan_tmp_words(int64_t n) { return (size_t)((n + kScanPer - 1) / kScanPer) + 1; }
+
+cudaError_t launch_scan(uint32_t* data, int64_t n, const unsigned long long* d_base, uint32_t* d_tmp,
+                        unsigned long long* d_total, cudaStream_t stream) {
+    const int64_t nb = (n + kScanPer - 1) / kScanPer;
+    scan_local_kernel<<<(unsigned)nb, kScanThreads, 0, stream>>>(data, n, d_tmp);
+    scan_sums_kernel<<<1, kScanThreads, 0, stream>>>(d_tmp, nb, d_base, d_total);
+    scan_add_kernel<<<(unsigned)nb, kScanThreads, 0, stream>>>(data, n, d_tmp);
     return cudaGetLastError();
 }
 

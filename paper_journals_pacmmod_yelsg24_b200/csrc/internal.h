@@ -30,6 +30,18 @@ struct Plan {
     uint32_t seed_len;
     PlanStep step[kMaxQV];
     uint32_t qadj[kMaxQV];  // bit j: (phi[j], phi[d]) is a query edge, any j != d
+    uint8_t uq[kMaxQV];     // phi[d] (query vertex at depth d: row of cbits)
+    uint8_t eidx[kMaxQV][kMaxQV];  // directed query edge (phi[j] -> phi[d]) index, j in B(d)
+};
+
+// Candidate filter of one query vertex (NEXT-1): label, degree, and the per-label
+// neighbour counts NLF requires.
+struct QFilter {
+    int32_t label;
+    int32_t deg;
+    int32_t npairs;
+    int32_t plabel[kMaxQV];
+    int32_t pcount[kMaxQV];
 };
 
 // Device-resident data graph, relaid out for the sampler:
@@ -39,10 +51,20 @@ struct Plan {
 //   bloom: blocked Bloom filter over the undirected edge set (one 64-bit word per
 //   test, 3 bits, ~16 bits per edge): "no" is exact, "maybe" falls back to the
 //   binary search.  NULL = disabled.
+//   clist/cg_off/cbits: the lists the sampler draws from.  Filter 0 (label only):
+//   clist = col, runs located through seg.  Filters 1-2 (LDF/NLF, NEXT-1): the
+//   candidate graph (Def. 5, Fig. 4) -- one CSR per directed query edge
+//   e = (u -> u'): clist[cg_off[e*(n+1) + v] .. cg_off[e*(n+1) + v + 1]) =
+//   C(u, u', v) = N(v) ∩ C(u') ascending (empty when v is not in C(u)); cbits row u =
+//   membership bitmap of C(u).
 struct DeviceGraph {
     const int32_t* col;
     const uint32_t* seg;
-    const int32_t* bucket;
+    const int32_t* bucket;     // seed list: label buckets, or C(phi[0]) under a filter
+    const int32_t* clist;
+    const uint32_t* cg_off;
+    const uint32_t* cbits;
+    uint32_t cwords;           // words per cbits row
     const unsigned long long* bloom;
     uint64_t bloom_mask;  // words - 1 (words is a power of two)
     // exact edge set: open addressing, 32-byte buckets of 4 keys (min<<32 | max),
@@ -97,6 +119,22 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
 cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_out4, double* d_sectors,
                           cudaStream_t stream);
 cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream);
+// candidate graph build (NEXT-1)
+cudaError_t launch_filter(const DeviceGraph& g, const QFilter* d_qf, int nq, int filter, uint32_t* cbits,
+                          const int32_t* d_vlabel, cudaStream_t stream);
+cudaError_t launch_cg_count(const DeviceGraph& g, const uint32_t* cbits, int u, int u2, int32_t label2,
+                            uint32_t* counts, cudaStream_t stream);
+cudaError_t launch_cg_fill(const DeviceGraph& g, const uint32_t* cbits, int u, int u2, int32_t label2,
+                           const uint32_t* off, int32_t* out, cudaStream_t stream);
+cudaError_t launch_bits_count(const uint32_t* cbits, uint32_t cwords, int u, int64_t n, uint32_t* counts,
+                              cudaStream_t stream);
+cudaError_t launch_bits_fill(const uint32_t* cbits, uint32_t cwords, int u, int64_t n, const uint32_t* off,
+                             int32_t* out, cudaStream_t stream);
+// exclusive scan of n u32 in place, offset by *d_base (64-bit, may be NULL = 0); the
+// 64-bit grand total goes to *d_total.  d_tmp holds scan_tmp_words(n) words.
+size_t scan_tmp_words(int64_t n);
+cudaError_t launch_scan(uint32_t* data, int64_t n, const unsigned long long* d_base, uint32_t* d_tmp,
+                        unsigned long long* d_total, cudaStream_t stream);
 constexpr unsigned long long kEmptyKey = ~0ull;
 cudaError_t launch_build_eset(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* keys,
                               uint64_t mask, cudaStream_t stream);

@@ -29,6 +29,8 @@ OPT_L2_PERSIST = 3
 OPT_COOP_THRESHOLD = 4
 OPT_BLOOM = 5
 OPT_EDGE_SET = 6
+OPT_FILTER = 7
+FILTER_LABEL, FILTER_LDF, FILTER_NLF = 0, 1, 2
 CUDA_STREAM_LEGACY = 0x1  # cudaStreamLegacy
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOGRAPH", -3: "ENOQUERY", -4: "EORDER", -5: "EGRAPH",
@@ -52,6 +54,11 @@ class _Result(ctypes.Structure):
     _fields_ = [("estimate", ctypes.c_double), ("variance", ctypes.c_double), ("sum", ctypes.c_double),
                 ("sumsq", ctypes.c_double), ("n_samples", ctypes.c_uint64), ("n_valid", ctypes.c_uint64),
                 ("seconds", ctypes.c_double)]
+
+
+class _QueryStats(ctypes.Structure):
+    _fields_ = [("nq", ctypes.c_int32), ("filter", ctypes.c_int32), ("candidates", ctypes.c_uint64 * MAX_QV),
+                ("cg_entries", ctypes.c_uint64), ("build_seconds", ctypes.c_double)]
 
 
 class _PlanInfo(ctypes.Structure):
@@ -82,6 +89,7 @@ def _load_library() -> ctypes.CDLL:
         "gsword_launch_info": ([P, P, P, P], ctypes.c_int),
         "gsword_last_kernel_seconds": ([P, P], ctypes.c_int),
         "gsword_phase_cycles": ([P, P], ctypes.c_int),
+        "gsword_query_info": ([P, ctypes.POINTER(_QueryStats)], ctypes.c_int),
         "gsword_check_graph": ([I64, P, P, P, I32], ctypes.c_int),
         "gsword_plan_query": ([I32, P, P, P, P, I32, ctypes.POINTER(_PlanInfo)], ctypes.c_int),
         "gsword_last_error": ([], ctypes.c_char_p),
@@ -227,6 +235,12 @@ class Context:
         _check(_lib.gsword_load_query(self._h, qlab.shape[0], _ptr(qrp), _ptr(qcol), _ptr(qlab), _ptr(od)))
         self.nq = int(qlab.shape[0])
         return int(qrp.nbytes + qcol.nbytes + qlab.nbytes + od.nbytes)
+
+    def query_info(self) -> Dict[str, object]:
+        st = _QueryStats()
+        _check(_lib.gsword_query_info(self._h, ctypes.byref(st)))
+        return {"nq": st.nq, "filter": st.filter, "candidates": list(st.candidates)[:st.nq],
+                "cg_entries": int(st.cg_entries), "build_seconds": st.build_seconds}
 
     # convenience for workloads.gen.Graph / Query objects
     def load_graph_obj(self, g) -> None:

@@ -295,3 +295,58 @@ def test_async_matches_sync_on_torch_stream(ctx, G, c0):
         assert r["sum"] == ref["sum"] and r["n_valid"] == ref["n_valid"]
     finally:
         ctx.set_stream(None)
+
+
+# ------------------------------------------------------------------ NEXT-1: candidate graph
+def _parity_filtered(ctx, G, g, q, method, seed, first, count, filt, threads=8):
+    ctx.load_query_obj(q)
+    rec = ctx.trace_samples(method, first, count, seed)
+    y, ref = oracle.sample_range(g, q, method, seed, first, count, records=True, threads=threads, filter=filt)
+    _records_equal(rec, ref, f"{g.name}/{q.name}/m{method}/f{filt}")
+    _agg_close(ctx.estimate(method, count, seed, first=first), oracle.aggregate(y), G)
+
+
+@pytest.mark.parametrize("filt", [1, 2])
+def test_filtered_parity_small_and_c0(ctx, G, c0, filt):
+    ctx.set_option(G.OPT_FILTER, filt)
+    try:
+        for seed in range(8):
+            rng = np.random.default_rng(seed)
+            g = gen.random_small_graph(int(rng.integers(6, 30)), 0.4, int(rng.integers(1, 4)), seed=900 + seed)
+            try:
+                q = gen.extract_query(g, int(rng.integers(2, 6)), seed=seed, dense=bool(seed % 2))
+            except RuntimeError:
+                q = gen.random_connected_query(3, 0.5, g.n_labels, seed)
+            ctx.load_graph_obj(g)
+            for m in (0, 1):
+                _parity_filtered(ctx, G, g, q, m, seed, 0, 3000, filt)
+        g, qs = c0
+        ctx.load_graph_obj(g)
+        for i, q in enumerate(qs):
+            for m in (0, 1):
+                _parity_filtered(ctx, G, g, q, m, 3 + i, 0, 50_000, filt)
+            info = ctx.query_info()
+            cs = oracle.candidate_sets(g, q, filt)
+            assert info["filter"] == filt and info["candidates"] == [int(x) for x in cs.sum(axis=1)]
+    finally:
+        ctx.set_option(G.OPT_FILTER, 0)
+
+
+@pytest.mark.parametrize("filt", [1, 2])
+def test_filtered_parity_c2_c1(ctx, G, c1, filt):
+    ctx.set_option(G.OPT_FILTER, filt)
+    try:
+        for g, qs, count in (gen.config_c2() + (20_000,), c1 + (10_000,)):
+            ctx.load_graph_obj(g)
+            for q in qs:
+                for m in (0, 1):
+                    _parity_filtered(ctx, G, g, q, m, 5, 0, count, filt, threads=16)
+                    for coop in (0, 128):
+                        ctx.set_option(G.OPT_COOP_THRESHOLD, coop)
+                        ctx.load_query_obj(q)
+                        rec = ctx.trace_samples(m, 777, 2000, 5)
+                        _, ref = oracle.sample_range(g, q, m, 5, 777, 2000, records=True, threads=16, filter=filt)
+                        _records_equal(rec, ref, f"{q.name}/f{filt}/coop{coop}")
+                    ctx.set_option(G.OPT_COOP_THRESHOLD, 64)
+    finally:
+        ctx.set_option(G.OPT_FILTER, 0)
