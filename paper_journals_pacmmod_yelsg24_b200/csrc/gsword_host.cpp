@@ -357,14 +357,16 @@ DeviceGraph device_graph(const gsword_ctx* ctx) {
 
 int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, uint64_t seed, double* d_out4,
         gsword_sample_record* d_records, double* d_sectors) {
+    if (ctx->q_filter) mode |= gsword::kModeCG;
     LaunchCfg cfg;
     int rc = launch_config(ctx, method, mode, &cfg);
     if (rc) return rc;
     CUDA_TRY(cudaEventRecord(ctx->evk0, ctx->stream));
-    if (mode == gsword::kModeCount) CUDA_TRY(cudaMemsetAsync(ctx->d_phase, 0, 8 * sizeof(unsigned long long), ctx->stream));
+    const bool counting = (mode & 3) == gsword::kModeCount;
+    if (counting) CUDA_TRY(cudaMemsetAsync(ctx->d_phase, 0, 8 * sizeof(unsigned long long), ctx->stream));
     cudaError_t e = gsword::launch_sample(method, mode, device_graph(ctx), ctx->plan, cfg, first, count, seed,
                                           ctx->d_queue, ctx->d_partials, d_records,
-                                          mode == gsword::kModeCount ? ctx->d_phase : nullptr, ctx->stream);
+                                          counting ? ctx->d_phase : nullptr, ctx->stream);
     if (e != cudaSuccess) return cuda_fail(e, "launch sample kernel");
     CUDA_TRY(cudaEventRecord(ctx->evk1, ctx->stream));
     e = gsword::launch_reduce(ctx->d_partials, cfg.grid, d_out4, d_sectors, ctx->stream);

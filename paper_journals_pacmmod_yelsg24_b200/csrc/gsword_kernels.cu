@@ -151,9 +151,10 @@ __device__ __forceinline__ void segment(const DeviceGraph& g, uint32_t v, int32_
 // Run of the local candidate list C(phi[j], phi[d], v) in clist (Def. 4): the
 // label-filtered adjacency run (filter 0) or the candidate-graph row of directed
 // query edge e (filters 1-2).
+template <bool CG>
 __device__ __forceinline__ void local_run(const DeviceGraph& g, int e, uint32_t v, int32_t l, uint32_t* a,
                                           uint32_t* b) {
-    if (g.cg_off) {
+    if (CG) {
         const uint32_t* off = g.cg_off + (size_t)e * (size_t)(g.n + 1) + v;
         *a = ldg_u32(off);
         *b = ldg_u32(off + 1);
@@ -224,7 +225,7 @@ __device__ __forceinline__ bool not_matched(const uint32_t* Ms, int stride, int 
 #define GSWORD_AL_MIN_BLOCKS 5  // 51 registers: 40 warps per SM (measured best)
 #endif
 
-template <int METHOD, int MODE>
+template <int METHOD, int MODE, bool CG>
 __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLOCKS : GSWORD_AL_MIN_BLOCKS)
     sample_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
                                                      const uint64_t count, const uint64_t seed, const int chunk,
@@ -343,7 +344,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 // one backward neighbour: p is fixed by the plan; the segment load is left
                 // in flight and consumed after the exclusion tests (which need only M)
                 p = __ffs(ps.back) - 1;
-                local_run(g, eidx_s[d][p], Ms[p * T + tid], ps.label, &seg_a, &seg_b);
+                local_run<CG>(g, eidx_s[d][p], Ms[p * T + tid], ps.label, &seg_a, &seg_b);
                 deferred = true;
                 if (MODE == kModeCount) sectors += 1.0;
             } else {
@@ -354,7 +355,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     const int j = __ffs(bm) - 1;
                     bm &= bm - 1;
                     uint32_t a, b;
-                    local_run(g, eidx_s[d][j], Ms[j * T + tid], ps.label, &a, &b);
+                    local_run<CG>(g, eidx_s[d][j], Ms[j * T + tid], ps.label, &a, &b);
                     if (b - a < len_p) {
                         len_p = b - a;
                         lo_p = a;
@@ -437,7 +438,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 const uint32_t qa = qadj_s[p];
                 kind = 1;
                 uint32_t cdup = ps.dup & ~(1u << p);
-                if (g.cbits) {
+                if (CG) {
                     // under a filter S_p lies inside C(phi[d]): matched vertices outside it
                     // cannot be in S_p
                     uint32_t m = cdup;
@@ -936,20 +937,27 @@ __global__ void scan_add_kernel(uint32_t* __restrict__ data, int64_t n, const ui
     if (i0 + 1 < n) data[i0 + 1] += add;
 }
 
-template <int METHOD, int MODE>
+template <int METHOD, int MODE, bool CG>
 const void* kernel_ptr() {
-    return reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE>);
+    return reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE, CG>);
 }
 
-const void* select_kernel(int method, int mode) {
+template <bool CG>
+const void* select_kernel_cg(int method, int mode) {
     if (method == GSWORD_WJ) {
-        if (mode == kModeTrace) return kernel_ptr<GSWORD_WJ, kModeTrace>();
-        if (mode == kModeCount) return kernel_ptr<GSWORD_WJ, kModeCount>();
-        return kernel_ptr<GSWORD_WJ, kModeEstimate>();
+        if (mode == kModeTrace) return kernel_ptr<GSWORD_WJ, kModeTrace, CG>();
+        if (mode == kModeCount) return kernel_ptr<GSWORD_WJ, kModeCount, CG>();
+        return kernel_ptr<GSWORD_WJ, kModeEstimate, CG>();
     }
-    if (mode == kModeTrace) return kernel_ptr<GSWORD_ALLEY, kModeTrace>();
-    if (mode == kModeCount) return kernel_ptr<GSWORD_ALLEY, kModeCount>();
-    return kernel_ptr<GSWORD_ALLEY, kModeEstimate>();
+    if (mode == kModeTrace) return kernel_ptr<GSWORD_ALLEY, kModeTrace, CG>();
+    if (mode == kModeCount) return kernel_ptr<GSWORD_ALLEY, kModeCount, CG>();
+    return kernel_ptr<GSWORD_ALLEY, kModeEstimate, CG>();
+}
+
+// mode: kMode* | kModeCG when the query was loaded with a candidate filter
+const void* select_kernel(int method, int mode) {
+    return (mode & kModeCG) ? select_kernel_cg<true>(method, mode & ~kModeCG)
+                            : select_kernel_cg<false>(method, mode & ~kModeCG);
 }
 
 }  // namespace

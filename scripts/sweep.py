@@ -18,6 +18,7 @@ ap.add_argument("--samples", type=float, default=1e8)
 ap.add_argument("--grid", default='{"coop": [32]}', help="JSON dict option -> list of values")
 ap.add_argument("--methods", default="0,1")
 ap.add_argument("--reps", type=int, default=2)
+ap.add_argument("--filter", type=int, default=0)
 args = ap.parse_args()
 OPT = {"coop": G.OPT_COOP_THRESHOLD, "threads": G.OPT_THREADS, "chunk": G.OPT_CHUNK, "bps": G.OPT_BLOCKS_PER_SM,
        "l2": G.OPT_L2_PERSIST, "bloom": G.OPT_BLOOM, "eset": G.OPT_EDGE_SET}
@@ -27,8 +28,10 @@ g, qs = gen.CONFIGS[args.config]()
 queries = qs if args.query < 0 else [qs[args.query]]
 with G.Context(0) as ctx:
     ctx.load_graph_obj(g)
+    ctx.set_option(G.OPT_FILTER, args.filter)
     for q in queries:
         ctx.load_query_obj(q)
+        qi = ctx.query_info()
         for m in [int(x) for x in args.methods.split(",")]:
             ctx.estimate(m, 1_000_000, 1)
             keys = list(grid)
@@ -42,7 +45,9 @@ with G.Context(0) as ctx:
                     r = ctx.estimate(m, int(args.samples), 42)
                     t = ctx.last_kernel_seconds()
                     best = t if best is None else min(best, t)
-                print(json.dumps({"config": args.config, "query": q.name, "method": m,
+                print(json.dumps({"config": args.config, "query": q.name, "method": m, "filter": args.filter,
+                                  "cg_entries": qi["cg_entries"], "cg_build_s": qi["build_seconds"],
+                                  "candidates": qi["candidates"],
                                   "opts": dict(zip(keys, vals)), "kernel_s": best,
                                   "rate": args.samples / best, "valid": r["n_valid"], "est": r["estimate"]}),
                       flush=True)
