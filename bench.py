@@ -193,6 +193,32 @@ def run_reference(args):
     return 0
 
 
+# ---------------------------------------------------------------- q-error
+def qerror_leg(G, ctx, args, samples: int = 100_000_000):
+    """q-error against the exact count where one exists: BASELINE configs[0] (C0), exact
+    counts from tests/golden/c0_exact_counts.txt (written by the oracle's enumerator).
+    Untimed; runs after the timed region on the same context."""
+    from workloads import gen
+    path = os.path.join(ROOT, "tests", "golden", "c0_exact_counts.txt")
+    exact = {}
+    for line in open(path):
+        if line.strip() and not line.startswith("#"):
+            i, qname, c = line.split()
+            exact[qname] = int(c)
+    g, qs = gen.config_c0()
+    ctx.load_graph_obj(g)
+    out = {}
+    for m, key in ((G.WJ, "wj"), (G.ALLEY, "alley")):
+        errs = []
+        for q in qs:
+            ctx.load_query_obj(q)
+            r = ctx.estimate(m, samples, args.seed)
+            errs.append(G.qerror(exact[q.name], r["estimate"]))
+        out[key] = {"median": statistics.median(errs), "max": max(errs)}
+    return {"config": "C0 (BASELINE configs[0]): 11 four-vertex queries", "samples_per_query": samples,
+            "exact_from": "tests/golden/c0_exact_counts.txt (oracle enumerator)", **out}
+
+
 # ---------------------------------------------------------------- our arm
 def run_ours(args):
     import numpy as np
@@ -337,6 +363,7 @@ def run_ours(args):
 
     info = ctx.launch_info()
     name = {G.WJ: "wj", G.ALLEY: "alley"}
+    qerr = qerror_leg(G, ctx, args) if not args.quick else None
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": 1e3 * max_time / args.steps, "higher_is_better": True,
@@ -361,6 +388,7 @@ def run_ours(args):
                 "d2h_bytes_per_step": 32 * len(methods), "graph_load_s": graph_load_s,
                 "note": "per step: gsword_load_query from host arrays + gsword_estimate per method "
                         "(synchronous, host result); graph loaded once (P:L1057 excludes it)"},
+        "qerror": qerr,
         "gpu_launches": 2 * len(methods) * args.steps,
         "clocks": clocks.summary(),
     }

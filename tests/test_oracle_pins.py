@@ -314,3 +314,12 @@ def test_filtered_tree_walk_and_records(seed, method, filt):
         for d in range(int(r["depth_reached"]) + 1):
             prefix = tuple(int(x) for x in r["path"][:d])
             assert int(r["csize"][d]) == len(cand[prefix])
+
+
+def test_c0_golden_counts_in_sync(c0):
+    """tests/golden/c0_exact_counts.txt (read by bench.py) equals the oracle's counts."""
+    g, qs = c0
+    rows = read_golden("c0_exact_counts.txt")
+    assert len(rows) == len(qs)
+    for (i, name, cnt), q in zip(rows, qs):
+        assert name == q.name and int(cnt) == oracle.count_embeddings(g, q)
