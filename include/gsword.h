@@ -168,6 +168,32 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
  * time (Tab. 3 analogue).  Errors: EINVAL, ENOQUERY. */
 int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out);
 
+/* ---- matching order (NEXT-4) --------------------------------- */
+
+typedef enum {
+    GSWORD_ORDER_QUICKSI = 0, /* infrequent-edge-first order from data label statistics (A22) */
+    GSWORD_ORDER_TRIAL = 1    /* G-CARE-style trial: pilot-estimate candidate orders on the GPU,
+                                 keep the smallest single-sample variance        */
+} gsword_order_strategy;
+
+/* Host-only QuickSI-style order (reading A22).  Graph arrays as gsword_load_graph (labels
+ * may be NULL with n_labels 1); query CSR + labels as gsword_load_query.  order_out receives
+ * n_qv query-vertex ids with every prefix connected.  Errors: EINVAL, ELIMIT, EORDER. */
+int gsword_quicksi_order(int64_t n_vertices, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                         int32_t n_labels, int32_t n_qv, const int32_t* q_row_ptr, const int32_t* q_col,
+                         const int32_t* q_labels, int32_t* order_out);
+
+/* Choose a matching order for the loaded graph and LOAD the query with it.
+ *   GSWORD_ORDER_QUICKSI: as gsword_quicksi_order (no sampling).
+ *   GSWORD_ORDER_TRIAL: candidates = the QuickSI order + every directed query edge as the
+ *     first two positions completed in QuickSI preference; each is pilot-estimated with
+ *     `m`, samples [0, pilot_samples) and `seed`; the smallest variance of one sample wins
+ *     (ties: earliest candidate).  score_out (may be NULL) receives it.
+ * order_out: n_qv entries.  Errors: ENOGRAPH, EINVAL, EORDER, ELIMIT, ECUDA. */
+int gsword_select_order(gsword_ctx* ctx, int strategy, gsword_method m, int32_t n_qv, const int32_t* q_row_ptr,
+                        const int32_t* q_col, const int32_t* q_labels, uint64_t pilot_samples, uint64_t seed,
+                        int32_t* order_out, double* score_out);
+
 /* ---- estimation ----------------------------------------------------------------------- */
 
 /* Draw samples 0 .. n_samples-1 with `method` and `seed`, return the HT aggregate

@@ -209,6 +209,7 @@ struct gsword_ctx {
     bool query_loaded = false;
     Plan plan{};
     int32_t* d_vlabel = nullptr;      // vertex labels (filters need them on the device)
+    std::vector<uint64_t> pair_freq;  // data adjacency entries per (label, label) (QuickSI order)
     // candidate graph of the loaded query (filters 1-2, NEXT-1)
     int opt_filter = 0;
     int q_filter = 0;                 // filter the loaded query was built with
@@ -372,6 +373,92 @@ int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, u
     e = gsword::launch_reduce(ctx->d_partials, cfg.grid, d_out4, d_sectors, ctx->stream);
     if (e != cudaSuccess) return cuda_fail(e, "launch reduce kernel");
     return GSWORD_OK;
+}
+
+// QuickSI-style matching order (NEXT-4, reading A22): infrequent edges first.
+// vfreq[l] = |{v : L(v) = l}|; pfreq(l1, l2) = data adjacency entries with those labels.
+int quicksi_order_impl(int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                       int32_t n_labels, const std::vector<int64_t>& label_off, const std::vector<uint64_t>& pfreq,
+                       int32_t* order) {
+    Plan tmp;
+    std::vector<int32_t> ident((size_t)std::max(nq, 1));
+    for (int i = 0; i < nq; ++i) ident[(size_t)i] = i;
+    // validates the query CSR and labels (any order works for that; connectivity checked below)
+    if (nq < 1) return fail(GSWORD_EINVAL, "order: n_qv < 1");
+    if (nq > GSWORD_MAX_QV) return fail(GSWORD_ELIMIT, "order: n_qv > %d", GSWORD_MAX_QV);
+    bool adj[GSWORD_MAX_QV][GSWORD_MAX_QV] = {};
+    int deg[GSWORD_MAX_QV] = {};
+    for (int u = 0; u < nq; ++u) {
+        if (q_labels[u] < 0 || q_labels[u] >= n_labels) return fail(GSWORD_EINVAL, "order: label out of range");
+        for (int32_t i = q_row_ptr[u]; i < q_row_ptr[u + 1]; ++i) {
+            if (q_col[i] < 0 || q_col[i] >= nq || q_col[i] == u) return fail(GSWORD_EINVAL, "order: bad query edge");
+            adj[u][q_col[i]] = adj[q_col[i]][u] = true;
+        }
+    }
+    for (int u = 0; u < nq; ++u)
+        for (int w = 0; w < nq; ++w) deg[u] += adj[u][w] ? 1 : 0;
+    auto vf = [&](int u) { return (uint64_t)(label_off[(size_t)q_labels[u] + 1] - label_off[(size_t)q_labels[u]]); };
+    auto ef = [&](int a, int b) -> uint64_t {
+        if (pfreq.empty()) return vf(a) * vf(b);
+        return pfreq[(size_t)q_labels[a] * (size_t)n_labels + (size_t)q_labels[b]];
+    };
+    if (nq == 1) {
+        order[0] = 0;
+        return GSWORD_OK;
+    }
+    // first edge: (freq, -(deg a + deg b), min id, max id)
+    int ba = -1, bb = -1;
+    for (int a = 0; a < nq; ++a)
+        for (int b = a + 1; b < nq; ++b) {
+            if (!adj[a][b]) continue;
+            if (ba < 0) { ba = a; bb = b; continue; }
+            const uint64_t f = ef(a, b), fb = ef(ba, bb);
+            const int dg = deg[a] + deg[b], dgb = deg[ba] + deg[bb];
+            if (f < fb || (f == fb && dg > dgb)) { ba = a; bb = b; }
+        }
+    if (ba < 0) return fail(GSWORD_EORDER, "order: query has no edge but %d vertices", nq);
+    auto vkey_less = [&](int x, int y) {  // (vertex freq, -deg, id)
+        if (vf(x) != vf(y)) return vf(x) < vf(y);
+        if (deg[x] != deg[y]) return deg[x] > deg[y];
+        return x < y;
+    };
+    bool used[GSWORD_MAX_QV] = {};
+    order[0] = vkey_less(ba, bb) ? ba : bb;
+    order[1] = order[0] == ba ? bb : ba;
+    used[ba] = used[bb] = true;
+    for (int d = 2; d < nq; ++d) {
+        int best = -1;
+        uint64_t bf = 0;
+        for (int b = 0; b < nq; ++b) {
+            if (used[b]) continue;
+            for (int j = 0; j < d; ++j) {
+                const int a = order[j];
+                if (!adj[a][b]) continue;
+                const uint64_t f = ef(a, b);
+                if (best < 0 || f < bf || (f == bf && (deg[b] > deg[best] || (deg[b] == deg[best] && b < best)))) {
+                    best = b;
+                    bf = f;
+                }
+            }
+        }
+        if (best < 0) return fail(GSWORD_EORDER, "order: query is not connected");
+        order[d] = best;
+        used[best] = true;
+    }
+    (void)tmp;
+    return GSWORD_OK;
+}
+
+void label_pair_freq(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int32_t nL,
+                     std::vector<uint64_t>* out) {
+    out->clear();
+    if (nL > 1024) return;  // too many labels for a dense table: vertex frequencies only
+    out->assign((size_t)nL * (size_t)nL, 0);
+    for (int64_t v = 0; v < n; ++v) {
+        const int32_t lv = labels ? labels[v] : 0;
+        for (int64_t i = row_ptr[v]; i < row_ptr[v + 1]; ++i)
+            (*out)[(size_t)lv * (size_t)nL + (size_t)(labels ? labels[col[i]] : 0)] += 1;
+    }
 }
 
 // Candidate graph of the query (NEXT-1; Def. 4-5, Fig. 4):
@@ -622,6 +709,91 @@ int gsword_plan_query(int32_t n_qv, const int32_t* q_row_ptr, const int32_t* q_c
     return plan_query_impl(n_qv, q_row_ptr, q_col, q_labels, order, n_labels, nullptr, out);
 }
 
+int gsword_quicksi_order(int64_t n_vertices, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                         int32_t n_labels, int32_t n_qv, const int32_t* q_row_ptr, const int32_t* q_col,
+                         const int32_t* q_labels, int32_t* order_out) {
+    if (!row_ptr || !q_row_ptr || !q_labels || !order_out || n_vertices < 0 || n_labels < 1)
+        return fail(GSWORD_EINVAL, "quicksi_order: bad argument");
+    std::vector<int64_t> off((size_t)n_labels + 1, 0);
+    for (int64_t v = 0; v < n_vertices; ++v) {
+        const int32_t l = labels ? labels[v] : 0;
+        if (l < 0 || l >= n_labels) return fail(GSWORD_EINVAL, "quicksi_order: label out of range");
+        off[(size_t)l + 1] += 1;
+    }
+    for (int32_t l = 0; l < n_labels; ++l) off[(size_t)l + 1] += off[(size_t)l];
+    std::vector<uint64_t> pf;
+    label_pair_freq(n_vertices, row_ptr, col, labels, n_labels, &pf);
+    return quicksi_order_impl(n_qv, q_row_ptr, q_col, q_labels, n_labels, off, pf, order_out);
+}
+
+int gsword_select_order(gsword_ctx* ctx, int strategy, gsword_method m, int32_t n_qv, const int32_t* q_row_ptr,
+                        const int32_t* q_col, const int32_t* q_labels, uint64_t pilot_samples, uint64_t seed,
+                        int32_t* order_out, double* score_out) {
+    if (!ctx || !order_out) return fail(GSWORD_EINVAL, "select_order: NULL argument");
+    if (!ctx->graph_loaded) return fail(GSWORD_ENOGRAPH, "select_order: no graph loaded");
+    if (strategy != GSWORD_ORDER_QUICKSI && strategy != GSWORD_ORDER_TRIAL)
+        return fail(GSWORD_EINVAL, "select_order: unknown strategy %d", strategy);
+    int32_t qo[GSWORD_MAX_QV];
+    int rc = quicksi_order_impl(n_qv, q_row_ptr, q_col, q_labels, ctx->n_labels, ctx->label_off, ctx->pair_freq, qo);
+    if (rc) return rc;
+    if (strategy == GSWORD_ORDER_QUICKSI) {
+        std::memcpy(order_out, qo, sizeof(int32_t) * (size_t)n_qv);
+        if (score_out) *score_out = 0.0;
+        return gsword_load_query(ctx, n_qv, q_row_ptr, q_col, q_labels, order_out);
+    }
+    if (pilot_samples < 2) return fail(GSWORD_EINVAL, "select_order: pilot_samples must be >= 2");
+    // candidate orders: QuickSI, then every directed query edge as the first two positions,
+    // completed with the same infrequent-edge rule; each scored by a GPU pilot estimate
+    // (G-CARE's trial): the variance of one sample, smallest wins (ties: first).
+    bool adj[GSWORD_MAX_QV][GSWORD_MAX_QV] = {};
+    for (int u = 0; u < n_qv; ++u)
+        for (int32_t i = q_row_ptr[u]; i < q_row_ptr[u + 1]; ++i) adj[u][q_col[i]] = adj[q_col[i]][u] = true;
+    std::vector<std::vector<int32_t>> cands;
+    cands.emplace_back(qo, qo + n_qv);
+    for (int a = 0; a < n_qv; ++a)
+        for (int b = 0; b < n_qv; ++b) {
+            if (!adj[a][b]) continue;
+            std::vector<int32_t> o = {a, b};
+            bool used[GSWORD_MAX_QV] = {};
+            used[a] = used[b] = true;
+            while ((int)o.size() < n_qv) {
+                // the QuickSI order's relative preference: earliest position in qo among frontier vertices
+                int best = -1;
+                for (int t = 0; t < n_qv && best < 0; ++t) {
+                    const int c = qo[t];
+                    if (used[c]) continue;
+                    for (int x : o)
+                        if (adj[x][c]) { best = c; break; }
+                }
+                if (best < 0) break;
+                o.push_back(best);
+                used[best] = true;
+            }
+            if ((int)o.size() == n_qv) {
+                bool dup = false;
+                for (auto& c : cands) dup |= (c == o);
+                if (!dup) cands.push_back(o);
+            }
+        }
+    double best_score = 0.0;
+    int best = -1;
+    for (size_t c = 0; c < cands.size(); ++c) {
+        rc = gsword_load_query(ctx, n_qv, q_row_ptr, q_col, q_labels, cands[c].data());
+        if (rc) return rc;
+        gsword_result r;
+        rc = gsword_estimate_range(ctx, m, 0, pilot_samples, seed, &r);
+        if (rc) return rc;
+        const double score = std::isnan(r.variance) ? 0.0 : r.variance * (double)r.n_samples;
+        if (best < 0 || score < best_score) {
+            best = (int)c;
+            best_score = score;
+        }
+    }
+    std::memcpy(order_out, cands[(size_t)best].data(), sizeof(int32_t) * (size_t)n_qv);
+    if (score_out) *score_out = best_score;
+    return gsword_load_query(ctx, n_qv, q_row_ptr, q_col, q_labels, order_out);
+}
+
 int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
                       int32_t n_labels) {
     if (!ctx) return fail(GSWORD_EINVAL, "load_graph: NULL context");
@@ -727,6 +899,7 @@ int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const 
     ctx->nnz = nnz;
     ctx->n_labels = L;
     ctx->label_off = off;
+    label_pair_freq(n, row_ptr, col, labels, L, &ctx->pair_freq);
     ctx->graph_loaded = true;
     ctx->query_loaded = false;
     return apply_l2_window(ctx);

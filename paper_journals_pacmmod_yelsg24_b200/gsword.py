@@ -90,6 +90,8 @@ def _load_library() -> ctypes.CDLL:
         "gsword_last_kernel_seconds": ([P, P], ctypes.c_int),
         "gsword_phase_cycles": ([P, P], ctypes.c_int),
         "gsword_query_info": ([P, ctypes.POINTER(_QueryStats)], ctypes.c_int),
+        "gsword_quicksi_order": ([I64, P, P, P, I32, I32, P, P, P, P], ctypes.c_int),
+        "gsword_select_order": ([P, ctypes.c_int, ctypes.c_int, I32, P, P, P, U64, U64, P, P], ctypes.c_int),
         "gsword_check_graph": ([I64, P, P, P, I32], ctypes.c_int),
         "gsword_plan_query": ([I32, P, P, P, P, I32, ctypes.POINTER(_PlanInfo)], ctypes.c_int),
         "gsword_last_error": ([], ctypes.c_char_p),
@@ -156,6 +158,24 @@ def plan_query(q_row_ptr, q_col, q_labels, order, n_labels: int) -> Dict[str, li
     nq = info.nq
     return {"nq": nq, "label": list(info.label)[:nq], "back_mask": list(info.back_mask)[:nq],
             "dup_mask": list(info.dup_mask)[:nq]}
+
+
+ORDER_QUICKSI = 0
+ORDER_TRIAL = 1
+
+
+def quicksi_order(row_ptr, col, labels, n_labels, q_row_ptr, q_col, q_labels) -> list:
+    """gsword_quicksi_order: infrequent-edge-first matching order (host only, reading A22)."""
+    rp = np.ascontiguousarray(row_ptr, np.int64)
+    cl = np.ascontiguousarray(col, np.int32)
+    if cl.shape[0] == 0:
+        cl = np.zeros(1, np.int32)
+    lb = None if labels is None or n_labels == 1 else np.ascontiguousarray(labels, np.int32)
+    qrp, qcol, qlab, _ = _query_arrays(q_row_ptr, q_col, q_labels, np.zeros(1, np.int32))
+    out = np.zeros(qlab.shape[0], np.int32)
+    _check(_lib.gsword_quicksi_order(rp.shape[0] - 1, _ptr(rp), _ptr(cl), _ptr(lb), int(n_labels), qlab.shape[0],
+                                     _ptr(qrp), _ptr(qcol), _ptr(qlab), _ptr(out)))
+    return out.tolist()
 
 
 def qerror(c: float, c_hat: float) -> float:
@@ -235,6 +255,17 @@ class Context:
         _check(_lib.gsword_load_query(self._h, qlab.shape[0], _ptr(qrp), _ptr(qcol), _ptr(qlab), _ptr(od)))
         self.nq = int(qlab.shape[0])
         return int(qrp.nbytes + qcol.nbytes + qlab.nbytes + od.nbytes)
+
+    def select_order(self, strategy: int, method: int, q_row_ptr, q_col, q_labels, pilot_samples: int = 100_000,
+                     seed: int = 1):
+        """gsword_select_order: choose and LOAD a matching order; returns (order, score)."""
+        qrp, qcol, qlab, _ = _query_arrays(q_row_ptr, q_col, q_labels, np.zeros(1, np.int32))
+        out = np.zeros(qlab.shape[0], np.int32)
+        score = ctypes.c_double()
+        _check(_lib.gsword_select_order(self._h, int(strategy), int(method), qlab.shape[0], _ptr(qrp), _ptr(qcol),
+                                        _ptr(qlab), int(pilot_samples), int(seed), _ptr(out), ctypes.byref(score)))
+        self.nq = int(qlab.shape[0])
+        return out.tolist(), score.value
 
     def query_info(self) -> Dict[str, object]:
         st = _QueryStats()

@@ -134,3 +134,29 @@ def test_product_package_does_not_touch_oracle():
             if f.endswith((".py", ".cu", ".cpp", ".h", ".cuh")):
                 src = open(os.path.join(dirpath, f)).read()
                 assert "oracle" not in src.replace("CPU oracle", ""), f
+
+
+def test_quicksi_order_golden():
+    rows = {r[0]: r[1:] for r in read_golden("quicksi_example.txt")}
+    labels = np.array([int(x) for x in rows["ex1_labels"]], np.int32)
+    e = [tuple(int(y) for y in x.split("-")) for x in rows["ex1_edges"]]
+    g = gen.make_graph(labels.shape[0], [a for a, _ in e], [b for _, b in e], labels, 3)
+    qe = [tuple(int(y) for y in x.split("-")) for x in rows["ex1_qedges"]]
+    q = gen.query_from_edges(4, qe, labels=[int(x) for x in rows["ex1_qlabels"]], order=[0, 1, 2, 3])
+    qrp, qcol = q.csr()
+    assert G.quicksi_order(g.row_ptr, g.col, g.labels, 3, qrp, qcol, q.labels) == [int(x) for x in rows["ex1_order"]]
+    ring = gen.ring_graph(10)
+    p4 = gen.path_query(4)
+    qrp, qcol = p4.csr()
+    assert G.quicksi_order(ring.row_ptr, ring.col, None, 1, qrp, qcol, p4.labels) == [int(x) for x in rows["ex2_order"]]
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_quicksi_order_valid(seed):
+    g = gen.random_small_graph(15, 0.3, 3, seed=seed)
+    q = gen.random_connected_query(2 + seed % 10, 0.3, 3, seed)
+    qrp, qcol = q.csr()
+    order = G.quicksi_order(g.row_ptr, g.col, g.labels, 3, qrp, qcol, q.labels)
+    assert sorted(order) == list(range(q.nq))
+    p = G.plan_query(qrp, qcol, q.labels, order, 3)  # raises EORDER unless every prefix is connected
+    assert p["nq"] == q.nq

@@ -350,3 +350,46 @@ def test_filtered_parity_c2_c1(ctx, G, c1, filt):
                     ctx.set_option(G.OPT_COOP_THRESHOLD, 64)
     finally:
         ctx.set_option(G.OPT_FILTER, 0)
+
+
+# ------------------------------------------------------------------ NEXT-4: matching order
+def _trial_candidates(q, qo):
+    """The documented candidate set of GSWORD_ORDER_TRIAL (include/gsword.h)."""
+    adj = q.adj
+    cands = [list(qo)]
+    for a in range(q.nq):
+        for b in range(q.nq):
+            if not adj[a, b]:
+                continue
+            o = [a, b]
+            while len(o) < q.nq:
+                nxt = next((c for c in qo if c not in o and any(adj[x, c] for x in o)), None)
+                if nxt is None:
+                    break
+                o.append(nxt)
+            if len(o) == q.nq and o not in cands:
+                cands.append(o)
+    return cands
+
+
+@pytest.mark.parametrize("method", [0, 1])
+def test_order_selection_trial_matches_oracle(ctx, G, c0, method):
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    for q in qs[:6]:
+        qrp, qcol = q.csr()
+        qo = G.quicksi_order(g.row_ptr, g.col, g.labels, g.n_labels, qrp, qcol, q.labels)
+        order, score = ctx.select_order(G.ORDER_TRIAL, method, qrp, qcol, q.labels, pilot_samples=20_000, seed=9)
+        scores = []
+        for o in _trial_candidates(q, qo):
+            agg = oracle.aggregate(oracle.sample_range(g, q.with_order(o), method, 9, 0, 20_000, records=False)[0])
+            scores.append((agg["variance"] * agg["n"], o))
+        best = min(scores, key=lambda t: t[0])  # min keeps the first of equal scores
+        assert order == best[1]
+        assert score == pytest.approx(best[0], rel=1e-9, abs=1e-9)
+        # the chosen order is loaded: estimates now follow it
+        r = ctx.estimate(method, 5000, 3)
+        ref = oracle.aggregate(oracle.sample_range(g, q.with_order(order), method, 3, 0, 5000, records=False)[0])
+        assert r["sum"] == pytest.approx(ref["sum"], rel=1e-12)
+        o2, _ = ctx.select_order(G.ORDER_QUICKSI, method, qrp, qcol, q.labels)
+        assert o2 == qo
