@@ -43,6 +43,14 @@ RECORD_DTYPE = np.dtype([
 ])
 assert RECORD_DTYPE.itemsize == 152
 
+# trawling record (168 bytes): status 0 prefix died, 1 enumerated, 2 budget exceeded
+TRAWL_DTYPE = np.dtype([
+    ("sample_id", "<u8"), ("status", "u1"), ("d", "u1"), ("pad", "u1", (6,)),
+    ("path", "<i4", (MAX_QV,)), ("csize", "<u4", (MAX_QV,)), ("weight", "<f8"), ("count", "<u8"),
+    ("nodes", "<u8"),
+])
+assert TRAWL_DTYPE.itemsize == 168
+
 
 def build(force: bool = False) -> str:
     """Compile oracle.c -> liboracle.so (gcc, plain -O2)."""
@@ -71,6 +79,12 @@ def _load():
             lib.or_sample_range_f.restype = ctypes.c_int
             lib.or_candidate_sets.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, ctypes.c_int, P]
             lib.or_candidate_sets.restype = ctypes.c_int
+            lib.or_trawl_range.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, ctypes.c_int,
+                                           ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64,
+                                           ctypes.c_int, P, P, P]
+            lib.or_trawl_range.restype = ctypes.c_int
+            lib.or_trawl_record_size.restype = ctypes.c_int
+            assert lib.or_trawl_record_size() == TRAWL_DTYPE.itemsize
             lib.or_count_embeddings.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, P, P]
             lib.or_count_embeddings.restype = ctypes.c_int
             lib.or_record_size.restype = ctypes.c_int
@@ -156,6 +170,44 @@ def sample_range(g, q, method: int, seed: int, first: int, count: int, records: 
     if rc != 0:
         raise ValueError(f"oracle rejected input (rc={rc})")
     return y, rec
+
+
+def trawl_range(g, q, method: int, seed: int, first: int, count: int, budget: int = 2**62, filter: int = 0,
+                records: bool = True, threads: int = 1):
+    """Trawling (Alg. 4; reading A23): T values, statuses, records."""
+    lib = _load()
+    pr = _Prepared(g, q)
+    t = np.zeros(count, np.float64)
+    st = np.zeros(count, np.uint8)
+    rec = np.zeros(count, TRAWL_DTYPE) if records else None
+
+    def run(a: int, b: int) -> int:
+        return lib.or_trawl_range(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq, _ptr(pr.qrp),
+                                  _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order), int(method), int(seed),
+                                  int(first + a), int(b - a), int(budget), int(filter),
+                                  ctypes.c_void_p(t.ctypes.data + 8 * a), ctypes.c_void_p(st.ctypes.data + a),
+                                  ctypes.c_void_p(rec.ctypes.data + TRAWL_DTYPE.itemsize * a) if records else None)
+
+    if threads <= 1 or count < 2 * threads:
+        rc = run(0, count) if count else 0
+    else:
+        chunk = max(1, min(65536, count // (threads * 8) or 1))
+        bounds = [(a, min(count, a + chunk)) for a in range(0, count, chunk)]
+        with ThreadPoolExecutor(max_workers=threads) as ex:
+            rcs = list(ex.map(lambda ab: run(*ab), bounds))
+        rc = min(rcs) if rcs else 0
+    if rc != 0:
+        raise ValueError(f"oracle rejected input (rc={rc})")
+    return t, st, rec
+
+
+def trawl_aggregate(t: np.ndarray, status: np.ndarray) -> Dict[str, float]:
+    """Trawling estimate: mean of T over the samples whose enumeration finished (the
+    paper keeps only completed enumerations); timeouts reported separately."""
+    done = status != 2
+    agg = aggregate(t[done])
+    agg["n_timeout"] = int(np.count_nonzero(~done))
+    return agg
 
 
 def aggregate(y: np.ndarray) -> Dict[str, float]:

@@ -139,3 +139,42 @@ def is_embedding_prefix(g, q, path) -> bool:
             if q.adj[order[j], order[i]] and path[j] not in adj[v]:
                 return False
     return True
+
+
+def trawl_d_probs(nq: int):
+    """P(d = j) proportional to 2^-j for j in [3, nq]; d = nq when nq <= 3."""
+    if nq <= 3:
+        return {nq: Fraction(1)}
+    w = {j: Fraction(1, 2 ** j) for j in range(3, nq + 1)}
+    z = sum(w.values())
+    return {j: x / z for j, x in w.items()}
+
+
+def trawl_expectation(g, q, method: int, filter: int = 0) -> Fraction:
+    """E[T] of the trawling estimator (Alg. 4) computed exactly: sum over d of P(d) times the
+    sum over sampled prefixes s of length d of P(s) * W(s) * cnt(s), where cnt(s) counts the
+    embeddings whose first d matched vertices are s (brute force)."""
+    order = [int(x) for x in q.order]
+    embs = embeddings(g, q)
+    _, _, cand = tree_walk(g, q, method, filter)
+    adj = _adjacency_sets(g)
+    total = Fraction(0)
+    for d, pd in trawl_d_probs(q.nq).items():
+        # enumerate the sampler's prefixes of length d with their probability and weight
+        stack = [((), Fraction(1), 1)]
+        while stack:
+            prefix, prob, w = stack.pop()
+            if len(prefix) == d:
+                cnt = sum(1 for f in embs if all(f[order[i]] == prefix[i] for i in range(d)))
+                total += pd * prob * w * cnt
+                continue
+            c = cand.get(prefix, ())
+            if not c:
+                continue
+            for v in c:
+                if method == 0 and len(prefix) > 0:  # WanderJoin: Validate the drawn vertex
+                    u = order[len(prefix)]
+                    if v in prefix or any(q.adj[order[j], u] and v not in adj[prefix[j]] for j in range(len(prefix))):
+                        continue
+                stack.append((prefix + (v,), prob / len(c), w * len(c)))
+    return total

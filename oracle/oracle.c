@@ -146,12 +146,14 @@ static int64_t local_candidates(const or_graph* G, int32_t v, const uint8_t* inC
 }
 
 /* ---- one sample (Alg. 1 inner loop) --------------------------------- */
-/* method: 0 = WanderJoin, 1 = Alley.  Returns Y (0 if not a complete instance). */
-static double one_sample(const or_graph* G, const or_query* Q, int method, uint64_t seed, uint64_t sid,
-                         const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
-                         or_record* rec) {
+/* method: 0 = WanderJoin, 1 = Alley.  Samples positions 0 .. stop-1 (stop = |V_q| for
+ * the plain estimator; the trawling prefix length d otherwise).  Returns Y = W if all
+ * `stop` positions were matched, else 0; M and W are left in *Mout / *Wout. */
+static double walk(const or_graph* G, const or_query* Q, int method, uint64_t seed, uint64_t sid, int stop,
+                   const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
+                   or_record* rec, int32_t* Mout, double* Wout) {
     int32_t M[OR_MAX_QV];
-    int nq = Q->nq;
+    int nq = stop;
     double W = 0.0;
     int valid = 0, depth_reached = 0;
     if (rec) {
@@ -227,7 +229,7 @@ static double one_sample(const or_graph* G, const or_query* Q, int method, uint6
             if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
         }
     }
-    /* all |V_q| vertices matched: a complete instance */
+    /* all `stop` positions matched: a complete (partial) instance */
     valid = 1;
     depth_reached = nq - 1;
 done:
@@ -236,7 +238,15 @@ done:
         rec->depth_reached = (uint8_t)depth_reached;
         rec->weight = W;
     }
+    if (Mout) memcpy(Mout, M, sizeof(M));
+    if (Wout) *Wout = W;
     return valid ? W : 0.0;
+}
+
+static double one_sample(const or_graph* G, const or_query* Q, int method, uint64_t seed, uint64_t sid,
+                         const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
+                         or_record* rec) {
+    return walk(G, Q, method, seed, sid, Q->nq, C0, C0_len, inC, S, refine, rec, NULL, NULL);
 }
 
 static int load_query(or_query* Q, int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col,
@@ -384,5 +394,156 @@ int or_count_embeddings(int64_t n, const int64_t* row_ptr, const int32_t* col, c
     *count_hi = (uint64_t)(st.count >> 64);
     return 0;
 }
+
+/* ---- trawling (Alg. 4; NEXT-2, reading A23) --------------------------- */
+typedef struct {
+    uint64_t sample_id;
+    uint8_t status; /* 0 prefix died (T = 0), 1 enumerated, 2 enumeration budget exceeded */
+    uint8_t d;      /* number of sampled vertices */
+    uint8_t pad[6];
+    int32_t path[OR_MAX_QV];
+    uint32_t csize[OR_MAX_QV];
+    double weight;  /* W_d = prod_{j<d} |C_j| (running product) */
+    uint64_t count; /* completions of the sampled partial instance */
+    uint64_t nodes; /* enumeration nodes visited */
+} or_trawl_record; /* 168 bytes */
+
+/* d ~ P(d = j) proportional to 2^-j, j in [3, |V_q|], drawn exactly in integers:
+ * weights 2^(nq-j), total 2^(nq-2) - 1, index = mulhi64(r(sid, 31), total). */
+static int choose_d(uint64_t seed, uint64_t sid, int nq) {
+    if (nq <= 3) return nq;
+    uint64_t total = (1ull << (nq - 2)) - 1ull;
+    uint64_t k = uniform_index(draw_r(seed, sid, 31u), total);
+    uint64_t acc = 0;
+    for (int j = 3; j <= nq; ++j) {
+        acc += 1ull << (nq - j);
+        if (k < acc) return j;
+    }
+    return nq;
+}
+
+typedef struct {
+    const or_graph* G;
+    const or_query* Q;
+    const uint8_t* inC;
+    int32_t M[OR_MAX_QV];
+    int32_t* buf; /* per (level, backward slot) candidate lists */
+    int64_t stride;
+    uint64_t count, nodes, budget;
+    int timeout;
+} trawl_state;
+
+/* Count the completions of M[0..t-1]: every extension keeps a partial instance, so the
+ * candidates at t are the Alley refine set (intersection of the local candidate lists of
+ * the matched query neighbours, minus matched vertices), enumerated in ascending order. */
+static void enumerate_completions(trawl_state* st, int t) {
+    const or_query* Q = st->Q;
+    if (st->timeout) return;
+    if (t == Q->nq) {
+        st->count += 1;
+        return;
+    }
+    int32_t u = Q->order[t];
+    int B[OR_MAX_QV], nb = 0;
+    for (int j = 0; j < t; ++j)
+        if (Q->adj[Q->order[j]][u]) B[nb++] = j;
+    int64_t len[OR_MAX_QV];
+    int32_t* S[OR_MAX_QV];
+    int p = 0;
+    for (int b = 0; b < nb; ++b) {
+        S[b] = st->buf + ((int64_t)t * OR_MAX_QV + b) * st->stride;
+        len[b] = local_candidates(st->G, st->M[B[b]], st->inC + (int64_t)u * st->G->n, S[b]);
+        if (len[b] < len[p]) p = b;
+    }
+    for (int64_t i = 0; i < len[p]; ++i) {
+        int32_t x = S[p][i];
+        int keep = 1;
+        for (int b = 0; b < nb && keep; ++b)
+            if (b != p && !contains(S[b], len[b], x)) keep = 0;
+        for (int j = 0; j < t && keep; ++j)
+            if (st->M[j] == x) keep = 0;
+        if (!keep) continue;
+        if (st->nodes == st->budget) {
+            st->timeout = 1;
+            return;
+        }
+        st->nodes += 1;
+        st->M[t] = x;
+        enumerate_completions(st, t + 1);
+        if (st->timeout) return;
+    }
+}
+
+/* Trawling samples [first, first + count): t_out[i] = T_i = W_d * cnt (0 when the prefix
+ * dies), status_out[i] as or_trawl_record.status, rec_out optional. */
+int or_trawl_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int32_t nq,
+                   const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels, const int32_t* order,
+                   int method, uint64_t seed, uint64_t first, uint64_t count, uint64_t budget, int filter,
+                   double* t_out, uint8_t* status_out, or_trawl_record* rec_out) {
+    or_graph G = {n, row_ptr, col, labels};
+    or_query Q;
+    int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
+    if (rc) return rc;
+    int64_t maxdeg = 0;
+    for (int64_t v = 0; v < n; ++v)
+        if (row_ptr[v + 1] - row_ptr[v] > maxdeg) maxdeg = row_ptr[v + 1] - row_ptr[v];
+    int64_t stride = maxdeg + 1;
+    int32_t* C0 = (int32_t*)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+    int32_t* buf = (int32_t*)malloc(sizeof(int32_t) * (size_t)stride * (OR_MAX_QV + 1));
+    int32_t* ebuf = (int32_t*)malloc(sizeof(int32_t) * (size_t)stride * OR_MAX_QV * OR_MAX_QV);
+    uint8_t* inC = (uint8_t*)malloc((size_t)(n > 0 ? n : 1) * (size_t)nq);
+    if (!C0 || !buf || !ebuf || !inC) { free(C0); free(buf); free(ebuf); free(inC); return -1; }
+    candidate_sets(&G, &Q, filter, inC);
+    int64_t C0_len = 0;
+    const uint8_t* in0 = inC + (int64_t)Q.order[0] * n;
+    for (int64_t v = 0; v < n; ++v)
+        if (in0[v]) C0[C0_len++] = (int32_t)v;
+    int32_t* S[OR_MAX_QV];
+    for (int b = 0; b < OR_MAX_QV; ++b) S[b] = buf + (size_t)b * (size_t)stride;
+    int32_t* refine = buf + (size_t)OR_MAX_QV * (size_t)stride;
+    for (uint64_t i = 0; i < count; ++i) {
+        uint64_t sid = first + i;
+        int d = choose_d(seed, sid, nq);
+        or_record r;
+        trawl_state st;
+        memset(&st, 0, sizeof(st));
+        double W = 0.0;
+        double y = walk(&G, &Q, method, seed, sid, d, C0, C0_len, inC, S, refine, &r, st.M, &W);
+        uint8_t status = 0;
+        double t = 0.0;
+        if (r.valid) {
+            st.G = &G;
+            st.Q = &Q;
+            st.inC = inC;
+            st.buf = ebuf;
+            st.stride = stride;
+            st.budget = budget;
+            enumerate_completions(&st, d);
+            status = st.timeout ? 2 : 1;
+            t = st.timeout ? 0.0 : y * (double)st.count;
+        }
+        if (t_out) t_out[i] = t;
+        if (status_out) status_out[i] = status;
+        if (rec_out) {
+            or_trawl_record* o = &rec_out[i];
+            memset(o, 0, sizeof(*o));
+            o->sample_id = sid;
+            o->status = status;
+            o->d = (uint8_t)d;
+            memcpy(o->path, r.path, sizeof(o->path));
+            memcpy(o->csize, r.csize, sizeof(o->csize));
+            o->weight = W;
+            o->count = st.count;
+            o->nodes = st.nodes;
+        }
+    }
+    free(C0);
+    free(buf);
+    free(ebuf);
+    free(inC);
+    return 0;
+}
+
+int or_trawl_record_size(void) { return (int)sizeof(or_trawl_record); }
 
 int or_record_size(void) { return (int)sizeof(or_record); }

@@ -323,3 +323,67 @@ def test_c0_golden_counts_in_sync(c0):
     assert len(rows) == len(qs)
     for (i, name, cnt), q in zip(rows, qs):
         assert name == q.name and int(cnt) == oracle.count_embeddings(g, q)
+
+
+# ---------------------------------------------------------------- trawling (NEXT-2)
+@pytest.mark.parametrize("seed", range(8))
+@pytest.mark.parametrize("method", [oracle.WJ, oracle.ALLEY])
+def test_trawling_unbiased_exact(seed, method):
+    """E[T] = C, computed exactly with rational probabilities."""
+    g = gen.random_small_graph(7, 0.55, n_labels=1 + seed % 2, seed=1100 + seed)
+    try:
+        q = gen.extract_query(g, 3 + seed % 3, seed=1200 + seed, dense=bool(seed % 2))
+    except RuntimeError:
+        q = gen.random_connected_query(4, 0.5, g.n_labels, 1200 + seed)
+    assert exact.trawl_expectation(g, q, method) == exact.brute_force_count(g, q)
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("method", [oracle.WJ, oracle.ALLEY])
+def test_trawling_records(seed, method):
+    """Every enumerated record's count equals the embeddings extending its prefix."""
+    g = gen.random_small_graph(8, 0.5, n_labels=1 + seed % 2, seed=1300 + seed)
+    try:
+        q = gen.extract_query(g, 4 + seed % 3, seed=1400 + seed, dense=True)
+    except RuntimeError:
+        q = gen.random_connected_query(5, 0.5, g.n_labels, 1400 + seed)
+    embs = exact.embeddings(g, q)
+    order = [int(x) for x in q.order]
+    t, st, rec = oracle.trawl_range(g, q, method, seed, 0, 600)
+    probs = exact.trawl_d_probs(q.nq)
+    for r, tv, s in zip(rec, t, st):
+        d = int(r["d"])
+        assert d in probs
+        if s == 1:
+            prefix = [int(x) for x in r["path"][:d]]
+            cnt = sum(1 for f in embs if all(f[order[i]] == prefix[i] for i in range(d)))
+            assert int(r["count"]) == cnt
+            assert tv == r["weight"] * cnt
+        else:
+            assert s == 0 and tv == 0.0
+
+
+def test_trawling_d_distribution():
+    g = gen.random_small_graph(9, 0.5, 1, seed=5)
+    q = gen.extract_query(g, 6, seed=6, dense=False)
+    _, _, rec = oracle.trawl_range(g, q, oracle.ALLEY, 1, 0, 20_000)
+    probs = exact.trawl_d_probs(q.nq)
+    for d, p in probs.items():
+        frac = float(np.mean(rec["d"] == d))
+        assert abs(frac - float(p)) < 5 * math.sqrt(float(p) * (1 - float(p)) / 20_000)
+
+
+def test_trawling_budget_and_c0(c0):
+    g, qs = c0
+    for q in qs[:5]:
+        truth = oracle.count_embeddings(g, q)
+        t, st, _ = oracle.trawl_range(g, q, oracle.WJ, 3, 0, 50_000, records=False, threads=4)
+        agg = oracle.trawl_aggregate(t, st)
+        assert agg["n_timeout"] == 0
+        assert abs(agg["estimate"] - truth) <= 4 * math.sqrt(agg["variance"]) + 1e-9
+        # a budget of 0 nodes times out every sample that needs enumeration
+        t0, st0, rec0 = oracle.trawl_range(g, q, oracle.WJ, 3, 0, 2000, budget=0)
+        need = (rec0["d"] < q.nq) & (st0 != 0)
+        assert np.all((st0[need] == 2) | (rec0["count"][need] == 0))
+        assert np.any(st0[need] == 2)
+        assert np.all(rec0["nodes"] == 0)
