@@ -81,6 +81,25 @@ typedef struct {
     double weight;
 } gsword_sample_record;
 
+/* One traced trawling sample (168 bytes; gsword_trace_trawl).
+ *   status  0: the sampled prefix died (T = 0); 1: completions enumerated; 2: the node
+ *           budget was exceeded (the sample is left out of the estimate)
+ *   d       number of sampled vertices (positions 0 .. d-1), the rest enumerated
+ *   path/csize/weight as gsword_sample_record for the sampled prefix (W_d)
+ *   count   completions of the prefix (T = weight * count when status == 1)
+ *   nodes   enumeration nodes visited (vertices placed at positions >= d) */
+typedef struct {
+    uint64_t sample_id;
+    uint8_t status;
+    uint8_t d;
+    uint8_t pad[6];
+    int32_t path[GSWORD_MAX_QV];
+    uint32_t csize[GSWORD_MAX_QV];
+    double weight;
+    uint64_t count;
+    uint64_t nodes;
+} gsword_trawl_record;
+
 /* Host-side view of a compiled query plan (for inspection / tests).
  *   back_mask[d]  bit j set iff j < d and (phi[j], phi[d]) is a query edge: B(d)
  *   dup_mask[d]   bit j set iff j < d and L_q(phi[j]) == L_q(phi[d]) (injectivity
@@ -214,6 +233,20 @@ int gsword_estimate_range(gsword_ctx* ctx, gsword_method m, uint64_t first_sampl
  * and by device-side timing.  Counts are exact as fp64 below 2^53. */
 int gsword_estimate_async(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples,
                           uint64_t seed, double* d_out4);
+
+/* Trawling estimator (NEXT-2; Alg. 4; reading A23) over samples
+ * [first, first + n): each sample draws d ~ P(d = j) proportional to 2^-j, j in [3, |V_q|]
+ * (P:L1012), samples positions 0..d-1 with `m` (the same draws as gsword_estimate), counts
+ * every completion exactly with a depth-first enumeration of at most node_budget nodes,
+ * and contributes T = W_d * count (unbiased).  Samples over budget are left out
+ * (P:L1026): out->n_samples counts the finished ones, *n_timeout (may be NULL) the rest;
+ * out->n_valid counts T > 0.  Synchronous. */
+int gsword_trawl_range(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples, uint64_t seed,
+                       uint64_t node_budget, gsword_result* out, uint64_t* n_timeout);
+
+/* Parity entry for trawling: n records in sample-id order.  Synchronous. */
+int gsword_trace_trawl(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples, uint64_t seed,
+                       uint64_t node_budget, gsword_trawl_record* host_out);
 
 /* Host-only: turn 4 aggregated values {sum, sumsq, n_valid, n_samples} into a result. */
 int gsword_finalize(const double* host4, gsword_result* out);

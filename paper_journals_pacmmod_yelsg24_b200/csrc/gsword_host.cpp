@@ -1012,6 +1012,66 @@ int gsword_trace_samples(gsword_ctx* ctx, gsword_method m, uint64_t first, uint6
     return rc;
 }
 
+namespace {
+int run_trawl(gsword_ctx* ctx, int m, uint64_t first, uint64_t n, uint64_t seed, uint64_t budget,
+              gsword_trawl_record* d_rec, double* h4, double* h_timeout) {
+    const int grid = ctx->num_sms * 8;
+    if (grid > ctx->partial_cap) {
+        if (ctx->d_partials) cudaFree(ctx->d_partials);
+        ctx->d_partials = nullptr;
+        CUDA_TRY(cudaMalloc(&ctx->d_partials, sizeof(Partial) * (size_t)grid));
+        ctx->partial_cap = grid;
+    }
+    CUDA_TRY(cudaEventRecord(ctx->evk0, ctx->stream));
+    CUDA_TRY(gsword::launch_trawl(m, d_rec != nullptr, ctx->q_filter != 0, device_graph(ctx), ctx->plan, grid, first,
+                                  n, seed, budget, ctx->d_queue, ctx->d_partials, d_rec, ctx->stream));
+    CUDA_TRY(cudaEventRecord(ctx->evk1, ctx->stream));
+    CUDA_TRY(gsword::launch_reduce(ctx->d_partials, grid, ctx->d_out4, ctx->d_sectors, ctx->stream));
+    CUDA_TRY(cudaMemcpyAsync(h4, ctx->d_out4, 4 * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+    CUDA_TRY(cudaMemcpyAsync(h_timeout, ctx->d_sectors, sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+    CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    return GSWORD_OK;
+}
+}  // namespace
+
+int gsword_trawl_range(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_t n_samples, uint64_t seed,
+                       uint64_t budget, gsword_result* out, uint64_t* n_timeout) {
+    int rc = ensure_ready(ctx, (int)m);
+    if (rc) return rc;
+    if (!out) return fail(GSWORD_EINVAL, "trawl: out NULL");
+    if (n_samples == 0) return fail(GSWORD_EINVAL, "trawl: n_samples must be >= 1");
+    double h[4], to = 0.0;
+    rc = run_trawl(ctx, (int)m, first, n_samples, seed, budget, nullptr, h, &to);
+    if (rc) return rc;
+    gsword_finalize(h, out);
+    float ms = 0.f;
+    CUDA_TRY(cudaEventElapsedTime(&ms, ctx->evk0, ctx->evk1));
+    out->seconds = ms * 1e-3;
+    if (n_timeout) *n_timeout = (uint64_t)to;
+    return GSWORD_OK;
+}
+
+int gsword_trace_trawl(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_t n_samples, uint64_t seed,
+                       uint64_t budget, gsword_trawl_record* host_out) {
+    int rc = ensure_ready(ctx, (int)m);
+    if (rc) return rc;
+    if (!host_out) return fail(GSWORD_EINVAL, "trace_trawl: host_out NULL");
+    if (n_samples == 0) return GSWORD_OK;
+    gsword_trawl_record* d_rec = nullptr;
+    const size_t bytes = sizeof(gsword_trawl_record) * (size_t)n_samples;
+    cudaError_t e = cudaMalloc(&d_rec, bytes);
+    if (e != cudaSuccess) return fail(GSWORD_ENOMEM, "trace_trawl: cudaMalloc(%zu): %s", bytes, cudaGetErrorString(e));
+    CUDA_TRY(cudaMemsetAsync(d_rec, 0, bytes, ctx->stream));
+    double h[4], to = 0.0;
+    rc = run_trawl(ctx, (int)m, first, n_samples, seed, budget, d_rec, h, &to);
+    if (rc == GSWORD_OK) {
+        e = cudaMemcpy(host_out, d_rec, bytes, cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) rc = cuda_fail(e, "trace_trawl: copy back");
+    }
+    cudaFree(d_rec);
+    return rc;
+}
+
 int gsword_count_sectors(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_t n_samples, uint64_t seed,
                          double* sectors_out) {
     int rc = ensure_ready(ctx, (int)m);

@@ -712,6 +712,229 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
     }
 }
 
+// ---------------------------------------------------------------- trawling (NEXT-2)
+// Alg. 4 (reading A23): per sample, d ~ P(d = j) proportional to 2^-j,
+// j in [3, |V_q|], drawn exactly in integers from r(sid, 31); the first d
+// positions are sampled with the method's rules (the same Philox draws as the plain
+// sampler), then every completion is counted by a per-lane depth-first enumeration
+// (ascending candidates, node budget); T = W_d * count.  One lane per sample; samples
+// are taken one at a time from the queue.
+__device__ __forceinline__ int choose_d(uint64_t seed, uint64_t sid, int nq) {
+    if (nq <= 3) return nq;
+    const uint64_t total = (1ull << (nq - 2)) - 1ull;
+    const uint64_t k = __umul64hi(philox_r(seed, sid, 31u), total);
+    uint64_t acc = 0;
+    for (int j = 3; j <= nq; ++j) {
+        acc += 1ull << (nq - j);
+        if (k < acc) return j;
+    }
+    return nq;
+}
+
+template <bool CG>
+__device__ __forceinline__ void getmin_local(const DeviceGraph& g, const PlanStep& ps, const uint8_t (*eidx)[kMaxQV],
+                                             int d, const int32_t* M, uint32_t* lo, uint32_t* len, int* p) {
+    uint32_t bm = ps.back;
+    *len = 0xFFFFFFFFu;
+    while (bm) {
+        const int j = __ffs(bm) - 1;
+        bm &= bm - 1;
+        uint32_t a, b;
+        local_run<CG>(g, eidx[d][j], (uint32_t)M[j], ps.label, &a, &b);
+        if (b - a < *len) {
+            *len = b - a;
+            *lo = a;
+            *p = j;
+        }
+    }
+}
+
+// x (drawn from S_p) extends M[0..d-1] at position d: in every other backward list and
+// not matched (the Alley refine predicate; the enumeration uses it at every level)
+__device__ __forceinline__ bool extends(const DeviceGraph& g, const PlanStep& ps, int p, const int32_t* M, int d,
+                                        int32_t x) {
+    for (int j = 0; j < d; ++j)
+        if (M[j] == x) return false;
+    uint32_t bm = ps.back & ~(1u << p);
+    double sec = 0.0;
+    while (bm) {
+        const int j = __ffs(bm) - 1;
+        bm &= bm - 1;
+        if (!is_edge<false>(g, (uint32_t)M[j], (uint32_t)x, ps.label, sec)) return false;
+    }
+    return true;
+}
+
+template <int METHOD, bool TRACE, bool CG>
+__global__ void __launch_bounds__(128) trawl_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
+                                                    const uint64_t count, const uint64_t seed, const uint64_t budget,
+                                                    unsigned long long* __restrict__ queue,
+                                                    Partial* __restrict__ partials,
+                                                    gsword_trawl_record* __restrict__ records) {
+    __shared__ PlanStep plan_s[kMaxQV];
+    __shared__ uint8_t eidx_s[kMaxQV][kMaxQV];
+    __shared__ Partial warp_part[32];
+    const int tid = threadIdx.x, lane = tid & 31;
+    if (tid < kMaxQV) plan_s[tid] = plan_in.step[tid];
+    if (tid < kMaxQV * kMaxQV) eidx_s[tid / kMaxQV][tid % kMaxQV] = plan_in.eidx[tid / kMaxQV][tid % kMaxQV];
+    __syncthreads();
+    const int nq = plan_in.nq;
+    double s_sum = 0.0, c_sum = 0.0, s_sq = 0.0, c_sq = 0.0, n_timeout = 0.0;
+    unsigned long long n_nonzero = 0, n_done = 0;
+    int32_t M[kMaxQV];
+    uint32_t lvl_lo[kMaxQV], lvl_len[kMaxQV], lvl_i[kMaxQV];
+    int lvl_p[kMaxQV];
+    while (true) {
+        const unsigned long long idx = atomicAdd(queue, 1ull);
+        if (idx >= count) break;
+        const uint64_t sid = first + idx;
+        const int dd = choose_d(seed, sid, nq);
+        gsword_trawl_record* rec = TRACE ? records + idx : nullptr;
+        if (TRACE) {
+            rec->sample_id = sid;
+            rec->d = (uint8_t)dd;
+            for (int i = 0; i < kMaxQV; ++i) {
+                rec->path[i] = -1;
+                rec->csize[i] = 0;
+            }
+        }
+        // ---- sampled prefix: positions 0 .. dd-1 (same rules and draws as the sampler)
+        double W = 0.0;
+        bool alive = true;
+        for (int d = 0; d < dd && alive; ++d) {
+            const PlanStep ps = plan_s[d];
+            const uint64_t r = philox_r(seed, sid, (uint32_t)d);
+            uint32_t lo = 0, len = 0, cnt = 0;
+            int p = 0;
+            int32_t v = -1;
+            if (d == 0) {
+                lo = plan_in.seed_lo;
+                cnt = len = plan_in.seed_len;
+                if (cnt > 0) {
+                    const uint64_t k = __umul64hi(r, (uint64_t)cnt);
+                    v = plan_in.seed_identity ? (int32_t)(lo + k) : __ldg(g.bucket + lo + k);
+                }
+            } else {
+                getmin_local<CG>(g, ps, eidx_s, d, M, &lo, &len, &p);
+                if (METHOD == GSWORD_WJ) {
+                    cnt = len;
+                    if (cnt > 0) {
+                        v = __ldg(g.clist + lo + __umul64hi(r, (uint64_t)cnt));
+                    }
+                } else {
+                    for (uint32_t i = 0; i < len; ++i) cnt += extends(g, ps, p, M, d, __ldg(g.clist + lo + i)) ? 1u : 0u;
+                    if (cnt > 0) {
+                        uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
+                        for (uint32_t i = 0; i < len; ++i) {
+                            const int32_t x = __ldg(g.clist + lo + i);
+                            if (!extends(g, ps, p, M, d, x)) continue;
+                            if (k == 0) {
+                                v = x;
+                                break;
+                            }
+                            --k;
+                        }
+                    }
+                }
+            }
+            W = (d == 0) ? (double)cnt : __dmul_rn(W, (double)cnt);
+            if (TRACE) {
+                rec->csize[d] = cnt;
+                rec->path[d] = cnt > 0 ? v : -1;
+            }
+            if (cnt == 0) {
+                alive = false;
+                break;
+            }
+            if (METHOD == GSWORD_WJ && d > 0 && !extends(g, ps, p, M, d, v)) alive = false;  // Validate
+            M[d] = v;
+        }
+        // ---- enumeration of positions dd .. nq-1
+        unsigned long long cnt_all = 0, nodes = 0;
+        bool timeout = false;
+        if (alive) {
+            if (dd == nq) {
+                cnt_all = 1;
+            } else {
+                int t = dd;
+                getmin_local<CG>(g, plan_s[t], eidx_s, t, M, &lvl_lo[t], &lvl_len[t], &lvl_p[t]);
+                lvl_i[t] = 0;
+                while (t >= dd) {
+                    if (lvl_i[t] >= lvl_len[t]) {  // level exhausted: back to the parent's next candidate
+                        --t;
+                        if (t >= dd) ++lvl_i[t];
+                        continue;
+                    }
+                    const int32_t x = __ldg(g.clist + lvl_lo[t] + lvl_i[t]);
+                    if (!extends(g, plan_s[t], lvl_p[t], M, t, x)) {
+                        ++lvl_i[t];
+                        continue;
+                    }
+                    if (nodes == budget) {
+                        timeout = true;
+                        break;
+                    }
+                    ++nodes;
+                    M[t] = x;
+                    if (t + 1 == nq) {
+                        ++cnt_all;
+                        ++lvl_i[t];
+                    } else {
+                        ++t;
+                        getmin_local<CG>(g, plan_s[t], eidx_s, t, M, &lvl_lo[t], &lvl_len[t], &lvl_p[t]);
+                        lvl_i[t] = 0;
+                    }
+                }
+            }
+        }
+        const uint8_t status = !alive ? 0 : (timeout ? 2 : 1);
+        if (TRACE) {
+            rec->status = status;
+            rec->weight = W;
+            rec->count = cnt_all;
+            rec->nodes = nodes;
+        }
+        if (status == 2) {
+            n_timeout += 1.0;
+        } else {
+            n_done += 1;
+            if (status == 1 && cnt_all > 0) {
+                const double T = __dmul_rn(W, (double)cnt_all);
+                n_nonzero += 1;
+                nsum(s_sum, c_sum, T);
+                nsum(s_sq, c_sq, __dmul_rn(T, T));
+            }
+        }
+    }
+    // block partial (fixed order); timeouts ride in the `sectors` slot
+    double sh = __dadd_rn(s_sum, c_sum), sl = __dsub_rn(c_sum, __dsub_rn(sh, s_sum));
+    double qh = __dadd_rn(s_sq, c_sq), ql = __dsub_rn(c_sq, __dsub_rn(qh, s_sq));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const double bh = shfl_xor_d(sh, o), bl = shfl_xor_d(sl, o);
+        const double ch = shfl_xor_d(qh, o), cl = shfl_xor_d(ql, o);
+        dd_add(sh, sl, bh, bl);
+        dd_add(qh, ql, ch, cl);
+        n_nonzero += __shfl_xor_sync(kFull, n_nonzero, o);
+        n_done += __shfl_xor_sync(kFull, n_done, o);
+        n_timeout += shfl_xor_d(n_timeout, o);
+    }
+    if (lane == 0) warp_part[tid >> 5] = Partial{sh, sl, qh, ql, n_nonzero, n_done, n_timeout, 0.0};
+    __syncthreads();
+    if (tid == 0) {
+        Partial acc = warp_part[0];
+        for (int w = 1; w < (int)(blockDim.x >> 5); ++w) {
+            const Partial& o = warp_part[w];
+            dd_add(acc.sum_hi, acc.sum_lo, o.sum_hi, o.sum_lo);
+            dd_add(acc.sq_hi, acc.sq_lo, o.sq_hi, o.sq_lo);
+            acc.valid += o.valid;
+            acc.n += o.n;
+            acc.sectors += o.sectors;
+        }
+        partials[blockIdx.x] = acc;
+    }
+}
+
 // Grid reduction in CTA order (one warp; lane-strided then a fixed butterfly).
 __global__ void reduce_kernel(const Partial* __restrict__ partials, int n, double* __restrict__ out4,
                               double* __restrict__ sectors_out) {
@@ -1042,6 +1265,24 @@ cudaError_t launch_scan(uint32_t* data, int64_t n, const unsigned long long* d_b
     scan_local_kernel<<<(unsigned)nb, kScanThreads, 0, stream>>>(data, n, d_tmp);
     scan_sums_kernel<<<1, kScanThreads, 0, stream>>>(d_tmp, nb, d_base, d_total);
     scan_add_kernel<<<(unsigned)nb, kScanThreads, 0, stream>>>(data, n, d_tmp);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_trawl(int method, bool trace, bool cg, const DeviceGraph& g, const Plan& plan, int grid,
+                         uint64_t first, uint64_t count, uint64_t seed, uint64_t budget, unsigned long long* d_queue,
+                         Partial* d_partials, gsword_trawl_record* d_records, cudaStream_t stream) {
+    cudaError_t e = cudaMemsetAsync(d_queue, 0, sizeof(unsigned long long), stream);
+    if (e != cudaSuccess) return e;
+#define GSWORD_TRAWL(M, TR, CGF) \
+    trawl_kernel<M, TR, CGF><<<grid, 128, 0, stream>>>(g, plan, first, count, seed, budget, d_queue, d_partials, d_records)
+    if (method == GSWORD_WJ) {
+        if (trace) { if (cg) GSWORD_TRAWL(GSWORD_WJ, true, true); else GSWORD_TRAWL(GSWORD_WJ, true, false); }
+        else { if (cg) GSWORD_TRAWL(GSWORD_WJ, false, true); else GSWORD_TRAWL(GSWORD_WJ, false, false); }
+    } else {
+        if (trace) { if (cg) GSWORD_TRAWL(GSWORD_ALLEY, true, true); else GSWORD_TRAWL(GSWORD_ALLEY, true, false); }
+        else { if (cg) GSWORD_TRAWL(GSWORD_ALLEY, false, true); else GSWORD_TRAWL(GSWORD_ALLEY, false, false); }
+    }
+#undef GSWORD_TRAWL
     return cudaGetLastError();
 }
 

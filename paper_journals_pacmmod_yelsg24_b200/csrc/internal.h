@@ -119,6 +119,9 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
 cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_out4, double* d_sectors,
                           cudaStream_t stream);
 cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream);
+cudaError_t launch_trawl(int method, bool trace, bool cg, const DeviceGraph& g, const Plan& plan, int grid,
+                         uint64_t first, uint64_t count, uint64_t seed, uint64_t budget, unsigned long long* d_queue,
+                         Partial* d_partials, gsword_trawl_record* d_records, cudaStream_t stream);
 // candidate graph build (NEXT-1)
 cudaError_t launch_filter(const DeviceGraph& g, const QFilter* d_qf, int nq, int filter, uint32_t* cbits,
                           const int32_t* d_vlabel, cudaStream_t stream);

@@ -43,6 +43,14 @@ RECORD_DTYPE = np.dtype([
 ])
 assert RECORD_DTYPE.itemsize == 152
 
+# gsword_trawl_record (168 bytes)
+TRAWL_DTYPE = np.dtype([
+    ("sample_id", "<u8"), ("status", "u1"), ("d", "u1"), ("pad", "u1", (6,)),
+    ("path", "<i4", (MAX_QV,)), ("csize", "<u4", (MAX_QV,)), ("weight", "<f8"), ("count", "<u8"),
+    ("nodes", "<u8"),
+])
+assert TRAWL_DTYPE.itemsize == 168
+
 
 class GswordError(RuntimeError):
     def __init__(self, status: int, message: str):
@@ -91,6 +99,8 @@ def _load_library() -> ctypes.CDLL:
         "gsword_phase_cycles": ([P, P], ctypes.c_int),
         "gsword_query_info": ([P, ctypes.POINTER(_QueryStats)], ctypes.c_int),
         "gsword_quicksi_order": ([I64, P, P, P, I32, I32, P, P, P, P], ctypes.c_int),
+        "gsword_trawl_range": ([P, ctypes.c_int, U64, U64, U64, U64, ctypes.POINTER(_Result), P], ctypes.c_int),
+        "gsword_trace_trawl": ([P, ctypes.c_int, U64, U64, U64, U64, P], ctypes.c_int),
         "gsword_select_order": ([P, ctypes.c_int, ctypes.c_int, I32, P, P, P, U64, U64, P, P], ctypes.c_int),
         "gsword_check_graph": ([I64, P, P, P, I32], ctypes.c_int),
         "gsword_plan_query": ([I32, P, P, P, P, I32, ctypes.POINTER(_PlanInfo)], ctypes.c_int),
@@ -293,6 +303,22 @@ class Context:
         ptr = out4.data_ptr() if hasattr(out4, "data_ptr") else int(out4)
         _check(_lib.gsword_estimate_async(self._h, int(method), int(first), int(n_samples), int(seed),
                                           ctypes.c_void_p(ptr)))
+
+    def trawl(self, method: int, n_samples: int, seed: int, first: int = 0, node_budget: int = 2**62):
+        """gsword_trawl_range: trawling estimate (Alg. 4) over [first, first+n)."""
+        r = _Result()
+        to = ctypes.c_uint64()
+        _check(_lib.gsword_trawl_range(self._h, int(method), int(first), int(n_samples), int(seed),
+                                       int(node_budget), ctypes.byref(r), ctypes.byref(to)))
+        out = _result_dict(r)
+        out["n_timeout"] = int(to.value)
+        return out
+
+    def trace_trawl(self, method: int, first: int, n_samples: int, seed: int, node_budget: int = 2**62):
+        rec = np.zeros(int(n_samples), TRAWL_DTYPE)
+        _check(_lib.gsword_trace_trawl(self._h, int(method), int(first), int(n_samples), int(seed),
+                                       int(node_budget), _ptr(rec)))
+        return rec
 
     def trace_samples(self, method: int, first: int, n_samples: int, seed: int) -> np.ndarray:
         rec = np.zeros(int(n_samples), RECORD_DTYPE)

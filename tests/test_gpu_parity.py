@@ -393,3 +393,49 @@ def test_order_selection_trial_matches_oracle(ctx, G, c0, method):
         assert r["sum"] == pytest.approx(ref["sum"], rel=1e-12)
         o2, _ = ctx.select_order(G.ORDER_QUICKSI, method, qrp, qcol, q.labels)
         assert o2 == qo
+
+
+# ------------------------------------------------------------------ NEXT-2: trawling
+def _trawl_parity(ctx, G, g, q, method, seed, first, count, budget, filt=0, threads=8):
+    ctx.load_query_obj(q)
+    rec = ctx.trace_trawl(method, first, count, seed, budget)
+    t, st, ref = oracle.trawl_range(g, q, method, seed, first, count, budget=budget, filter=filt, threads=threads)
+    assert rec.tobytes() == ref.tobytes(), f"trawl records differ ({q.name}, m{method}, budget {budget})"
+    r = ctx.trawl(method, count, seed, first=first, node_budget=budget)
+    agg = oracle.trawl_aggregate(t, st)
+    assert r["n_timeout"] == agg["n_timeout"] and r["n"] == agg["n"] and r["n_valid"] == agg["n_valid"]
+    assert r["sum"] == pytest.approx(agg["sum"], rel=REL)
+    assert r["sumsq"] == pytest.approx(agg["sumsq"], rel=REL)
+
+
+@pytest.mark.parametrize("method", [0, 1])
+def test_trawl_parity(ctx, G, c0, method):
+    for seed in range(6):
+        g = gen.random_small_graph(12 + seed, 0.4, 1 + seed % 3, seed=2000 + seed)
+        try:
+            q = gen.extract_query(g, 4 + seed % 3, seed=2100 + seed, dense=bool(seed % 2))
+        except RuntimeError:
+            q = gen.random_connected_query(4, 0.5, g.n_labels, 2100 + seed)
+        ctx.load_graph_obj(g)
+        for budget in (2**62, 3, 0):
+            _trawl_parity(ctx, G, g, q, method, seed, 17, 2000, budget)
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    for q in qs:
+        _trawl_parity(ctx, G, g, q, method, 5, 0, 20_000, 2**62)
+        truth = oracle.count_embeddings(g, q)
+        r = ctx.trawl(method, 1_000_000, 8)
+        assert abs(r["estimate"] - truth) <= 5 * math.sqrt(max(r["variance"], 0.0)) + 1e-9
+
+
+def test_trawl_parity_c2_and_filter(ctx, G):
+    g, qs = gen.config_c2()
+    ctx.load_graph_obj(g)
+    for filt in (0, 2):
+        ctx.set_option(G.OPT_FILTER, filt)
+        try:
+            for q in qs:
+                for m in (0, 1):
+                    _trawl_parity(ctx, G, g, q, m, 3, 0, 5000, 100_000, filt=filt, threads=16)
+        finally:
+            ctx.set_option(G.OPT_FILTER, 0)
