@@ -80,6 +80,9 @@ class Query:
     def with_order(self, order: Sequence[int]) -> "Query":
         return Query(self.adj.copy(), self.labels.copy(), np.asarray(order, np.int32), self.name)
 
+    def _renamed(self, name: str) -> "Query":
+        return Query(self.adj, self.labels, self.order, name)
+
 
 # --------------------------------------------------------------------------
 # CSR construction
@@ -227,11 +230,14 @@ def kronecker(scale: int, n_edges_target: int, seed: int, abcd=(0.57, 0.19, 0.19
     keys = np.zeros(0, np.int64)
     while keys.shape[0] < n_edges_target:
         need = n_edges_target - keys.shape[0]
-        pu, pv = draw_pairs(rng, int(need * 1.3) + 1024)
-        ok = pu != pv
-        pu, pv = pu[ok], pv[ok]
-        k = np.minimum(pu, pv) * n + np.maximum(pu, pv)
-        keys = _sorted_unique(np.concatenate([keys, k]))
+        total = int(need * 1.3) + 1024
+        parts = []
+        for c0 in range(0, total, 1 << 24):  # bounded memory per chunk
+            pu, pv = draw_pairs(rng, min(1 << 24, total - c0))
+            ok = pu != pv
+            pu, pv = pu[ok], pv[ok]
+            parts.append(_sorted_unique(np.minimum(pu, pv) * n + np.maximum(pu, pv)))
+        keys = _sorted_unique(np.concatenate([keys] + parts))
     if keys.shape[0] > n_edges_target:
         keys = keys[np.sort(rng.choice(keys.shape[0], size=n_edges_target, replace=False))]
     labels = uniform_labels(n, n_labels, labels_seed) if n_labels > 1 else None
@@ -489,4 +495,29 @@ def config_c3() -> Tuple[Graph, List[Query]]:
     return g, qs
 
 
-CONFIGS = {"C0": config_c0, "C1": config_c1, "C2": config_c2, "C3": config_c3}
+def star_query_from(g: Graph, s: int, seed: int) -> Query:
+    """K_{1,s} labelled from a data vertex of degree >= s and s of its neighbours."""
+    rng = np.random.default_rng(seed)
+    deg = g.degree()
+    cand = np.nonzero(deg >= s)[0]
+    v = int(cand[rng.integers(cand.shape[0])])
+    nb = rng.choice(g.neighbors(v), size=s, replace=False)
+    labels = [int(g.labels[v])] + [int(g.labels[w]) for w in nb]
+    return star_query(s, labels).with_order(list(range(s + 1)))._renamed(f"star{s}_s{seed}")
+
+
+def config_c4(scale: int = 23, n_edges: int = 100_000_000, sizes=(4, 6, 8, 10, 12, 14, 16)):
+    """C4: Graph500 Kronecker (0.57, 0.19, 0.19, 0.05), 2^scale vertices, exactly n_edges
+    undirected edges, random vertex permutation (seed 500), 16 uniform labels (seed 16);
+    queries: for each size k a labelled path (sparse) and a dense random-walk query, plus
+    labelled stars K_{1,3..5} (exact counts by closed form)."""
+    g = kronecker(scale, n_edges, seed=500, n_labels=16, labels_seed=16, name=f"C4_kron{scale}")
+    qs = []
+    for k in sizes:
+        qs.append(extract_query(g, k, seed=4000 + k, dense=False))
+        qs.append(extract_query(g, k, seed=5000 + k, dense=True, require_dense=True))
+    qs += [star_query_from(g, s, 6000 + s) for s in (3, 4, 5)]
+    return g, qs
+
+
+CONFIGS = {"C0": config_c0, "C1": config_c1, "C2": config_c2, "C3": config_c3, "C4": config_c4}
