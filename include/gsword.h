@@ -135,6 +135,12 @@ typedef enum {
     GSWORD_OPT_BLOOM = 5,          /* 1 = edge Bloom pre-test (L2-resident filter)    */
     GSWORD_OPT_EDGE_SET = 6,       /* 1 = exact edge hash set for adjacency tests;    */
                                    /* 0 = binary search in the adjacency run          */
+    GSWORD_OPT_SCHEDULE = 8,       /* 0 refill free lanes every round (default);      */
+                                   /* 1 sample synchronisation (comparison);  */
+                                   /* 2 = 1 + sample inheritance (Alg. 2, NEXT-3,     */
+                                   /*   reading A24; estimates only, no traces; the   */
+                                   /*   variance uses groups of 32 ids; sumsq of the  */
+                                   /*   async output holds squared group totals)      */
     GSWORD_OPT_FILTER = 7          /* candidate filter applied by the next            */
                                    /* gsword_load_query: 0 label only, 1 LDF, 2 NLF   */
                                    /* (1-2 build the candidate graph, reading A21)    */

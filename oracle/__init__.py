@@ -85,6 +85,9 @@ def _load():
             lib.or_trawl_range.restype = ctypes.c_int
             lib.or_trawl_record_size.restype = ctypes.c_int
             assert lib.or_trawl_record_size() == TRAWL_DTYPE.itemsize
+            lib.or_inherit_range.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, ctypes.c_int,
+                                             ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_int, P, P]
+            lib.or_inherit_range.restype = ctypes.c_int
             lib.or_count_embeddings.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, P, P]
             lib.or_count_embeddings.restype = ctypes.c_int
             lib.or_record_size.restype = ctypes.c_int
@@ -199,6 +202,28 @@ def trawl_range(g, q, method: int, seed: int, first: int, count: int, budget: in
     if rc != 0:
         raise ValueError(f"oracle rejected input (rc={rc})")
     return t, st, rec
+
+
+def inherit_range(g, q, method: int, seed: int, first: int, count: int, filter: int = 0) -> Dict[str, float]:
+    """Sample inheritance (Alg. 2) over groups of 32 consecutive ids (reading A24).
+    estimate = sum of group totals / count; variance from the group totals (the groups are
+    the independent units): m (sum G^2 - (sum G)^2 / m) / ((m - 1) count^2)."""
+    lib = _load()
+    pr = _Prepared(g, q)
+    m = (count + 31) // 32
+    groups = np.zeros(max(m, 1), np.float64)
+    nc = np.zeros(1, np.uint64)
+    rc = lib.or_inherit_range(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq, _ptr(pr.qrp),
+                              _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order), int(method), int(seed), int(first),
+                              int(count), int(filter), _ptr(groups), _ptr(nc))
+    if rc != 0:
+        raise ValueError(f"oracle rejected input (rc={rc})")
+    groups = groups[:m]
+    s = math.fsum(groups.tolist())
+    sq = math.fsum((groups * groups).tolist())
+    var = m * (sq - s * s / m) / ((m - 1) * count * count) if m >= 2 else float("nan")
+    return {"sum": s, "sumsq": sq, "n": count, "groups": m, "n_valid": int(nc[0]), "estimate": s / count,
+            "variance": var, "group_totals": groups}
 
 
 def trawl_aggregate(t: np.ndarray, status: np.ndarray) -> Dict[str, float]:

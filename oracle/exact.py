@@ -178,3 +178,8 @@ def trawl_expectation(g, q, method: int, filter: int = 0) -> Fraction:
                         continue
                 stack.append((prefix + (v,), prob / len(c), w * len(c)))
     return total
+
+
+def inheritance_expectation_check(g, q, method, seed_values, count, inherit_fn):
+    """Helper for tests: mean of the inheritance estimator over several seeds."""
+    return [inherit_fn(g, q, method, s, 0, count)["estimate"] for s in seed_values]

@@ -146,93 +146,99 @@ static int64_t local_candidates(const or_graph* G, int32_t v, const uint8_t* inC
 }
 
 /* ---- one sample (Alg. 1 inner loop) --------------------------------- */
-/* method: 0 = WanderJoin, 1 = Alley.  Samples positions 0 .. stop-1 (stop = |V_q| for
- * the plain estimator; the trawling prefix length d otherwise).  Returns Y = W if all
- * `stop` positions were matched, else 0; M and W are left in *Mout / *Wout. */
+/* One position d of a sample (method 0 = WanderJoin, 1 = Alley): forms C_d from the
+ * matched prefix M[0..d-1], draws M[d] with r(sid, d), multiplies *W by |C_d| (the running
+ * product of Eq. 1 in depth order, reading A7; *W starts as |C_0| at d = 0) and validates.
+ * Returns 1 if M[0..d] is still a valid partial instance, 0 if the sample died here. */
+static int step_at(const or_graph* G, const or_query* Q, int method, uint64_t seed, uint64_t sid, int d,
+                   const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
+                   int32_t* M, double* W, or_record* rec) {
+    if (d == 0) {
+        /* seed from the global candidate set C(phi[0]) */
+        *W = (double)C0_len;
+        if (C0_len == 0) return 0;
+        uint64_t k = uniform_index(draw_r(seed, sid, 0), (uint64_t)C0_len);
+        M[0] = C0[k];
+        if (rec) { rec->path[0] = M[0]; rec->csize[0] = (uint32_t)C0_len; }
+        return 1;
+    }
+    int32_t u = Q->order[d];
+    /* backward positions B(d) = { j < d : (phi[j], phi[d]) in E_q } */
+    int B[OR_MAX_QV], nb = 0;
+    for (int j = 0; j < d; ++j)
+        if (Q->adj[Q->order[j]][u]) B[nb++] = j;
+    /* GetMinCandidate (Alg. 1 l.8): local lists S_j of every matched neighbour,
+     * p = the smallest one, ties -> smallest position j (reading A3) */
+    int64_t len[OR_MAX_QV];
+    int p = 0;
+    for (int b = 0; b < nb; ++b) {
+        len[b] = local_candidates(G, M[B[b]], inC + (int64_t)u * G->n, S[b]);
+        if (len[b] < len[p]) p = b;
+    }
+    int64_t clen;
+    const int32_t* cand = S[p];
+    if (method == 0) {
+        /* WanderJoin Refine: refine = cand (Fig. 19 WJ) */
+        clen = len[p];
+        *W = *W * (double)clen;
+        if (clen == 0) return 0;
+        /* Sample: uniform vertex of refine, prob 1/rlen */
+        uint64_t k = uniform_index(draw_r(seed, sid, (uint32_t)d), (uint64_t)clen);
+        int32_t v = cand[k];
+        M[d] = v;
+        if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
+        /* Validate: DupCheck against all matched vertices, IsEdge for every other
+         * matched query neighbour */
+        for (int j = 0; j < d; ++j)
+            if (M[j] == v) return 0;
+        for (int b = 0; b < nb; ++b) {
+            if (b == p) continue;
+            if (!contains(S[b], len[b], v)) return 0;
+        }
+        return 1;
+    }
+    /* Alley Refine: keep each x of cand that lies in every other local list and is not
+     * already matched (Fig. 19 AL; reading A5) */
+    clen = 0;
+    for (int64_t i = 0; i < len[p]; ++i) {
+        int32_t x = cand[i];
+        int keep = 1;
+        for (int b = 0; b < nb && keep; ++b) {
+            if (b == p) continue;
+            if (!contains(S[b], len[b], x)) keep = 0;
+        }
+        for (int j = 0; j < d && keep; ++j)
+            if (M[j] == x) keep = 0;
+        if (keep) refine[clen++] = x;
+    }
+    *W = *W * (double)clen;
+    /* empty refined set: the sample stops */
+    if (clen == 0) return 0;
+    uint64_t k = uniform_index(draw_r(seed, sid, (uint32_t)d), (uint64_t)clen);
+    int32_t v = refine[k];
+    M[d] = v;
+    if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
+    return 1;
+}
+
+/* Samples positions 0 .. stop-1 (stop = |V_q| for the plain estimator; the trawling
+ * prefix length d otherwise).  Returns Y = W if all `stop` positions were matched, else 0;
+ * M and W are left in *Mout / *Wout. */
 static double walk(const or_graph* G, const or_query* Q, int method, uint64_t seed, uint64_t sid, int stop,
                    const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
                    or_record* rec, int32_t* Mout, double* Wout) {
     int32_t M[OR_MAX_QV];
-    int nq = stop;
     double W = 0.0;
-    int valid = 0, depth_reached = 0;
+    int valid = 1, depth_reached = 0;
     if (rec) {
         memset(rec, 0, sizeof(*rec));
         rec->sample_id = sid;
         for (int i = 0; i < OR_MAX_QV; ++i) rec->path[i] = -1;
     }
-    /* d = 0: seed from the global candidate set C(phi[0]).  W is the running
-     * product prod |C_d| (Eq. 1), taken in depth order (reading A7). */
-    W = (double)C0_len;
-    if (C0_len == 0) goto done;
-    {
-        uint64_t k = uniform_index(draw_r(seed, sid, 0), (uint64_t)C0_len);
-        M[0] = C0[k];
-        if (rec) { rec->path[0] = M[0]; rec->csize[0] = (uint32_t)C0_len; }
-    }
-    for (int d = 1; d < nq; ++d) {
+    for (int d = 0; d < stop && valid; ++d) {
         depth_reached = d;
-        int32_t u = Q->order[d];
-        /* backward positions B(d) = { j < d : (phi[j], phi[d]) in E_q } */
-        int B[OR_MAX_QV], nb = 0;
-        for (int j = 0; j < d; ++j)
-            if (Q->adj[Q->order[j]][u]) B[nb++] = j;
-        /* GetMinCandidate (Alg. 1 l.8): local lists S_j of every matched neighbour,
-         * p = the smallest one, ties -> smallest position j (reading A3) */
-        int64_t len[OR_MAX_QV];
-        int p = 0;
-        for (int b = 0; b < nb; ++b) {
-            len[b] = local_candidates(G, M[B[b]], inC + (int64_t)u * G->n, S[b]);
-            if (len[b] < len[p]) p = b;
-        }
-        int64_t clen;
-        const int32_t* cand = S[p];
-        if (method == 0) {
-            /* WanderJoin Refine: refine = cand (Fig. 19 WJ) */
-            clen = len[p];
-            W = W * (double)clen;
-            if (clen == 0) goto done;
-            /* Sample: uniform vertex of refine, prob 1/rlen */
-            uint64_t k = uniform_index(draw_r(seed, sid, (uint32_t)d), (uint64_t)clen);
-            int32_t v = cand[k];
-            M[d] = v;
-            if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
-            /* Validate: DupCheck against all matched vertices, IsEdge for every other
-             * matched query neighbour */
-            for (int j = 0; j < d; ++j)
-                if (M[j] == v) goto done;
-            for (int b = 0; b < nb; ++b) {
-                if (b == p) continue;
-                if (!contains(S[b], len[b], v)) goto done;
-            }
-        } else {
-            /* Alley Refine: keep each x of cand that lies in every other local list and
-             * is not already matched (Fig. 19 AL; reading A5) */
-            clen = 0;
-            for (int64_t i = 0; i < len[p]; ++i) {
-                int32_t x = cand[i];
-                int keep = 1;
-                for (int b = 0; b < nb && keep; ++b) {
-                    if (b == p) continue;
-                    if (!contains(S[b], len[b], x)) keep = 0;
-                }
-                for (int j = 0; j < d && keep; ++j)
-                    if (M[j] == x) keep = 0;
-                if (keep) refine[clen++] = x;
-            }
-            W = W * (double)clen;
-            /* empty refined set: the sample stops */
-            if (clen == 0) goto done;
-            uint64_t k = uniform_index(draw_r(seed, sid, (uint32_t)d), (uint64_t)clen);
-            int32_t v = refine[k];
-            M[d] = v;
-            if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
-        }
+        valid = step_at(G, Q, method, seed, sid, d, C0, C0_len, inC, S, refine, M, &W, rec);
     }
-    /* all `stop` positions matched: a complete (partial) instance */
-    valid = 1;
-    depth_reached = nq - 1;
-done:
     if (rec) {
         rec->valid = (uint8_t)valid;
         rec->depth_reached = (uint8_t)depth_reached;
@@ -545,5 +551,85 @@ int or_trawl_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const 
 }
 
 int or_trawl_record_size(void) { return (int)sizeof(or_trawl_record); }
+
+/* ---- sample inheritance (Alg. 2; NEXT-3, reading A24) ------------------- */
+/* Groups of 32 consecutive sample ids [first + 32g, first + 32g + 32) run in lock step, one
+ * position per round (sample synchronisation).  After a round that is not the last,
+ * if some group members hold a valid partial sample and others do not, every member without
+ * one inherits the valid sample of the lowest such member (the parent, Alg. 2 l.2), and the
+ * parent and its k copies all carry W / (k + 1) (the push-down of the recursive estimator,
+ * P:L902-L910).  A copy keeps drawing with its own sample id.  group_out[g] = the sum of
+ * the weights of the complete instances of group g; *n_complete counts those instances. */
+int or_inherit_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int32_t nq,
+                     const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels, const int32_t* order,
+                     int method, uint64_t seed, uint64_t first, uint64_t count, int filter, double* group_out,
+                     uint64_t* n_complete) {
+    or_graph G = {n, row_ptr, col, labels};
+    or_query Q;
+    int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
+    if (rc) return rc;
+    int64_t maxdeg = 0;
+    for (int64_t v = 0; v < n; ++v)
+        if (row_ptr[v + 1] - row_ptr[v] > maxdeg) maxdeg = row_ptr[v + 1] - row_ptr[v];
+    int64_t stride = maxdeg + 1;
+    int32_t* C0 = (int32_t*)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+    int32_t* buf = (int32_t*)malloc(sizeof(int32_t) * (size_t)stride * (OR_MAX_QV + 1));
+    uint8_t* inC = (uint8_t*)malloc((size_t)(n > 0 ? n : 1) * (size_t)nq);
+    if (!C0 || !buf || !inC) { free(C0); free(buf); free(inC); return -1; }
+    candidate_sets(&G, &Q, filter, inC);
+    int64_t C0_len = 0;
+    const uint8_t* in0 = inC + (int64_t)Q.order[0] * n;
+    for (int64_t v = 0; v < n; ++v)
+        if (in0[v]) C0[C0_len++] = (int32_t)v;
+    int32_t* S[OR_MAX_QV];
+    for (int b = 0; b < OR_MAX_QV; ++b) S[b] = buf + (size_t)b * (size_t)stride;
+    int32_t* refine = buf + (size_t)OR_MAX_QV * (size_t)stride;
+    uint64_t completes = 0;
+    uint64_t g = 0;
+    for (uint64_t g0 = 0; g0 < count; g0 += 32, ++g) {
+        int L = (int)((count - g0) < 32 ? (count - g0) : 32);
+        int32_t M[32][OR_MAX_QV];
+        double W[32];
+        int alive[32];
+        double total = 0.0;
+        for (int l = 0; l < L; ++l) alive[l] = 1;
+        for (int d = 0; d < nq; ++d) {
+            int any = 0;
+            for (int l = 0; l < L; ++l) {
+                if (!alive[l]) continue;
+                alive[l] = step_at(&G, &Q, method, seed, first + g0 + (uint64_t)l, d, C0, C0_len, inC, S, refine,
+                                   M[l], &W[l], NULL);
+                any |= alive[l];
+            }
+            if (!any) break;
+            if (d == nq - 1) {
+                for (int l = 0; l < L; ++l)
+                    if (alive[l]) { total += W[l]; completes += 1; }
+                break;
+            }
+            int parent = -1, k = 0;
+            for (int l = 0; l < L; ++l) {
+                if (alive[l] && parent < 0) parent = l;
+                if (!alive[l]) k += 1;
+            }
+            if (k > 0) {
+                double Wn = W[parent] / (double)(k + 1);
+                W[parent] = Wn;
+                for (int l = 0; l < L; ++l) {
+                    if (alive[l]) continue;
+                    memcpy(M[l], M[parent], sizeof(int32_t) * (size_t)(d + 1));
+                    W[l] = Wn;
+                    alive[l] = 1;
+                }
+            }
+        }
+        group_out[g] = total;
+    }
+    *n_complete = completes;
+    free(C0);
+    free(buf);
+    free(inC);
+    return 0;
+}
 
 int or_record_size(void) { return (int)sizeof(or_record); }

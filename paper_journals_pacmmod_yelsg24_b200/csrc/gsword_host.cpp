@@ -250,6 +250,7 @@ struct gsword_ctx {
     int opt_l2 = 0;
     int opt_coop = 64;
     int opt_bloom = 1;
+    int opt_sched = 0;
     int opt_eset = 1;
     // last launch
     int last_grid = 0, last_threads = 0;
@@ -324,8 +325,9 @@ int launch_config(gsword_ctx* ctx, int method, int mode, LaunchCfg* cfg) {
     const int bps = ctx->opt_blocks_per_sm > 0 ? std::min(ctx->opt_blocks_per_sm, occ) : occ;
     cfg->grid = ctx->num_sms * bps;
     cfg->threads = ctx->opt_threads;
-    cfg->chunk = ctx->opt_chunk;
+    cfg->chunk = ctx->opt_sched ? ((ctx->opt_chunk + 31) / 32) * 32 : ctx->opt_chunk;  // groups of 32 ids
     cfg->coop_threshold = ctx->opt_coop;
+    cfg->sched = ctx->opt_sched;
     if (cfg->grid > ctx->partial_cap) {
         if (ctx->d_partials) cudaFree(ctx->d_partials);
         ctx->d_partials = nullptr;
@@ -683,6 +685,10 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
         case GSWORD_OPT_BLOOM:
             ctx->opt_bloom = value ? 1 : 0;
             return GSWORD_OK;
+        case GSWORD_OPT_SCHEDULE:
+            if (value < 0 || value > 2) return fail(GSWORD_EINVAL, "schedule must be 0, 1 or 2");
+            ctx->opt_sched = (int)value;
+            return GSWORD_OK;
         case GSWORD_OPT_FILTER:
             if (value < 0 || value > 2) return fail(GSWORD_EINVAL, "filter must be 0 (label), 1 (LDF) or 2 (NLF)");
             ctx->opt_filter = (int)value;
@@ -983,6 +989,13 @@ int gsword_estimate_range(gsword_ctx* ctx, gsword_method m, uint64_t first, uint
     float ms = 0.f;
     CUDA_TRY(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
     gsword_finalize(h, out);
+    if (ctx->opt_sched == 2) {
+        // inheritance: sumsq holds the squared group totals; the groups of 32 consecutive ids
+        // are the independent units (reading A24)
+        const double n = h[3], m = std::ceil(n / 32.0);
+        out->variance = m >= 2 ? m * (h[1] - h[0] * h[0] / m) / ((m - 1.0) * n * n)
+                               : std::numeric_limits<double>::quiet_NaN();
+    }
     out->seconds = ms * 1e-3;
     return GSWORD_OK;
 }
@@ -996,6 +1009,7 @@ int gsword_trace_samples(gsword_ctx* ctx, gsword_method m, uint64_t first, uint6
     int rc = ensure_ready(ctx, (int)m);
     if (rc) return rc;
     if (!host_out) return fail(GSWORD_EINVAL, "trace: host_out NULL");
+    if (ctx->opt_sched == 2) return fail(GSWORD_EINVAL, "trace: no per-sample records under sample inheritance");
     if (n_samples == 0) return GSWORD_OK;
     gsword_sample_record* d_rec = nullptr;
     const size_t bytes = sizeof(gsword_sample_record) * (size_t)n_samples;

@@ -229,7 +229,7 @@ template <int METHOD, int MODE, bool CG>
 __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLOCKS : GSWORD_AL_MIN_BLOCKS)
     sample_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
                                                      const uint64_t count, const uint64_t seed, const int chunk,
-                                                     const uint32_t coop_threshold,
+                                                     const uint32_t coop_threshold, const int sched,
                                                      unsigned long long* __restrict__ queue,
                                                      Partial* __restrict__ partials,
                                                      gsword_sample_record* __restrict__ records,
@@ -271,6 +271,12 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
     // warp chunk of the queue (warp-uniform)
     uint64_t q_next = 0, q_end = 0;
     bool exhausted = false;
+    // scheduling (NEXT-3 comparison modes): 0 refill free lanes every round; 1 sample
+    // synchronisation (a warp refills only when all 32 lanes are free); 2 sample
+    // synchronisation + sample inheritance (Alg. 2, reading A24)
+    bool member = false;   // the lane holds a sample id of the warp's current group
+    double g_acc = 0.0;    // sched 2: this lane's complete-instance weights in the group
+    bool group_open = false;
 
     // count build only: warp-level cycle split of the loop (lane 0 of every warp)
     unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
@@ -290,6 +296,20 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
         mark(0);
         // ---------------- A1: refill free lanes from the sample queue ----------------
         unsigned need = __ballot_sync(kFull, !has);
+        if (sched == 2 && need == kFull && group_open) {
+            // group finished: its total is one independent unit of the estimate
+            double gsum = g_acc;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) gsum = __dadd_rn(gsum, shfl_xor_d(gsum, o));
+            if (lane == 0) {
+                nsum(s_sum, c_sum, gsum);
+                nsum(s_sq, c_sq, __dmul_rn(gsum, gsum));
+            }
+            g_acc = 0.0;
+            group_open = false;
+        }
+        if (sched != 0 && need != kFull) need = 0u;  // sample synchronisation: wait for the group
+        if (need == kFull) member = false;
         while (need && !exhausted) {
             if (q_next == q_end) {
                 unsigned long long base = 0;
@@ -306,6 +326,8 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             const uint32_t rank = __popc(need & lt_mask);
             if (!has && rank < avail) {
                 has = true;
+                member = true;
+                n_done += 1;  // every sample id counts in n (reading A8)
                 sid = first + q_next + rank;
                 d = 0;
                 W = 1.0;
@@ -321,6 +343,8 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             }
             q_next += min((uint32_t)__popc(need), avail);
             need = __ballot_sync(kFull, !has);
+            group_open = true;
+            if (sched != 0) break;  // one group of <= 32 consecutive ids at a time
         }
         if (!__any_sync(kFull, has)) break;
         __syncwarp();
@@ -655,11 +679,14 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 if (d + 1 == nq) complete = true;
             }
             if (dead || complete) {
-                n_done += 1;
                 if (complete) {
                     n_valid += 1;
-                    nsum(s_sum, c_sum, W);
-                    nsum(s_sq, c_sq, __dmul_rn(W, W));
+                    if (sched == 2) {
+                        g_acc = __dadd_rn(g_acc, W);
+                    } else {
+                        nsum(s_sum, c_sum, W);
+                        nsum(s_sq, c_sq, __dmul_rn(W, W));
+                    }
                 }
                 if (MODE == kModeTrace) {
                     gsword_sample_record* rec = records + (sid - first);
@@ -671,6 +698,35 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             } else {
                 d += 1;
             }
+        }
+        if (sched == 2) {
+            // Alg. 2: members without a valid partial sample inherit the lowest valid one; the
+            // parent and its k copies carry W / (k + 1) (push-down)
+            const unsigned alive_m = __ballot_sync(kFull, has);
+            const unsigned idle_m = __ballot_sync(kFull, member && !has);
+            if (alive_m != 0u && idle_m != 0u) {
+                const int par = __ffs(alive_m) - 1;
+                const double Wn = __ddiv_rn(__shfl_sync(kFull, W, par), (double)(__popc(idle_m) + 1));
+                const int dp = __shfl_sync(kFull, d, par);
+                __syncwarp();
+                if (lane == par) W = Wn;
+                if ((idle_m >> lane) & 1u) {
+                    for (int j = 0; j < dp; ++j) Ms[j * T + tid] = Ms[j * T + wbase + par];
+                    d = dp;
+                    W = Wn;
+                    has = true;
+                }
+                __syncwarp();
+            }
+        }
+    }
+    if (sched == 2 && group_open) {
+        double gsum = g_acc;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) gsum = __dadd_rn(gsum, shfl_xor_d(gsum, o));
+        if (lane == 0) {
+            nsum(s_sum, c_sum, gsum);
+            nsum(s_sq, c_sq, __dmul_rn(gsum, gsum));
         }
     }
 
@@ -1204,7 +1260,8 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
     const size_t smem = (size_t)kMaxQV * (size_t)cfg.threads * sizeof(uint32_t);
     const uint32_t thr = (uint32_t)cfg.coop_threshold;
     void* args[] = {(void*)&g,      (void*)&plan,  (void*)&first,   (void*)&count,     (void*)&seed,
-                    (void*)&cfg.chunk, (void*)&thr, (void*)&d_queue, (void*)&d_partials, (void*)&d_records,
+                    (void*)&cfg.chunk, (void*)&thr, (void*)&cfg.sched, (void*)&d_queue, (void*)&d_partials,
+                    (void*)&d_records,
                     (void*)&d_phase};
     return cudaLaunchKernel(select_kernel(method, mode), dim3(cfg.grid), dim3(cfg.threads), args, smem, stream);
 }

@@ -99,6 +99,7 @@ struct LaunchCfg {
     int threads;
     int chunk;
     int coop_threshold;
+    int sched;  // 0 refill, 1 sample synchronisation, 2 + inheritance (NEXT-3)
 };
 
 // Per-CTA partial aggregate (written by the sampling kernel, reduced in CTA order).

@@ -439,3 +439,42 @@ def test_trawl_parity_c2_and_filter(ctx, G):
                     _trawl_parity(ctx, G, g, q, m, 3, 0, 5000, 100_000, filt=filt, threads=16)
         finally:
             ctx.set_option(G.OPT_FILTER, 0)
+
+
+# ------------------------------------------------------------------ NEXT-3: schedules
+def test_sample_sync_schedule_parity(ctx, G, c0):
+    """Sample synchronisation changes only when lanes take new ids: identical samples."""
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    ctx.set_option(G.OPT_SCHEDULE, G.SCHED_SAMPLE_SYNC)
+    try:
+        for q in qs[:4]:
+            for m in (0, 1):
+                _parity(ctx, G, g, q, m, seed=21, first=5, count=30_000, loaded=True)
+    finally:
+        ctx.set_option(G.OPT_SCHEDULE, G.SCHED_REFILL)
+
+
+@pytest.mark.parametrize("filt", [0, 2])
+def test_inheritance_matches_oracle(ctx, G, c0, filt):
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    ctx.set_option(G.OPT_FILTER, filt)
+    ctx.set_option(G.OPT_SCHEDULE, G.SCHED_INHERIT)
+    try:
+        for first, count in ((0, 64_000), (7, 10_013)):  # a ragged last group
+            for q in qs:
+                ctx.load_query_obj(q)
+                for m in (0, 1):
+                    r = ctx.estimate(m, count, 31, first=first)
+                    ref = oracle.inherit_range(g, q, m, 31, first, count, filter=filt)
+                    assert r["n"] == count and r["n_valid"] == ref["n_valid"], (q.name, m)
+                    assert r["sum"] == pytest.approx(ref["sum"], rel=REL, abs=1e-300)
+                    assert r["sumsq"] == pytest.approx(ref["sumsq"], rel=REL, abs=1e-300)
+                    if ref["sumsq"] > 0:
+                        assert r["variance"] == pytest.approx(ref["variance"], rel=1e-9, abs=1e-12 * ref["sumsq"])
+        with pytest.raises(G.GswordError):
+            ctx.trace_samples(0, 0, 10, 1)
+    finally:
+        ctx.set_option(G.OPT_SCHEDULE, G.SCHED_REFILL)
+        ctx.set_option(G.OPT_FILTER, 0)

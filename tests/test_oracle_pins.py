@@ -387,3 +387,33 @@ def test_trawling_budget_and_c0(c0):
         assert np.all((st0[need] == 2) | (rec0["count"][need] == 0))
         assert np.any(st0[need] == 2)
         assert np.all(rec0["nodes"] == 0)
+
+
+# ---------------------------------------------------------------- sample inheritance (NEXT-3)
+def test_inheritance_examples_arithmetic():
+    # Ex. 6/7: treating inherited copies as independent samples biases the
+    # estimate (12 vs the true count 1); the push-down average of two copies gives 1.
+    assert (3 * 24 + 3 * 0) / 6 == 12
+    assert (1 + 1) / 2 == 1
+
+
+@pytest.mark.parametrize("method", [oracle.WJ, oracle.ALLEY])
+def test_inheritance_unbiased(method):
+    """Theorem 1: the inheritance estimator is unbiased.  Mean over 40 seeds of
+    1024-sample estimates lies within 4 standard errors of the exact count."""
+    g = gen.random_small_graph(10, 0.45, 2, seed=55)
+    q = gen.extract_query(g, 5, seed=56, dense=True)
+    truth = exact.brute_force_count(g, q)
+    ests = np.array([oracle.inherit_range(g, q, method, s, 0, 1024)["estimate"] for s in range(40)])
+    assert truth > 0
+    assert abs(ests.mean() - truth) <= 4 * ests.std(ddof=1) / math.sqrt(len(ests))
+
+
+def test_inheritance_single_lane_groups_equal_plain(c0):
+    """A group with every member alive to the end never inherits: with Alley on K_n (every
+    sample valid) the estimator equals the plain one exactly."""
+    g = gen.complete_graph(12)
+    q = gen.clique_query(4)
+    agg = oracle.inherit_range(g, q, oracle.ALLEY, 3, 0, 200)
+    y, _ = oracle.sample_range(g, q, oracle.ALLEY, 3, 0, 200, records=False)
+    assert agg["sum"] == oracle.aggregate(y)["sum"] and agg["n_valid"] == 200
