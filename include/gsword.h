@@ -141,6 +141,10 @@ typedef enum {
                                    /*   reading A24; estimates only, no traces; the   */
                                    /*   variance uses groups of 32 ids; sumsq of the  */
                                    /*   async output holds squared group totals)      */
+    GSWORD_OPT_REFILL_MIN = 9,     /* schedule 0: a warp refills only when at least    */
+                                   /* this many lanes are free (1..32; 32 = sample    */
+                                   /* synchronisation; default 16); no effect on    */
+                                   /* results                                         */
     GSWORD_OPT_FILTER = 7          /* candidate filter applied by the next            */
                                    /* gsword_load_query: 0 label only, 1 LDF, 2 NLF   */
                                    /* (1-2 build the candidate graph, reading A21)    */

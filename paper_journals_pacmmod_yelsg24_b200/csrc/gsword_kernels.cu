@@ -230,6 +230,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
     sample_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
                                                      const uint64_t count, const uint64_t seed, const int chunk,
                                                      const uint32_t coop_threshold, const int sched,
+                                                     const uint32_t refill_min,
                                                      unsigned long long* __restrict__ queue,
                                                      Partial* __restrict__ partials,
                                                      gsword_sample_record* __restrict__ records,
@@ -309,6 +310,8 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             group_open = false;
         }
         if (sched != 0 && need != kFull) need = 0u;  // sample synchronisation: wait for the group
+        // refill only when at least `refill_min` lanes are free (1 = every round, 32 = sample sync)
+        if (sched == 0 && (uint32_t)__popc(need) < refill_min) need = 0u;
         if (need == kFull) member = false;
         while (need && !exhausted) {
             if (q_next == q_end) {
@@ -1260,7 +1263,8 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
     const size_t smem = (size_t)kMaxQV * (size_t)cfg.threads * sizeof(uint32_t);
     const uint32_t thr = (uint32_t)cfg.coop_threshold;
     void* args[] = {(void*)&g,      (void*)&plan,  (void*)&first,   (void*)&count,     (void*)&seed,
-                    (void*)&cfg.chunk, (void*)&thr, (void*)&cfg.sched, (void*)&d_queue, (void*)&d_partials,
+                    (void*)&cfg.chunk, (void*)&thr, (void*)&cfg.sched, (void*)&cfg.refill_min, (void*)&d_queue,
+                    (void*)&d_partials,
                     (void*)&d_records,
                     (void*)&d_phase};
     return cudaLaunchKernel(select_kernel(method, mode), dim3(cfg.grid), dim3(cfg.threads), args, smem, stream);

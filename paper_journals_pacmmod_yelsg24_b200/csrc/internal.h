@@ -100,6 +100,7 @@ struct LaunchCfg {
     int chunk;
     int coop_threshold;
     int sched;  // 0 refill, 1 sample synchronisation, 2 + inheritance (NEXT-3)
+    uint32_t refill_min;  // sched 0: refill when at least this many lanes are free (1..32)
 };
 
 // Per-CTA partial aggregate (written by the sampling kernel, reduced in CTA order).

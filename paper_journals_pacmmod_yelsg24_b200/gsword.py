@@ -31,6 +31,7 @@ OPT_BLOOM = 5
 OPT_EDGE_SET = 6
 OPT_FILTER = 7
 OPT_SCHEDULE = 8
+OPT_REFILL_MIN = 9
 SCHED_REFILL, SCHED_SAMPLE_SYNC, SCHED_INHERIT = 0, 1, 2
 FILTER_LABEL, FILTER_LDF, FILTER_NLF = 0, 1, 2
 CUDA_STREAM_LEGACY = 0x1  # cudaStreamLegacy

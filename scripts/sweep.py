@@ -21,8 +21,9 @@ ap.add_argument("--reps", type=int, default=2)
 ap.add_argument("--filter", type=int, default=0)
 args = ap.parse_args()
 OPT = {"coop": G.OPT_COOP_THRESHOLD, "threads": G.OPT_THREADS, "chunk": G.OPT_CHUNK, "bps": G.OPT_BLOCKS_PER_SM,
-       "l2": G.OPT_L2_PERSIST, "bloom": G.OPT_BLOOM, "eset": G.OPT_EDGE_SET}
-DEF = {"coop": 64, "threads": 256, "chunk": 256, "bps": 0, "l2": 0, "bloom": 1, "eset": 1}
+       "l2": G.OPT_L2_PERSIST, "bloom": G.OPT_BLOOM, "eset": G.OPT_EDGE_SET,
+       "sched": G.OPT_SCHEDULE, "rmin": G.OPT_REFILL_MIN}
+DEF = {"coop": 64, "threads": 256, "chunk": 256, "bps": 0, "l2": 0, "bloom": 1, "eset": 1, "sched": 0, "rmin": 16}
 grid = json.loads(args.grid)
 g, qs = gen.CONFIGS[args.config]()
 queries = qs if args.query < 0 else [qs[args.query]]
@@ -49,5 +50,6 @@ with G.Context(0) as ctx:
                                   "cg_entries": qi["cg_entries"], "cg_build_s": qi["build_seconds"],
                                   "candidates": qi["candidates"],
                                   "opts": dict(zip(keys, vals)), "kernel_s": best,
-                                  "rate": args.samples / best, "valid": r["n_valid"], "est": r["estimate"]}),
+                                  "rate": args.samples / best, "valid": r["n_valid"], "est": r["estimate"],
+                                  "var": r["variance"], "var_x_s": r["variance"] * best}),
                       flush=True)

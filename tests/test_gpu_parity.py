@@ -146,6 +146,7 @@ def test_edge_index_invariance(ctx, G, bloom, eset):
     finally:
         ctx.set_option(G.OPT_BLOOM, 1)
         ctx.set_option(G.OPT_EDGE_SET, 1)
+        ctx.set_option(G.OPT_REFILL_MIN, 16)
         ctx.set_option(G.OPT_EDGE_SET, 1)
 
 
@@ -262,7 +263,7 @@ def test_scheduling_invariance(ctx, G, c0):
     try:
         for opt, val in ((G.OPT_CHUNK, 1), (G.OPT_CHUNK, 4096), (G.OPT_BLOCKS_PER_SM, 1),
                          (G.OPT_THREADS, 64), (G.OPT_L2_PERSIST, 1), (G.OPT_L2_PERSIST, 2), (G.OPT_BLOOM, 0),
-                         (G.OPT_EDGE_SET, 0)):
+                         (G.OPT_EDGE_SET, 0), (G.OPT_REFILL_MIN, 1), (G.OPT_REFILL_MIN, 32)):
             ctx.set_option(opt, val)
             for m in (0, 1):
                 r = ctx.estimate(m, 400_000, 9)
