@@ -50,6 +50,7 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="budget of the oracle timing")
     ap.add_argument("--traffic-file", default=os.path.join(ROOT, "profiles", "traffic_latest.json"))
     ap.add_argument("--quick", action="store_true", help="small config for smoke-testing the script")
+    ap.add_argument("--no-qerror", action="store_true", help="skip the (untimed) C0 q-error leg")
     return ap.parse_args()
 
 
@@ -363,7 +364,7 @@ def run_ours(args):
 
     info = ctx.launch_info()
     name = {G.WJ: "wj", G.ALLEY: "alley"}
-    qerr = qerror_leg(G, ctx, args) if not args.quick else None
+    qerr = qerror_leg(G, ctx, args) if not (args.quick or args.no_qerror) else None
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": 1e3 * max_time / args.steps, "higher_is_better": True,
