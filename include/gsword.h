@@ -183,6 +183,18 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value);
 int gsword_load_graph(gsword_ctx* ctx, int64_t n_vertices, const int64_t* row_ptr, const int32_t* col,
                       const int32_t* labels, int32_t n_labels);
 
+/* Load the data graph from DEVICE memory (e.g. torch tensors on the context's device).
+ *   d_row_ptr int64[n_vertices+1]  borrowed for the call only
+ *   d_col     int32[row_ptr[n]]    borrowed, NOT copied: the caller keeps it alive and
+ *                                  unchanged until the next load or gsword_destroy
+ *   d_labels  int32[n_vertices] or NULL (n_labels 1); borrowed like d_col
+ * Each row must already be sorted by (label, id) (= by id when unlabelled), with no self
+ * loop and a symmetric adjacency; this is checked on the device (EGRAPH).  The library
+ * derives and owns seg, the label buckets, the Bloom filter and the edge set.
+ * Errors: EINVAL, EGRAPH, ELIMIT, ENOMEM, ECUDA. */
+int gsword_load_graph_device(gsword_ctx* ctx, int64_t n_vertices, const int64_t* d_row_ptr, const int32_t* d_col,
+                             const int32_t* d_labels, int32_t n_labels);
+
 /* Load the query q and its matching order phi (Def. 2).  Host arrays, copied.
  * With GSWORD_OPT_FILTER > 0 this also builds the candidate graph on the device
  * (Def. 5; Fig. 4) and the sampler draws from its local candidate lists:

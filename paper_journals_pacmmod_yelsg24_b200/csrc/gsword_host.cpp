@@ -194,6 +194,8 @@ struct gsword_ctx {
     // graph
     bool graph_loaded = false;
     int32_t* d_col = nullptr;
+    bool own_col = true;      // false: borrowed from the caller (gsword_load_graph_device)
+    bool own_vlabel = true;
     uint32_t* d_seg = nullptr;
     void* d_hot = nullptr;     // one allocation: [Bloom filter words][seg] (the L2-window target)
     size_t hot_bytes = 0;
@@ -258,9 +260,10 @@ struct gsword_ctx {
 
     void free_graph() {
         free_query();
-        if (d_vlabel) cudaFree(d_vlabel);
+        if (d_vlabel && own_vlabel) cudaFree(d_vlabel);
         d_vlabel = nullptr;
-        if (d_col) cudaFree(d_col);
+        if (d_col && own_col) cudaFree(d_col);
+        own_col = own_vlabel = true;
         if (d_hot) cudaFree(d_hot);
         if (d_bucket) cudaFree(d_bucket);
         if (d_eset) cudaFree(d_eset);
@@ -912,6 +915,148 @@ int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const 
     ctx->n_labels = L;
     ctx->label_off = off;
     label_pair_freq(n, row_ptr, col, labels, L, &ctx->pair_freq);
+    ctx->graph_loaded = true;
+    ctx->query_loaded = false;
+    return apply_l2_window(ctx);
+}
+
+int gsword_load_graph_device(gsword_ctx* ctx, int64_t n, const int64_t* d_row_ptr, const int32_t* d_col,
+                             const int32_t* d_labels, int32_t n_labels) {
+    if (!ctx) return fail(GSWORD_EINVAL, "load_graph_device: NULL context");
+    if (n < 0 || !d_row_ptr || (n > 0 && !d_col)) return fail(GSWORD_EINVAL, "load_graph_device: bad argument");
+    if (n_labels < 1 || (!d_labels && n_labels != 1))
+        return fail(GSWORD_EINVAL, "load_graph_device: labels NULL requires n_labels == 1");
+    if (n >= (int64_t)1 << 31 || n * (int64_t)n_labels >= ((int64_t)1 << 31))
+        return fail(GSWORD_ELIMIT, "load_graph_device: |V| or |V| * n_labels >= 2^31");
+    CUDA_TRY(cudaSetDevice(ctx->device));
+    CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    ctx->free_graph();
+    cudaStream_t st = ctx->stream;
+    int64_t h_rp[2] = {0, 0};
+    CUDA_TRY(cudaMemcpy(&h_rp[0], d_row_ptr, sizeof(int64_t), cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpy(&h_rp[1], d_row_ptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost));
+    const int64_t nnz = h_rp[1];
+    if (h_rp[0] != 0) return fail(GSWORD_EGRAPH, "load_graph_device: row_ptr[0] != 0");
+    if (nnz < 0 || nnz >= ((int64_t)1 << 31) - 1) return fail(GSWORD_ELIMIT, "load_graph_device: 2|E| >= 2^31");
+    const int32_t L = n_labels;
+    int* d_bad = nullptr;
+    unsigned long long* d_hist = nullptr;
+    CUDA_TRY(cudaMalloc(&d_bad, sizeof(int)));
+    CUDA_TRY(cudaMalloc(&d_hist, sizeof(unsigned long long) * ((size_t)L + 2)));
+    auto cleanup = [&]() {
+        cudaFree(d_bad);
+        cudaFree(d_hist);
+    };
+    int bad = 0;
+    std::vector<unsigned long long> hist((size_t)L, 0);
+    cudaError_t e = cudaMemsetAsync(d_bad, 0, sizeof(int), st);
+    if (e == cudaSuccess) e = gsword::launch_dev_validate(d_row_ptr, d_col, d_labels, n, L, d_bad, st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(d_hist, 0, sizeof(unsigned long long) * (size_t)L, st);
+    if (e == cudaSuccess) e = gsword::launch_label_hist(d_labels, n, d_hist, st);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&bad, d_bad, sizeof(int), cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(hist.data(), d_hist, sizeof(unsigned long long) * (size_t)L,
+                                              cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) {
+        cleanup();
+        return cuda_fail(e, "load_graph_device: validation");
+    }
+    if (bad) {
+        cleanup();
+        return fail(bad & 1 ? GSWORD_EINVAL : GSWORD_EGRAPH,
+                    "load_graph_device: CSR not canonical (flags %d: 1 label range, 2 row_ptr, 4 id range/self "
+                    "loop, 8 row not ascending by (label, id), 16 asymmetric)", bad);
+    }
+    std::vector<int64_t> off((size_t)L + 1, 0);
+    for (int32_t l = 0; l < L; ++l) off[(size_t)l + 1] = off[(size_t)l] + (int64_t)hist[(size_t)l];
+    // hot buffer (Bloom words + seg), buckets, edge set; col and labels are borrowed
+    uint64_t words = 1;
+    {
+        const uint64_t want = std::max<uint64_t>(1, (uint64_t)(nnz / 2) * 16 / 64);
+        while (words < want) words <<= 1;
+    }
+    const size_t seg_n = (size_t)n * (size_t)L + 1;
+    const size_t hot_bytes = words * sizeof(unsigned long long) + sizeof(uint32_t) * seg_n;
+    uint64_t buckets = 1;
+    {
+        const uint64_t want_b = std::max<uint64_t>(1, ((uint64_t)(nnz / 2) + 1) / 2);
+        while (buckets < want_b) buckets <<= 1;
+    }
+    ctx->own_col = false;
+    ctx->d_col = const_cast<int32_t*>(d_col);
+    if ((e = cudaMalloc(&ctx->d_hot, hot_bytes)) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_bucket, sizeof(int32_t) * (size_t)std::max<int64_t>(n, 1))) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_eset, buckets * 4 * sizeof(unsigned long long))) != cudaSuccess) {
+        cleanup();
+        ctx->free_graph();
+        return fail(GSWORD_ENOMEM, "load_graph_device: cudaMalloc: %s", cudaGetErrorString(e));
+    }
+    if (d_labels) {
+        ctx->own_vlabel = false;
+        ctx->d_vlabel = const_cast<int32_t*>(d_labels);
+    } else {
+        if ((e = cudaMalloc(&ctx->d_vlabel, sizeof(int32_t) * (size_t)std::max<int64_t>(n, 1))) != cudaSuccess) {
+            cleanup();
+            ctx->free_graph();
+            return fail(GSWORD_ENOMEM, "load_graph_device: cudaMalloc(labels)");
+        }
+        CUDA_TRY(cudaMemsetAsync(ctx->d_vlabel, 0, sizeof(int32_t) * (size_t)std::max<int64_t>(n, 1), st));
+    }
+    ctx->hot_bytes = hot_bytes;
+    ctx->d_bloom = reinterpret_cast<unsigned long long*>(ctx->d_hot);
+    ctx->d_seg = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ctx->d_hot) + words * sizeof(unsigned long long));
+    ctx->bloom_words = words;
+    ctx->eset_buckets = buckets;
+    CUDA_TRY(gsword::launch_dev_seg(d_row_ptr, d_col, d_labels, n, L, ctx->d_seg, st));
+    if (L == 1) {
+        if (n > 0) CUDA_TRY(gsword::launch_build_bucket_identity(ctx->d_bucket, n, st));
+    } else {
+        uint32_t* d_cnt = nullptr;
+        uint32_t* d_tmp = nullptr;
+        unsigned long long* d_b = nullptr;
+        const size_t tmpw = gsword::scan_tmp_words(n + 1);
+        if ((e = cudaMalloc(&d_cnt, sizeof(uint32_t) * (size_t)(n + 1))) != cudaSuccess ||
+            (e = cudaMalloc(&d_tmp, sizeof(uint32_t) * tmpw)) != cudaSuccess ||
+            (e = cudaMalloc(&d_b, sizeof(unsigned long long) * 2 * (size_t)L)) != cudaSuccess) {
+            cudaFree(d_cnt);
+            cudaFree(d_tmp);
+            cleanup();
+            ctx->free_graph();
+            return fail(GSWORD_ENOMEM, "load_graph_device: bucket scratch");
+        }
+        std::vector<unsigned long long> bases((size_t)L);
+        for (int32_t l = 0; l < L; ++l) bases[(size_t)l] = (unsigned long long)off[(size_t)l];
+        CUDA_TRY(cudaMemcpyAsync(d_b, bases.data(), sizeof(unsigned long long) * (size_t)L, cudaMemcpyHostToDevice, st));
+        for (int32_t l = 0; l < L; ++l)
+            CUDA_TRY(gsword::launch_label_bucket(d_labels, n, l, d_cnt, d_b + l, d_tmp, d_b + L + l, ctx->d_bucket, st));
+        CUDA_TRY(cudaStreamSynchronize(st));
+        cudaFree(d_cnt);
+        cudaFree(d_tmp);
+        cudaFree(d_b);
+    }
+    // label-pair frequencies (QuickSI order) for up to 64 labels
+    ctx->pair_freq.clear();
+    if (L <= 64) {
+        unsigned long long* d_pf = nullptr;
+        CUDA_TRY(cudaMalloc(&d_pf, sizeof(unsigned long long) * (size_t)L * (size_t)L));
+        CUDA_TRY(cudaMemsetAsync(d_pf, 0, sizeof(unsigned long long) * (size_t)L * (size_t)L, st));
+        CUDA_TRY(gsword::launch_pair_hist(d_row_ptr, d_col, d_labels, n, L, d_pf, st));
+        std::vector<unsigned long long> pf((size_t)L * (size_t)L);
+        CUDA_TRY(cudaMemcpyAsync(pf.data(), d_pf, sizeof(unsigned long long) * pf.size(), cudaMemcpyDeviceToHost, st));
+        CUDA_TRY(cudaStreamSynchronize(st));
+        cudaFree(d_pf);
+        ctx->pair_freq.assign(pf.begin(), pf.end());
+    }
+    CUDA_TRY(cudaMemsetAsync(ctx->d_bloom, 0, words * sizeof(unsigned long long), st));
+    CUDA_TRY(cudaMemsetAsync(ctx->d_eset, 0xFF, buckets * 4 * sizeof(unsigned long long), st));
+    CUDA_TRY(gsword::launch_build_bloom(d_row_ptr, d_col, n, ctx->d_bloom, words - 1, st));
+    CUDA_TRY(gsword::launch_build_eset(d_row_ptr, d_col, n, ctx->d_eset, buckets - 1, st));
+    CUDA_TRY(cudaStreamSynchronize(st));
+    cleanup();
+    ctx->n = n;
+    ctx->nnz = nnz;
+    ctx->n_labels = L;
+    ctx->label_off = off;
     ctx->graph_loaded = true;
     ctx->query_loaded = false;
     return apply_l2_window(ctx);

@@ -1347,6 +1347,131 @@ cudaError_t launch_trawl(int method, bool trace, bool cg, const DeviceGraph& g, 
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------- device-side graph load
+// (gsword_load_graph_device: the CSR stays in caller-owned device memory)
+__device__ __forceinline__ bool key_less(int32_t la, int32_t a, int32_t lb, int32_t b) {
+    return la < lb || (la == lb && a < b);
+}
+
+// canonical check: ids in range, no self loop, rows strictly ascending by (label, id), and
+// the adjacency symmetric (v found in w's row by binary search on (label, id))
+__global__ void dev_validate_kernel(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
+                                    const int32_t* __restrict__ labels, int64_t n, int32_t n_labels,
+                                    int* __restrict__ bad) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t lv = labels ? labels[v] : 0;
+        if (lv < 0 || lv >= n_labels) { atomicOr(bad, 1); continue; }
+        const int64_t a = row_ptr[v], b = row_ptr[v + 1];
+        if (b < a) { atomicOr(bad, 2); continue; }
+        int32_t pl = -1, pw = -1;
+        for (int64_t i = a; i < b; ++i) {
+            const int32_t w = col[i];
+            if (w < 0 || w >= n || w == v) { atomicOr(bad, 4); break; }
+            const int32_t lw = labels ? labels[w] : 0;
+            if (i > a && !key_less(pl, pw, lw, w)) { atomicOr(bad, 8); break; }
+            pl = lw;
+            pw = w;
+            int64_t lo = row_ptr[w], hi = row_ptr[w + 1];
+            while (lo < hi) {
+                const int64_t mid = (lo + hi) >> 1;
+                const int32_t x = col[mid];
+                const int32_t lx = labels ? labels[x] : 0;
+                if (key_less(lx, x, lv, (int32_t)v)) lo = mid + 1; else hi = mid;
+            }
+            if (lo >= row_ptr[w + 1] || col[lo] != (int32_t)v) { atomicOr(bad, 16); break; }
+        }
+    }
+}
+
+__global__ void dev_seg_kernel(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
+                               const int32_t* __restrict__ labels, int64_t n, int32_t L, uint32_t* __restrict__ seg) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= n; v += (int64_t)gridDim.x * blockDim.x) {
+        if (v == n) {
+            seg[(size_t)n * L] = (uint32_t)row_ptr[n];
+            continue;
+        }
+        const int64_t a = row_ptr[v], b = row_ptr[v + 1];
+        int32_t l = 0;
+        for (int64_t i = a; i < b; ++i) {
+            const int32_t lw = labels ? labels[col[i]] : 0;
+            while (l <= lw) seg[(size_t)v * L + l++] = (uint32_t)i;
+        }
+        while (l < L) seg[(size_t)v * L + l++] = (uint32_t)b;
+    }
+}
+
+__global__ void label_hist_kernel(const int32_t* __restrict__ labels, int64_t n, unsigned long long* __restrict__ hist) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(hist + (labels ? labels[v] : 0), 1ull);
+}
+
+// data adjacency entries per (label, label): block-private histograms in shared memory
+__global__ void pair_hist_kernel(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
+                                 const int32_t* __restrict__ labels, int64_t n, int32_t L,
+                                 unsigned long long* __restrict__ hist) {
+    extern __shared__ unsigned long long h[];
+    const int bins = L * L;
+    for (int i = threadIdx.x; i < bins; i += blockDim.x) h[i] = 0ull;
+    __syncthreads();
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t lv = labels ? labels[v] : 0;
+        if (!labels) {
+            atomicAdd(&h[0], (unsigned long long)(row_ptr[v + 1] - row_ptr[v]));
+            continue;
+        }
+        for (int64_t i = row_ptr[v]; i < row_ptr[v + 1]; ++i) atomicAdd(&h[lv * L + labels[col[i]]], 1ull);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < bins; i += blockDim.x)
+        if (h[i]) atomicAdd(hist + i, h[i]);
+}
+
+__global__ void label_count_kernel(const int32_t* __restrict__ labels, int64_t n, int32_t l,
+                                   uint32_t* __restrict__ counts) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= n; v += (int64_t)gridDim.x * blockDim.x)
+        counts[v] = (v < n && labels[v] == l) ? 1u : 0u;
+}
+
+__global__ void label_fill_kernel(const int32_t* __restrict__ labels, int64_t n, int32_t l,
+                                  const uint32_t* __restrict__ off, int32_t* __restrict__ bucket) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        if (labels[v] == l) bucket[off[v]] = (int32_t)v;
+}
+
+cudaError_t launch_dev_validate(const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int64_t n,
+                                int32_t n_labels, int* d_bad, cudaStream_t stream) {
+    dev_validate_kernel<<<148 * 8, 256, 0, stream>>>(row_ptr, col, labels, n, n_labels, d_bad);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_dev_seg(const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int64_t n, int32_t L,
+                           uint32_t* seg, cudaStream_t stream) {
+    dev_seg_kernel<<<148 * 8, 256, 0, stream>>>(row_ptr, col, labels, n, L, seg);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_label_hist(const int32_t* labels, int64_t n, unsigned long long* hist, cudaStream_t stream) {
+    label_hist_kernel<<<148 * 4, 256, 0, stream>>>(labels, n, hist);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_pair_hist(const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int64_t n, int32_t L,
+                             unsigned long long* hist, cudaStream_t stream) {
+    const size_t smem = sizeof(unsigned long long) * (size_t)L * (size_t)L;
+    pair_hist_kernel<<<148 * 4, 256, smem, stream>>>(row_ptr, col, labels, n, L, hist);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_label_bucket(const int32_t* labels, int64_t n, int32_t l, uint32_t* counts,
+                                const unsigned long long* d_base, uint32_t* d_tmp, unsigned long long* d_total,
+                                int32_t* bucket, cudaStream_t stream) {
+    label_count_kernel<<<148 * 4, 256, 0, stream>>>(labels, n, l, counts);
+    cudaError_t e = launch_scan(counts, n + 1, d_base, d_tmp, d_total, stream);
+    if (e != cudaSuccess) return e;
+    label_fill_kernel<<<148 * 4, 256, 0, stream>>>(labels, n, l, counts, bucket);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream) {
     iota_kernel<<<148 * 4, 256, 0, stream>>>(bucket, n);
     return cudaGetLastError();

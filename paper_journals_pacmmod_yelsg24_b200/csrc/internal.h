@@ -121,6 +121,17 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
 cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_out4, double* d_sectors,
                           cudaStream_t stream);
 cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream);
+// device-side graph load (gsword_load_graph_device)
+cudaError_t launch_dev_validate(const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int64_t n,
+                                int32_t n_labels, int* d_bad, cudaStream_t stream);
+cudaError_t launch_dev_seg(const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int64_t n, int32_t L,
+                           uint32_t* seg, cudaStream_t stream);
+cudaError_t launch_label_hist(const int32_t* labels, int64_t n, unsigned long long* hist, cudaStream_t stream);
+cudaError_t launch_pair_hist(const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int64_t n, int32_t L,
+                             unsigned long long* hist, cudaStream_t stream);
+cudaError_t launch_label_bucket(const int32_t* labels, int64_t n, int32_t l, uint32_t* counts,
+                                const unsigned long long* d_base, uint32_t* d_tmp, unsigned long long* d_total,
+                                int32_t* bucket, cudaStream_t stream);
 cudaError_t launch_trawl(int method, bool trace, bool cg, const DeviceGraph& g, const Plan& plan, int grid,
                          uint64_t first, uint64_t count, uint64_t seed, uint64_t budget, unsigned long long* d_queue,
                          Partial* d_partials, gsword_trawl_record* d_records, cudaStream_t stream);

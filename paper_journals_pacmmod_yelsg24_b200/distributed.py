@@ -55,6 +55,37 @@ def estimate_distributed(ctx: Context, method: int, n_total: int, seed: int, fir
     return finalize(out4.cpu().numpy())
 
 
+def broadcast_graph(row_ptr=None, col=None, labels=None, n_labels: int = 1, device=None, src: int = 0, group=None):
+    """Replicate the graph from rank `src` to every rank over the process group (NCCL over
+    NVLink for CUDA tensors; gloo for CPU tensors).  Rank src passes numpy/torch arrays
+    (col sorted by (label, id) per row); the others pass None.  Returns (row_ptr, col,
+    labels, n_labels) as tensors on `device`, ready for Context.load_graph_device."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    rank = dist.get_rank(group)
+    hdr = torch.zeros(3, dtype=torch.int64, device=device)
+    if rank == src:
+        hdr[0] = int(len(row_ptr) - 1)
+        hdr[1] = int(len(col))
+        hdr[2] = int(n_labels)
+    dist.broadcast(hdr, src, group=group)
+    n, nnz, nl = (int(x) for x in hdr.tolist())
+    if rank == src:
+        rp = torch.as_tensor(np.ascontiguousarray(row_ptr, np.int64)).to(device)
+        cl = torch.as_tensor(np.ascontiguousarray(col, np.int32)).to(device)
+        lb = torch.as_tensor(np.ascontiguousarray(labels if labels is not None else np.zeros(n, np.int32),
+                                                  np.int32)).to(device)
+    else:
+        rp = torch.empty(n + 1, dtype=torch.int64, device=device)
+        cl = torch.empty(nnz, dtype=torch.int32, device=device)
+        lb = torch.empty(n, dtype=torch.int32, device=device)
+    for t in (rp, cl, lb):
+        dist.broadcast(t, src, group=group)
+    return rp, cl, lb, nl
+
+
 def combine_host(values4_per_rank) -> Dict[str, float]:
     """Host-side equivalent of the all_reduce + finalize (for checkpoint/resume of
     partial ranges): element-wise sum of {sum, sumsq, n_valid, n} then finalize."""

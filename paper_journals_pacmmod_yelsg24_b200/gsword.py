@@ -91,6 +91,7 @@ def _load_library() -> ctypes.CDLL:
         "gsword_set_option": ([P, ctypes.c_int, I64], ctypes.c_int),
         "gsword_load_graph": ([P, I64, P, P, P, I32], ctypes.c_int),
         "gsword_load_query": ([P, I32, P, P, P, P], ctypes.c_int),
+        "gsword_load_graph_device": ([P, I64, P, P, P, I32], ctypes.c_int),
         "gsword_estimate": ([P, ctypes.c_int, U64, U64, ctypes.POINTER(_Result)], ctypes.c_int),
         "gsword_estimate_range": ([P, ctypes.c_int, U64, U64, U64, ctypes.POINTER(_Result)], ctypes.c_int),
         "gsword_estimate_async": ([P, ctypes.c_int, U64, U64, U64, P], ctypes.c_int),
@@ -261,6 +262,18 @@ class Context:
             cl = np.zeros(1, np.int32)
         lb = None if labels is None or n_labels == 1 else np.ascontiguousarray(labels, np.int32)
         _check(_lib.gsword_load_graph(self._h, rp.shape[0] - 1, _ptr(rp), _ptr(cl), _ptr(lb), int(n_labels)))
+
+    def load_graph_device(self, row_ptr, col, labels=None, n_labels: int = 1) -> None:
+        """gsword_load_graph_device: CUDA tensors (int64 row_ptr, int32 col label-sorted per
+        row, int32 labels or None) on this context's device; col/labels are borrowed and kept
+        referenced here until the next load."""
+        for t in (row_ptr, col) + ((labels,) if labels is not None else ()):
+            if not t.is_cuda or not t.is_contiguous():
+                raise ValueError("load_graph_device needs contiguous CUDA tensors")
+        lab_ptr = ctypes.c_void_p(labels.data_ptr()) if labels is not None and n_labels > 1 else None
+        _check(_lib.gsword_load_graph_device(self._h, int(row_ptr.numel() - 1), ctypes.c_void_p(row_ptr.data_ptr()),
+                                             ctypes.c_void_p(col.data_ptr()), lab_ptr, int(n_labels)))
+        self._borrowed = (col, labels)
 
     def load_query(self, q_row_ptr, q_col, q_labels, order) -> int:
         """Returns the bytes handed to the library (query CSR + labels + order)."""

@@ -72,3 +72,45 @@ def test_gloo_two_ranks_combine():
     assert combined["sumsq"] == pytest.approx(ref["sumsq"], rel=1e-12)
     host = combine_host([[ref["sum"], ref["sumsq"], ref["n_valid"], ref["n"]]])
     assert host["estimate"] == pytest.approx(ref["estimate"], rel=1e-15)
+
+
+def _bcast_worker(rank, world, port, q):
+    from paper_journals_pacmmod_yelsg24_b200.distributed import broadcast_graph
+    from workloads import gen
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    if rank == 0:
+        g, _ = gen.config_c0()
+        out = broadcast_graph(g.row_ptr, g.label_sorted_col(), g.labels, g.n_labels, device="cpu")
+    else:
+        out = broadcast_graph(device="cpu")
+    rp, cl, lb, nl = out
+    q.put((rank, rp.numpy().tolist()[:50], int(cl.sum()), int(lb.sum()), nl, int(cl.numel())))
+    dist.destroy_process_group()
+
+
+def test_gloo_broadcast_graph():
+    from workloads import gen
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_bcast_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = dict((r[0], r[1:]) for r in (q.get(timeout=300) for _ in range(2)))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert res[0] == res[1]
+    g, _ = gen.config_c0()
+    assert res[0][0] == g.row_ptr.tolist()[:50] and res[0][4] == g.col.shape[0] and res[0][3] == 4
+
+
+def test_label_sorted_col():
+    from workloads import gen
+    g = gen.random_small_graph(20, 0.4, 3, seed=1)
+    c = g.label_sorted_col()
+    for v in range(g.n):
+        row = c[g.row_ptr[v]:g.row_ptr[v + 1]]
+        keys = list(zip(g.labels[row].tolist(), row.tolist()))
+        assert keys == sorted(keys) and sorted(row.tolist()) == g.neighbors(v).tolist()

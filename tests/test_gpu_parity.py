@@ -479,3 +479,30 @@ def test_inheritance_matches_oracle(ctx, G, c0, filt):
     finally:
         ctx.set_option(G.OPT_SCHEDULE, G.SCHED_REFILL)
         ctx.set_option(G.OPT_FILTER, 0)
+
+
+# ------------------------------------------------------------------ device-resident graph load
+def test_load_graph_device_equals_host(ctx, G, c0):
+    import torch
+    cases = [c0[0], gen.chung_lu(4000, 40_000, gamma=2.2, max_over_mean=50.0, seed=9), gen.config_c2()[0]]
+    for g in cases:
+        q = gen.extract_query(g, 5, seed=4, dense=True)
+        ctx.load_graph_obj(g)
+        ctx.load_query_obj(q)
+        ref = {m: ctx.trace_samples(m, 0, 20_000, 2) for m in (0, 1)}
+        qo_host = G.quicksi_order(g.row_ptr, g.col, g.labels, g.n_labels, *q.csr(), q.labels)
+        rp = torch.as_tensor(g.row_ptr).cuda()
+        cl = torch.as_tensor(g.label_sorted_col()).cuda()
+        lb = torch.as_tensor(g.labels).cuda()
+        ctx.load_graph_device(rp, cl, lb if g.n_labels > 1 else None, g.n_labels)
+        ctx.load_query_obj(q)
+        for m in (0, 1):
+            assert ctx.trace_samples(m, 0, 20_000, 2).tobytes() == ref[m].tobytes()
+        order, _ = ctx.select_order(G.ORDER_QUICKSI, 0, *q.csr(), q.labels)
+        assert order == qo_host
+    # non-canonical device input is rejected
+    g = c0[0]
+    bad = torch.as_tensor(g.col).cuda()  # id-sorted, not (label, id)-sorted
+    with pytest.raises(G.GswordError) as e:
+        ctx.load_graph_device(torch.as_tensor(g.row_ptr).cuda(), bad, torch.as_tensor(g.labels).cuda(), g.n_labels)
+    assert e.value.status == -5

@@ -49,6 +49,12 @@ class Graph:
     def neighbors(self, v: int) -> np.ndarray:
         return self.col[self.row_ptr[v]:self.row_ptr[v + 1]]
 
+    def label_sorted_col(self) -> np.ndarray:
+        """Adjacency with each row ordered by (label, id) (layout for device loading)."""
+        src = np.repeat(np.arange(self.n, dtype=np.int64), np.diff(self.row_ptr))
+        key = (src * max(self.n_labels, 1) + self.labels[self.col].astype(np.int64)) * self.n + self.col
+        return self.col[np.argsort(key, kind="stable")].astype(np.int32)
+
 
 @dataclasses.dataclass
 class Query:
