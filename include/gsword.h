@@ -122,6 +122,7 @@ typedef struct {
     uint64_t candidates[GSWORD_MAX_QV];
     uint64_t cg_entries;
     double build_seconds;
+    int32_t refill_min[2]; /* refill threshold in use per method (after autotune) */
 } gsword_query_stats;
 
 /* Tunables for gsword_set_option (defaults chosen by measurement). */
@@ -145,6 +146,9 @@ typedef enum {
                                    /* this many lanes are free (1..32; 32 = sample    */
                                    /* synchronisation; default 16); no effect on    */
                                    /* results                                         */
+    GSWORD_OPT_AUTOTUNE = 10,      /* 1 (default): gsword_load_query times pilots of   */
+                                   /* refill thresholds 8/16/24/32 per method and     */
+                                   /* keeps the fastest; results are unaffected       */
     GSWORD_OPT_FILTER = 7          /* candidate filter applied by the next            */
                                    /* gsword_load_query: 0 label only, 1 LDF, 2 NLF   */
                                    /* (1-2 build the candidate graph, reading A21)    */

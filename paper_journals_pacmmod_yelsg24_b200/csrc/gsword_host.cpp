@@ -253,7 +253,9 @@ struct gsword_ctx {
     int opt_coop = 64;
     int opt_bloom = 1;
     int opt_sched = 0;
-    int opt_refill_min = 16;  // measured: 1.2-1.35x over refilling every round on C1, neutral on C2/C3
+    int opt_refill_min = 16;
+    int opt_autotune = 1;         // pick the refill threshold per method with pilots at query load
+    int tuned_refill[2] = {0, 0}; // 0 = not tuned  // measured: 1.2-1.35x over refilling every round on C1, neutral on C2/C3
     int opt_eset = 1;
     // last launch
     int last_grid = 0, last_threads = 0;
@@ -332,7 +334,8 @@ int launch_config(gsword_ctx* ctx, int method, int mode, LaunchCfg* cfg) {
     cfg->chunk = ctx->opt_sched ? ((ctx->opt_chunk + 31) / 32) * 32 : ctx->opt_chunk;  // groups of 32 ids
     cfg->coop_threshold = ctx->opt_coop;
     cfg->sched = ctx->opt_sched;
-    cfg->refill_min = (uint32_t)ctx->opt_refill_min;
+    cfg->refill_min = (uint32_t)((ctx->opt_autotune && ctx->tuned_refill[method & 1] > 0) ? ctx->tuned_refill[method & 1]
+                                                                                       : ctx->opt_refill_min);
     if (cfg->grid > ctx->partial_cap) {
         if (ctx->d_partials) cudaFree(ctx->d_partials);
         ctx->d_partials = nullptr;
@@ -698,6 +701,10 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
             if (value < 1 || value > 32) return fail(GSWORD_EINVAL, "refill_min must be 1..32");
             ctx->opt_refill_min = (int)value;
             return GSWORD_OK;
+        case GSWORD_OPT_AUTOTUNE:
+            ctx->opt_autotune = value ? 1 : 0;
+            if (!value) ctx->tuned_refill[0] = ctx->tuned_refill[1] = 0;
+            return GSWORD_OK;
         case GSWORD_OPT_FILTER:
             if (value < 0 || value > 2) return fail(GSWORD_EINVAL, "filter must be 0 (label), 1 (LDF) or 2 (NLF)");
             ctx->opt_filter = (int)value;
@@ -792,18 +799,27 @@ int gsword_select_order(gsword_ctx* ctx, int strategy, gsword_method m, int32_t 
         }
     double best_score = 0.0;
     int best = -1;
+    const int autotune = ctx->opt_autotune;
+    ctx->opt_autotune = 0;  // pilots only matter for the order finally loaded
     for (size_t c = 0; c < cands.size(); ++c) {
         rc = gsword_load_query(ctx, n_qv, q_row_ptr, q_col, q_labels, cands[c].data());
-        if (rc) return rc;
+        if (rc) {
+            ctx->opt_autotune = autotune;
+            return rc;
+        }
         gsword_result r;
         rc = gsword_estimate_range(ctx, m, 0, pilot_samples, seed, &r);
-        if (rc) return rc;
+        if (rc) {
+            ctx->opt_autotune = autotune;
+            return rc;
+        }
         const double score = std::isnan(r.variance) ? 0.0 : r.variance * (double)r.n_samples;
         if (best < 0 || score < best_score) {
             best = (int)c;
             best_score = score;
         }
     }
+    ctx->opt_autotune = autotune;
     std::memcpy(order_out, cands[(size_t)best].data(), sizeof(int32_t) * (size_t)n_qv);
     if (score_out) *score_out = best_score;
     return gsword_load_query(ctx, n_qv, q_row_ptr, q_col, q_labels, order_out);
@@ -1087,6 +1103,35 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
     }
     ctx->plan = p;
     ctx->query_loaded = true;
+    ctx->tuned_refill[0] = ctx->tuned_refill[1] = 0;
+    if (ctx->opt_autotune && ctx->opt_sched == 0) {
+        // schedule autotune (no effect on any result): time pilot runs of each method with
+        // refill thresholds 8/16/24/32 and keep the fastest (samples of long-lived walks
+        // favour depth-synchronous warps, short-lived ones frequent refills)
+        static const int cand[4] = {8, 16, 24, 32};
+        const uint64_t pilot = 2000000;
+        for (int m = 0; m < 2; ++m) {
+            double best = 0.0;
+            int best_r = ctx->opt_refill_min;
+            for (int rep = 0; rep < 2; ++rep)
+                for (int c = 0; c < 4; ++c) {
+                    ctx->tuned_refill[m] = cand[c];
+                    gsword_result r;
+                    int rc2 = gsword_estimate_range(ctx, (gsword_method)m, 0, pilot, 0x5EEDull, &r);
+                    if (rc2) {
+                        ctx->tuned_refill[0] = ctx->tuned_refill[1] = 0;
+                        return rc2;
+                    }
+                    double t = 0.0;
+                    if (gsword_last_kernel_seconds(ctx, &t) != GSWORD_OK) t = r.seconds;
+                    if ((rep == 0 && c == 0) || t < best) {
+                        best = t;
+                        best_r = cand[c];
+                    }
+                }
+            ctx->tuned_refill[m] = best_r;
+        }
+    }
     return GSWORD_OK;
 }
 
@@ -1099,6 +1144,8 @@ int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out) {
     for (int u = 0; u < ctx->plan.nq; ++u) out->candidates[u] = ctx->cand_count[u];
     out->cg_entries = ctx->cg_entries;
     out->build_seconds = ctx->cg_seconds;
+    out->refill_min[0] = ctx->tuned_refill[0] ? ctx->tuned_refill[0] : ctx->opt_refill_min;
+    out->refill_min[1] = ctx->tuned_refill[1] ? ctx->tuned_refill[1] : ctx->opt_refill_min;
     return GSWORD_OK;
 }
 

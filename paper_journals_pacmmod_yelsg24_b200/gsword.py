@@ -32,6 +32,7 @@ OPT_EDGE_SET = 6
 OPT_FILTER = 7
 OPT_SCHEDULE = 8
 OPT_REFILL_MIN = 9
+OPT_AUTOTUNE = 10
 SCHED_REFILL, SCHED_SAMPLE_SYNC, SCHED_INHERIT = 0, 1, 2
 FILTER_LABEL, FILTER_LDF, FILTER_NLF = 0, 1, 2
 CUDA_STREAM_LEGACY = 0x1  # cudaStreamLegacy
@@ -69,7 +70,8 @@ class _Result(ctypes.Structure):
 
 class _QueryStats(ctypes.Structure):
     _fields_ = [("nq", ctypes.c_int32), ("filter", ctypes.c_int32), ("candidates", ctypes.c_uint64 * MAX_QV),
-                ("cg_entries", ctypes.c_uint64), ("build_seconds", ctypes.c_double)]
+                ("cg_entries", ctypes.c_uint64), ("build_seconds", ctypes.c_double),
+                ("refill_min", ctypes.c_int32 * 2)]
 
 
 class _PlanInfo(ctypes.Structure):
@@ -297,7 +299,8 @@ class Context:
         st = _QueryStats()
         _check(_lib.gsword_query_info(self._h, ctypes.byref(st)))
         return {"nq": st.nq, "filter": st.filter, "candidates": list(st.candidates)[:st.nq],
-                "cg_entries": int(st.cg_entries), "build_seconds": st.build_seconds}
+                "cg_entries": int(st.cg_entries), "build_seconds": st.build_seconds,
+                "refill_min": list(st.refill_min)}
 
     # convenience for workloads.gen.Graph / Query objects
     def load_graph_obj(self, g) -> None:

@@ -506,3 +506,18 @@ def test_load_graph_device_equals_host(ctx, G, c0):
     with pytest.raises(G.GswordError) as e:
         ctx.load_graph_device(torch.as_tensor(g.row_ptr).cuda(), bad, torch.as_tensor(g.labels).cuda(), g.n_labels)
     assert e.value.status == -5
+
+
+def test_autotune_does_not_change_results(ctx, G, c0):
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    q = qs[1]
+    ctx.set_option(G.OPT_AUTOTUNE, 0)
+    ctx.load_query_obj(q)
+    ref = {m: ctx.trace_samples(m, 0, 30_000, 4) for m in (0, 1)}
+    ctx.set_option(G.OPT_AUTOTUNE, 1)
+    ctx.load_query_obj(q)
+    info = ctx.query_info()
+    assert all(r in (8, 16, 24, 32) for r in info["refill_min"])
+    for m in (0, 1):
+        assert ctx.trace_samples(m, 0, 30_000, 4).tobytes() == ref[m].tobytes()
