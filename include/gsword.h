@@ -130,7 +130,9 @@ typedef enum {
     GSWORD_OPT_BLOCKS_PER_SM = 0,  /* persistent CTAs per SM; 0 = occupancy maximum  */
     GSWORD_OPT_THREADS = 1,        /* threads per CTA (multiple of 32, 64..256)       */
     GSWORD_OPT_CHUNK = 2,          /* sample ids a warp takes from the queue at once  */
-    GSWORD_OPT_L2_PERSIST = 3,     /* 1 = L2 access-policy window over the adjacency  */
+    GSWORD_OPT_L2_PERSIST = 3,     /* L2 access-policy window: 0 none, 1 adjacency,   */
+                                   /* 2 (default) edge filter + seg; sets the        */
+                                   /* device's persisting-L2 limit                    */
     GSWORD_OPT_COOP_THRESHOLD = 4, /* Alley |S_p| above which the warp refines it in   */
                                    /* 32-element chunks (0..128; below: task pool)    */
     GSWORD_OPT_BLOOM = 5,          /* 1 = edge Bloom pre-test (L2-resident filter)    */
@@ -149,6 +151,8 @@ typedef enum {
     GSWORD_OPT_AUTOTUNE = 10,      /* 1 (default): gsword_load_query times pilots of   */
                                    /* refill thresholds 8/16/24/32 per method and     */
                                    /* keeps the fastest; results are unaffected       */
+    GSWORD_OPT_BLOOM_BITS = 11,    /* edge filter bits per undirected edge (2..64,    */
+                                   /* default 16), applied at the next graph load     */
     GSWORD_OPT_FILTER = 7          /* candidate filter applied by the next            */
                                    /* gsword_load_query: 0 label only, 1 LDF, 2 NLF   */
                                    /* (1-2 build the candidate graph, reading A21)    */
@@ -298,6 +302,12 @@ int gsword_phase_cycles(gsword_ctx* ctx, double* out8);
 /* Device time (CUDA events on the context stream) of the last sampling-kernel launch
  * alone (without the queue reset and the grid reduction).  Waits for that launch. */
 int gsword_last_kernel_seconds(gsword_ctx* ctx, double* seconds);
+
+/* Measurement aid (SURVEY §8(d) "K5"): the random-gather roofline of this device — one
+ * 4-byte load per 32-byte sector at uniformly random positions of a buffer_bytes buffer,
+ * `inflight` (1..8) independent dependent-load chains per thread, 8 CTAs x 256 threads per
+ * SM.  *sectors_per_s receives the sustained sector rate (x 32 B = bytes/s). */
+int gsword_gather_roofline(gsword_ctx* ctx, uint64_t buffer_bytes, int inflight, double* sectors_per_s);
 
 /* Launch geometry used by the last estimate: grid CTAs, threads per CTA, kernel
  * launches per estimate.  Any pointer may be NULL. */

@@ -249,9 +249,10 @@ struct gsword_ctx {
     int opt_blocks_per_sm = 0;
     int opt_threads = 256;
     int opt_chunk = 256;
-    int opt_l2 = 0;
+    int opt_l2 = 2;  // L2 persistence window over the filter + seg (measured 3-5% on C1 Alley)
     int opt_coop = 64;
     int opt_bloom = 1;
+    int opt_bloom_bits = 16;  // filter bits per undirected edge (applied at the next graph load)
     int opt_sched = 0;
     int opt_refill_min = 16;
     int opt_autotune = 1;         // pick the refill threshold per method with pilots at query load
@@ -709,6 +710,10 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
             if (value < 0 || value > 2) return fail(GSWORD_EINVAL, "filter must be 0 (label), 1 (LDF) or 2 (NLF)");
             ctx->opt_filter = (int)value;
             return GSWORD_OK;
+        case GSWORD_OPT_BLOOM_BITS:
+            if (value < 2 || value > 64) return fail(GSWORD_EINVAL, "bloom bits per edge must be 2..64");
+            ctx->opt_bloom_bits = (int)value;
+            return GSWORD_OK;
         case GSWORD_OPT_EDGE_SET:
             ctx->opt_eset = value ? 1 : 0;
             return GSWORD_OK;
@@ -872,7 +877,7 @@ int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const 
     // blocked Bloom filter over the edge set: ~16 bits per undirected edge, power-of-two words
     uint64_t words = 1;
     {
-        const uint64_t want = std::max<uint64_t>(1, (uint64_t)(nnz / 2) * 16 / 64);
+        const uint64_t want = std::max<uint64_t>(1, (uint64_t)(nnz / 2) * (uint64_t)ctx->opt_bloom_bits / 64);
         while (words < want) words <<= 1;
     }
     cudaError_t e;
@@ -988,7 +993,7 @@ int gsword_load_graph_device(gsword_ctx* ctx, int64_t n, const int64_t* d_row_pt
     // hot buffer (Bloom words + seg), buckets, edge set; col and labels are borrowed
     uint64_t words = 1;
     {
-        const uint64_t want = std::max<uint64_t>(1, (uint64_t)(nnz / 2) * 16 / 64);
+        const uint64_t want = std::max<uint64_t>(1, (uint64_t)(nnz / 2) * (uint64_t)ctx->opt_bloom_bits / 64);
         while (words < want) words <<= 1;
     }
     const size_t seg_n = (size_t)n * (size_t)L + 1;
@@ -1313,6 +1318,37 @@ int gsword_last_kernel_seconds(gsword_ctx* ctx, double* seconds) {
     float ms = 0.f;
     CUDA_TRY(cudaEventElapsedTime(&ms, ctx->evk0, ctx->evk1));
     *seconds = (double)ms * 1e-3;
+    return GSWORD_OK;
+}
+
+int gsword_gather_roofline(gsword_ctx* ctx, uint64_t buffer_bytes, int inflight, double* sectors_per_s) {
+    if (!ctx || !sectors_per_s || buffer_bytes < 4096 || inflight < 1 || inflight > 8)
+        return fail(GSWORD_EINVAL, "gather_roofline: bad argument");
+    CUDA_TRY(cudaSetDevice(ctx->device));
+    uint32_t* buf = nullptr;
+    unsigned long long* sink = nullptr;
+    cudaError_t e = cudaMalloc(&buf, buffer_bytes);
+    if (e != cudaSuccess) return fail(GSWORD_ENOMEM, "gather_roofline: cudaMalloc(%llu)", (unsigned long long)buffer_bytes);
+    e = cudaMalloc(&sink, sizeof(unsigned long long));
+    if (e != cudaSuccess) {
+        cudaFree(buf);
+        return fail(GSWORD_ENOMEM, "gather_roofline: cudaMalloc(sink)");
+    }
+    const int threads = 256, blocks = ctx->num_sms * 8, steps = 256;
+    const uint64_t words = buffer_bytes / 4;
+    int rc = GSWORD_OK;
+    float ms = 0.f;
+    if ((e = cudaMemsetAsync(buf, 0x5A, buffer_bytes, ctx->stream)) != cudaSuccess ||
+        (e = gsword::launch_gather(buf, words, 8, inflight, blocks, threads, sink, ctx->stream)) != cudaSuccess ||
+        (e = cudaEventRecord(ctx->ev0, ctx->stream)) != cudaSuccess ||
+        (e = gsword::launch_gather(buf, words, steps, inflight, blocks, threads, sink, ctx->stream)) != cudaSuccess ||
+        (e = cudaEventRecord(ctx->ev1, ctx->stream)) != cudaSuccess || (e = cudaStreamSynchronize(ctx->stream)) != cudaSuccess ||
+        (e = cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1)) != cudaSuccess)
+        rc = cuda_fail(e, "gather_roofline");
+    cudaFree(buf);
+    cudaFree(sink);
+    if (rc) return rc;
+    *sectors_per_s = (double)blocks * threads * (double)steps * inflight / (ms * 1e-3);
     return GSWORD_OK;
 }
 

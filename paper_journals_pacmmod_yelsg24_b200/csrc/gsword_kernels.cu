@@ -1472,6 +1472,37 @@ cudaError_t launch_label_bucket(const int32_t* labels, int64_t n, int32_t l, uin
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------- gather roofline (K5)
+// Random 4-byte loads, one per 32-byte sector, uniformly over a buffer of `words` u32:
+// `inflight` independent chains per thread, each `steps` long (the next index depends on
+// the loaded value, like the sampler's dependent gathers).  Measures the sector rate the
+// memory system sustains for this access pattern.
+__global__ void gather_kernel(const uint32_t* __restrict__ buf, uint64_t words, int steps, int inflight,
+                              unsigned long long* __restrict__ sink) {
+    const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    uint32_t acc = 0;
+    uint64_t idx[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) idx[c] = (tid * 8 + c) * 0x9E3779B97F4A7C15ull;
+    for (int s = 0; s < steps; ++s) {
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+            if (c >= inflight) break;
+            const uint64_t i = ((idx[c] >> 17) % (words >> 3)) << 3;  // sector-aligned word
+            const uint32_t v = __ldg(buf + i);
+            acc ^= v;
+            idx[c] = (idx[c] + v + 0x632BE59BD9B4E019ull) * 0xD6E8FEB86659FD93ull;
+        }
+    }
+    if (acc == 0x12345678u) atomicAdd(sink, 1ull);
+}
+
+cudaError_t launch_gather(const uint32_t* buf, uint64_t words, int steps, int inflight, int blocks, int threads,
+                          unsigned long long* sink, cudaStream_t stream) {
+    gather_kernel<<<blocks, threads, 0, stream>>>(buf, words, steps, inflight, sink);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream) {
     iota_kernel<<<148 * 4, 256, 0, stream>>>(bucket, n);
     return cudaGetLastError();

@@ -121,6 +121,8 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
 cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_out4, double* d_sectors,
                           cudaStream_t stream);
 cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream);
+cudaError_t launch_gather(const uint32_t* buf, uint64_t words, int steps, int inflight, int blocks, int threads,
+                          unsigned long long* sink, cudaStream_t stream);
 // device-side graph load (gsword_load_graph_device)
 cudaError_t launch_dev_validate(const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int64_t n,
                                 int32_t n_labels, int* d_bad, cudaStream_t stream);

@@ -33,6 +33,7 @@ OPT_FILTER = 7
 OPT_SCHEDULE = 8
 OPT_REFILL_MIN = 9
 OPT_AUTOTUNE = 10
+OPT_BLOOM_BITS = 11
 SCHED_REFILL, SCHED_SAMPLE_SYNC, SCHED_INHERIT = 0, 1, 2
 FILTER_LABEL, FILTER_LDF, FILTER_NLF = 0, 1, 2
 CUDA_STREAM_LEGACY = 0x1  # cudaStreamLegacy
@@ -101,6 +102,7 @@ def _load_library() -> ctypes.CDLL:
         "gsword_trace_samples": ([P, ctypes.c_int, U64, U64, U64, P], ctypes.c_int),
         "gsword_count_sectors": ([P, ctypes.c_int, U64, U64, U64, P], ctypes.c_int),
         "gsword_launch_info": ([P, P, P, P], ctypes.c_int),
+        "gsword_gather_roofline": ([P, U64, ctypes.c_int, P], ctypes.c_int),
         "gsword_last_kernel_seconds": ([P, P], ctypes.c_int),
         "gsword_phase_cycles": ([P, P], ctypes.c_int),
         "gsword_query_info": ([P, ctypes.POINTER(_QueryStats)], ctypes.c_int),
@@ -240,6 +242,12 @@ class Context:
 
     def set_option(self, option: int, value: int) -> None:
         _check(_lib.gsword_set_option(self._h, int(option), int(value)))
+
+    def gather_roofline(self, buffer_bytes: int, inflight: int = 8) -> float:
+        """Sustained random 32-byte-sector gather rate (sectors/s) over a buffer of that size."""
+        out = ctypes.c_double()
+        _check(_lib.gsword_gather_roofline(self._h, int(buffer_bytes), int(inflight), ctypes.byref(out)))
+        return out.value
 
     def launch_info(self) -> Dict[str, int]:
         g, t, l = ctypes.c_int(), ctypes.c_int(), ctypes.c_int()

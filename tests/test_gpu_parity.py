@@ -262,7 +262,7 @@ def test_scheduling_invariance(ctx, G, c0):
     base = {m: ctx.estimate(m, 400_000, 9) for m in (0, 1)}
     try:
         for opt, val in ((G.OPT_CHUNK, 1), (G.OPT_CHUNK, 4096), (G.OPT_BLOCKS_PER_SM, 1),
-                         (G.OPT_THREADS, 64), (G.OPT_L2_PERSIST, 1), (G.OPT_L2_PERSIST, 2), (G.OPT_BLOOM, 0),
+                         (G.OPT_THREADS, 64), (G.OPT_L2_PERSIST, 1), (G.OPT_L2_PERSIST, 0), (G.OPT_BLOOM, 0),
                          (G.OPT_EDGE_SET, 0), (G.OPT_REFILL_MIN, 1), (G.OPT_REFILL_MIN, 32)):
             ctx.set_option(opt, val)
             for m in (0, 1):
@@ -274,7 +274,7 @@ def test_scheduling_invariance(ctx, G, c0):
         ctx.set_option(G.OPT_CHUNK, 256)
         ctx.set_option(G.OPT_BLOCKS_PER_SM, 0)
         ctx.set_option(G.OPT_THREADS, 256)
-        ctx.set_option(G.OPT_L2_PERSIST, 0)
+        ctx.set_option(G.OPT_L2_PERSIST, 2)
         ctx.set_option(G.OPT_BLOOM, 1)
         ctx.set_option(G.OPT_EDGE_SET, 1)
 
