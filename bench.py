@@ -380,6 +380,12 @@ def run_ours(args):
 
     info = ctx.launch_info()
     name = {G.WJ: "wj", G.ALLEY: "alley"}
+    # random-gather roofline of this device (K5): context for the "hbm" fraction above
+    gather = {"l2_64MB_sectors_per_s": ctx.gather_roofline(64 << 20, 4),
+              "hbm_2GB_sectors_per_s": ctx.gather_roofline(2 << 30, 4)}
+    gather["dominant_kernel_sectors_per_s"] = sectors[dom] / (dom_ms * 1e-3)
+    gather["note"] = ("one 4-byte load per random 32-byte sector, full occupancy (gsword_gather_roofline); "
+                      "the kernel mixes L2 hits and DRAM misses")
     qerr = qerror_leg(G, ctx, args) if not (args.quick or args.no_qerror) else None
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -400,6 +406,7 @@ def run_ours(args):
                      "frac": achieved / peak, "traffic": traffic, "kernel": f"sample_kernel<{name[dom]}>",
                      "peak_kind": peak_kind,
                      "note": "algorithmic 32-B sectors (DESIGN.md §6 model) x 32 B / sampling-kernel time"},
+        "gather_roofline": gather,
         "cpu_baseline": cpu_base,
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": 32 * len(methods), "graph_load_s": graph_load_s,
