@@ -251,6 +251,15 @@ int gsword_select_order(gsword_ctx* ctx, int strategy, gsword_method m, int32_t 
  * Errors: ENOGRAPH, ENOQUERY, EINVAL (n_samples == 0, out NULL, bad method), ECUDA. */
 int gsword_estimate(gsword_ctx* ctx, gsword_method m, uint64_t n_samples, uint64_t seed, gsword_result* out);
 
+/* Accuracy-targeted estimate: samples 0, 1, 2, ... in doubling batches (first batch
+ * min_samples) until the relative standard error sqrt(variance)/estimate <= rel_se_target
+ * or max_samples are drawn; the result is identical to gsword_estimate over the same
+ * number of samples (batches are sample-id ranges).  A zero estimate never meets the
+ * target (the underestimation regime) and runs to max_samples.
+ * Errors: as gsword_estimate, EINVAL (target <= 0, min_samples < 2, max < min). */
+int gsword_estimate_until(gsword_ctx* ctx, gsword_method m, uint64_t seed, double rel_se_target, uint64_t min_samples,
+                          uint64_t max_samples, gsword_result* out);
+
 /* Same for the sample-id range [first_sample_id, first_sample_id + n_samples): the
  * multi-GPU split and checkpoint/resume unit (sample ids are global). */
 int gsword_estimate_range(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples,

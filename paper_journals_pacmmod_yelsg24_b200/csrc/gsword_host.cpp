@@ -1207,6 +1207,36 @@ int gsword_estimate(gsword_ctx* ctx, gsword_method m, uint64_t n_samples, uint64
     return gsword_estimate_range(ctx, m, 0, n_samples, seed, out);
 }
 
+int gsword_estimate_until(gsword_ctx* ctx, gsword_method m, uint64_t seed, double rel_se_target, uint64_t min_samples,
+                          uint64_t max_samples, gsword_result* out) {
+    if (!out || !(rel_se_target > 0.0) || min_samples < 2 || max_samples < min_samples)
+        return fail(GSWORD_EINVAL, "estimate_until: bad argument");
+    if (ctx && ctx->opt_sched == 2) return fail(GSWORD_EINVAL, "estimate_until: not with sample inheritance");
+    // sample ids 0, 1, 2, ... in doubling batches (resume = a new range, sums add exactly as
+    // for a multi-GPU split); stop once sqrt(variance) / estimate <= target or at max_samples
+    double acc[4] = {0, 0, 0, 0};
+    uint64_t done = 0, batch = min_samples;
+    double seconds = 0.0;
+    while (done < max_samples) {
+        const uint64_t cnt = std::min(batch, max_samples - done);
+        gsword_result r;
+        int rc = gsword_estimate_range(ctx, m, done, cnt, seed, &r);
+        if (rc) return rc;
+        acc[0] += r.sum;
+        acc[1] += r.sumsq;
+        acc[2] += (double)r.n_valid;
+        acc[3] += (double)r.n_samples;
+        seconds += r.seconds;
+        done += cnt;
+        gsword_finalize(acc, out);
+        if (out->estimate > 0.0 && out->variance >= 0.0 && std::sqrt(out->variance) <= rel_se_target * out->estimate)
+            break;
+        batch = std::min<uint64_t>(batch * 2, (uint64_t)1 << 40);
+    }
+    out->seconds = seconds;
+    return GSWORD_OK;
+}
+
 int gsword_trace_samples(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_t n_samples, uint64_t seed,
                          gsword_sample_record* host_out) {
     int rc = ensure_ready(ctx, (int)m);

@@ -98,6 +98,8 @@ def _load_library() -> ctypes.CDLL:
         "gsword_estimate": ([P, ctypes.c_int, U64, U64, ctypes.POINTER(_Result)], ctypes.c_int),
         "gsword_estimate_range": ([P, ctypes.c_int, U64, U64, U64, ctypes.POINTER(_Result)], ctypes.c_int),
         "gsword_estimate_async": ([P, ctypes.c_int, U64, U64, U64, P], ctypes.c_int),
+        "gsword_estimate_until": ([P, ctypes.c_int, U64, ctypes.c_double, U64, U64, ctypes.POINTER(_Result)],
+                                  ctypes.c_int),
         "gsword_finalize": ([P, ctypes.POINTER(_Result)], ctypes.c_int),
         "gsword_trace_samples": ([P, ctypes.c_int, U64, U64, U64, P], ctypes.c_int),
         "gsword_count_sectors": ([P, ctypes.c_int, U64, U64, U64, P], ctypes.c_int),
@@ -323,6 +325,14 @@ class Context:
         r = _Result()
         _check(_lib.gsword_estimate_range(self._h, int(method), int(first), int(n_samples), int(seed),
                                           ctypes.byref(r)))
+        return _result_dict(r)
+
+    def estimate_until(self, method: int, seed: int, rel_se: float, min_samples: int = 1_000_000,
+                       max_samples: int = 10**10) -> Dict[str, float]:
+        """gsword_estimate_until: sample until the relative standard error reaches rel_se."""
+        r = _Result()
+        _check(_lib.gsword_estimate_until(self._h, int(method), int(seed), float(rel_se), int(min_samples),
+                                          int(max_samples), ctypes.byref(r)))
         return _result_dict(r)
 
     def estimate_async(self, method: int, first: int, n_samples: int, seed: int, out4) -> None:

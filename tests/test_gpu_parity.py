@@ -521,3 +521,16 @@ def test_autotune_does_not_change_results(ctx, G, c0):
     assert all(r in (8, 16, 24, 32) for r in info["refill_min"])
     for m in (0, 1):
         assert ctx.trace_samples(m, 0, 30_000, 4).tobytes() == ref[m].tobytes()
+
+
+def test_estimate_until(ctx, G, c0):
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    ctx.load_query_obj(qs[0])
+    r = ctx.estimate_until(G.ALLEY, 5, rel_se=1e-3, min_samples=10_000, max_samples=10**9)
+    assert math.sqrt(r["variance"]) <= 1e-3 * r["estimate"]
+    full = ctx.estimate(G.ALLEY, r["n"], 5)  # same sample ids: same aggregate
+    assert full["n_valid"] == r["n_valid"]
+    assert full["sum"] == pytest.approx(r["sum"], rel=REL)
+    with pytest.raises(G.GswordError):
+        ctx.estimate_until(G.ALLEY, 5, rel_se=0.0)
