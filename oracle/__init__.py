@@ -77,6 +77,8 @@ def _load():
             lib.or_sample_range.restype = ctypes.c_int
             lib.or_sample_range_f.argtypes = lib.or_sample_range.argtypes + [ctypes.c_int]
             lib.or_sample_range_f.restype = ctypes.c_int
+            lib.or_sample_range_v.argtypes = lib.or_sample_range_f.argtypes + [ctypes.c_int]
+            lib.or_sample_range_v.restype = ctypes.c_int
             lib.or_candidate_sets.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, ctypes.c_int, P]
             lib.or_candidate_sets.restype = ctypes.c_int
             lib.or_trawl_range.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, ctypes.c_int,
@@ -88,6 +90,8 @@ def _load():
             lib.or_inherit_range.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, ctypes.c_int,
                                              ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_int, P, P]
             lib.or_inherit_range.restype = ctypes.c_int
+            lib.or_inherit_range_v.argtypes = lib.or_inherit_range.argtypes + [ctypes.c_int]
+            lib.or_inherit_range_v.restype = ctypes.c_int
             lib.or_count_embeddings.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, P, P]
             lib.or_count_embeddings.restype = ctypes.c_int
             lib.or_record_size.restype = ctypes.c_int
@@ -133,6 +137,10 @@ FILTER_LABEL = 0
 FILTER_LDF = 1
 FILTER_NLF = 2
 
+# Alley selection rule: count-then-index (default) or warp streaming (Alg. 3, reading A25)
+SELECT_INDEX = 0
+SELECT_STREAM = 1
+
 
 def candidate_sets(g, q, filter: int) -> np.ndarray:
     """C(u) membership, bool[nq, n] (Def. 4; filter per reading A21)."""
@@ -147,8 +155,11 @@ def candidate_sets(g, q, filter: int) -> np.ndarray:
 
 
 def sample_range(g, q, method: int, seed: int, first: int, count: int, records: bool = True,
-                 threads: int = 1, filter: int = FILTER_LABEL) -> Tuple[np.ndarray, Optional[np.ndarray]]:
-    """Y values (and records) of samples [first, first+count), in sample-id order."""
+                 threads: int = 1, filter: int = FILTER_LABEL,
+                 select: int = SELECT_INDEX) -> Tuple[np.ndarray, Optional[np.ndarray]]:
+    """Y values (and records) of samples [first, first+count), in sample-id order.
+    select: Alley's selection rule, SELECT_INDEX (count-then-index) or SELECT_STREAM (warp
+    streaming, Alg. 3, reading A25)."""
     lib = _load()
     pr = _Prepared(g, q)
     y = np.zeros(count, np.float64)
@@ -157,9 +168,10 @@ def sample_range(g, q, method: int, seed: int, first: int, count: int, records: 
     def run(a: int, b: int) -> int:
         yp = ctypes.c_void_p(y.ctypes.data + 8 * a)
         rp = ctypes.c_void_p(rec.ctypes.data + RECORD_DTYPE.itemsize * a) if records else None
-        return lib.or_sample_range_f(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq,
+        return lib.or_sample_range_v(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq,
                                      _ptr(pr.qrp), _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order),
-                                     int(method), int(seed), int(first + a), int(b - a), yp, rp, int(filter))
+                                     int(method), int(seed), int(first + a), int(b - a), yp, rp, int(filter),
+                                     int(select))
 
     if threads <= 1 or count < 2 * threads:
         rc = run(0, count) if count else 0
@@ -204,7 +216,8 @@ def trawl_range(g, q, method: int, seed: int, first: int, count: int, budget: in
     return t, st, rec
 
 
-def inherit_range(g, q, method: int, seed: int, first: int, count: int, filter: int = 0) -> Dict[str, float]:
+def inherit_range(g, q, method: int, seed: int, first: int, count: int, filter: int = 0,
+                  select: int = 0) -> Dict[str, float]:
     """Sample inheritance (Alg. 2) over groups of 32 consecutive ids (reading A24).
     estimate = sum of group totals / count; variance from the group totals (the groups are
     the independent units): m (sum G^2 - (sum G)^2 / m) / ((m - 1) count^2)."""
@@ -213,9 +226,9 @@ def inherit_range(g, q, method: int, seed: int, first: int, count: int, filter: 
     m = (count + 31) // 32
     groups = np.zeros(max(m, 1), np.float64)
     nc = np.zeros(1, np.uint64)
-    rc = lib.or_inherit_range(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq, _ptr(pr.qrp),
-                              _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order), int(method), int(seed), int(first),
-                              int(count), int(filter), _ptr(groups), _ptr(nc))
+    rc = lib.or_inherit_range_v(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq, _ptr(pr.qrp),
+                                _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order), int(method), int(seed), int(first),
+                                int(count), int(filter), _ptr(groups), _ptr(nc), int(select))
     if rc != 0:
         raise ValueError(f"oracle rejected input (rc={rc})")
     groups = groups[:m]
@@ -250,8 +263,9 @@ def aggregate(y: np.ndarray) -> Dict[str, float]:
 
 
 def estimate(g, q, method: int, seed: int, n_samples: int, first: int = 0, threads: int = 1,
-             filter: int = FILTER_LABEL) -> Dict[str, float]:
-    y, _ = sample_range(g, q, method, seed, first, n_samples, records=False, threads=threads, filter=filter)
+             filter: int = FILTER_LABEL, select: int = 0) -> Dict[str, float]:
+    y, _ = sample_range(g, q, method, seed, first, n_samples, records=False, threads=threads, filter=filter,
+                        select=select)
     return aggregate(y)
 
 

@@ -183,3 +183,22 @@ def trawl_expectation(g, q, method: int, filter: int = 0) -> Fraction:
 def inheritance_expectation_check(g, q, method, seed_values, count, inherit_fn):
     """Helper for tests: mean of the inheritance estimator over several seeds."""
     return [inherit_fn(g, q, method, s, 0, count)["estimate"] for s in seed_values]
+
+
+def alley_candidates(g, q, prefix, adj=None):
+    """The Alley candidate set C_d after matching `prefix` (label-only filter), written out
+    from its definition: the data vertices with label L_q(phi[d]) that
+    are adjacent to the match of every backward query neighbour and not already matched,
+    ascending.  Independent of the choice of driver list."""
+    adj = adj if adj is not None else _adjacency_sets(g)
+    order = [int(x) for x in q.order]
+    d = len(prefix)
+    u = order[d]
+    want = int(q.labels[u])
+    back = [j for j in range(d) if q.adj[order[j], u]]
+    if d == 0:
+        return [v for v in range(g.n) if int(g.labels[v]) == want]
+    common = set(adj[prefix[back[0]]])
+    for j in back[1:]:
+        common &= adj[prefix[j]]
+    return sorted(v for v in common if int(g.labels[v]) == want and v not in prefix)

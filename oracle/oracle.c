@@ -61,14 +61,18 @@ void or_philox4x32_10(const uint32_t ctr_in[4], const uint32_t key_in[2], uint32
     out[0] = c0; out[1] = c1; out[2] = c2; out[3] = c3;
 }
 
-/* r(sid, d): key = seed, counter = (sid, d, 0); r = x1:x0 */
-static uint64_t draw_r(uint64_t seed, uint64_t sid, uint32_t d) {
-    uint32_t ctr[4] = {(uint32_t)sid, (uint32_t)(sid >> 32), d, 0u};
+/* r(sid, d, c): key = seed, counter = (sid, d, c); r = x1:x0.  The plain
+ * samplers use c = 0; warp streaming (reading A25) uses c = 1 + element index for the
+ * per-candidate draws and c = 0x80000000 | chunk for the per-chunk merge draws. */
+static uint64_t draw_rc(uint64_t seed, uint64_t sid, uint32_t d, uint32_t c) {
+    uint32_t ctr[4] = {(uint32_t)sid, (uint32_t)(sid >> 32), d, c};
     uint32_t key[2] = {(uint32_t)seed, (uint32_t)(seed >> 32)};
     uint32_t x[4];
     or_philox4x32_10(ctr, key, x);
     return ((uint64_t)x[1] << 32) | (uint64_t)x[0];
 }
+
+static uint64_t draw_r(uint64_t seed, uint64_t sid, uint32_t d) { return draw_rc(seed, sid, d, 0u); }
 
 /* uniform index in [0, c): floor(r * c / 2^64) */
 static uint64_t uniform_index(uint64_t r, uint64_t c) {
@@ -150,8 +154,68 @@ static int64_t local_candidates(const or_graph* G, int32_t v, const uint8_t* inC
  * matched prefix M[0..d-1], draws M[d] with r(sid, d), multiplies *W by |C_d| (the running
  * product of Eq. 1 in depth order, reading A7; *W starts as |C_0| at d = 0) and validates.
  * Returns 1 if M[0..d] is still a valid partial instance, 0 if the sample died here. */
-static int step_at(const or_graph* G, const or_query* Q, int method, uint64_t seed, uint64_t sid, int d,
-                   const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
+/* Alley refine predicate (Fig. 19 AL; reading A5): x of the driver list S[p]
+ * lies in every other local list and is not an already-matched vertex. */
+static int alley_keep(int32_t x, int32_t** S, const int64_t* len, int nb, int p, const int32_t* M, int d) {
+    for (int b = 0; b < nb; ++b) {
+        if (b == p) continue;
+        if (!contains(S[b], len[b], x)) return 0;
+    }
+    for (int j = 0; j < d; ++j)
+        if (M[j] == x) return 0;
+    return 1;
+}
+
+/* Warp streaming (Alg. 3; reading A25): Refine and Sample of one Alley position
+ * streamed over the driver list cand[0..clen) with the weighted reservoir of A-Res.  Every
+ * candidate has weight w = 1 if it passes refine, else 0, so its A-Res key u^(1/w) is u.
+ * Collaborative phase (l.5-17) while at least 32 candidates remain: the 32 "workers" take
+ * cand[it .. it+32), the survivor with the largest key is the chunk's pick (ties -> lowest
+ * worker), totalW = survivors, curTotalW += totalW, and the pick replaces curV with
+ * probability totalW / curTotalW.  Independent phase (l.18-22): one candidate at a time,
+ * curTotalW += w, replace with probability w / curTotalW.  "With probability a / b" is
+ * mulhi64(u, b) < a for a fresh draw u.  Returns curTotalW (= |C_d|, Theorem 2) and the
+ * pick in *v (-1 when curTotalW = 0). */
+static int64_t stream_select(uint64_t seed, uint64_t sid, int d, const int32_t* cand, int64_t clen, int32_t** S,
+                             const int64_t* len, int nb, int p, const int32_t* M, int32_t* v) {
+    int64_t cur_iter = 0;         /* l.1 */
+    int32_t cur_v = -1;           /* l.2 (dummy) */
+    uint64_t cur_total = 0;       /* l.4 (curW is 1 for every pick: the weights are 0/1) */
+    uint32_t chunk = 0;
+    while (clen - cur_iter >= 32) {                          /* l.5 */
+        int best = -1;
+        uint64_t best_key = 0, total = 0;
+        for (int t = 0; t < 32; ++t) {                       /* worker t: cand[cur_iter + t] (l.8) */
+            int32_t x = cand[cur_iter + t];
+            if (!alley_keep(x, S, len, nb, p, M, d)) continue;  /* l.9-10: w = 0, key 0 */
+            total += 1;
+            uint64_t key = draw_rc(seed, sid, (uint32_t)d, (uint32_t)(1 + cur_iter + t));  /* l.11 */
+            if (best < 0 || key > best_key) { best = t; best_key = key; }                 /* l.12 */
+        }
+        cur_total += total;                                   /* l.13-15 */
+        if (total > 0 &&
+            uniform_index(draw_rc(seed, sid, (uint32_t)d, 0x80000000u | chunk), cur_total) < total)  /* l.16 */
+            cur_v = cand[cur_iter + best];
+        cur_iter += 32;                                       /* l.17 */
+        chunk += 1;
+    }
+    while (cur_iter < clen) {                                 /* l.18 */
+        int32_t x = cand[cur_iter];
+        if (alley_keep(x, S, len, nb, p, M, d)) {             /* l.19-20: w = 1 */
+            cur_total += 1;                                   /* l.21 */
+            if (uniform_index(draw_rc(seed, sid, (uint32_t)d, (uint32_t)(1 + cur_iter)), cur_total) < 1)
+                cur_v = x;                                    /* l.22: with probability 1 / curTotalW */
+        }
+        cur_iter += 1;
+    }
+    *v = cur_v;
+    return (int64_t)cur_total;
+}
+
+/* select: 0 = count-then-index (the default sampler), 1 = Alley by warp streaming (Alg. 3).
+ * WanderJoin has no refine stage, so `select` does not change it. */
+static int step_at(const or_graph* G, const or_query* Q, int method, int select, uint64_t seed, uint64_t sid,
+                   int d, const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
                    int32_t* M, double* W, or_record* rec) {
     if (d == 0) {
         /* seed from the global candidate set C(phi[0]) */
@@ -197,6 +261,15 @@ static int step_at(const or_graph* G, const or_query* Q, int method, uint64_t se
         }
         return 1;
     }
+    if (select == 1) {
+        int32_t v = -1;
+        clen = stream_select(seed, sid, d, cand, len[p], S, len, nb, p, M, &v);
+        *W = *W * (double)clen;
+        if (clen == 0) return 0;
+        M[d] = v;
+        if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
+        return 1;
+    }
     /* Alley Refine: keep each x of cand that lies in every other local list and is not
      * already matched (Fig. 19 AL; reading A5) */
     clen = 0;
@@ -224,10 +297,10 @@ static int step_at(const or_graph* G, const or_query* Q, int method, uint64_t se
 /* Samples positions 0 .. stop-1 (stop = |V_q| for the plain estimator; the trawling
  * prefix length d otherwise).  Returns Y = W if all `stop` positions were matched, else 0;
  * M and W are left in *Mout / *Wout. */
-static double walk(const or_graph* G, const or_query* Q, int method, uint64_t seed, uint64_t sid, int stop,
+static double walk(const or_graph* G, const or_query* Q, int method, int select, uint64_t seed, uint64_t sid, int stop,
                    const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
                    or_record* rec, int32_t* Mout, double* Wout) {
-    int32_t M[OR_MAX_QV];
+    int32_t M[OR_MAX_QV] = {0};
     double W = 0.0;
     int valid = 1, depth_reached = 0;
     if (rec) {
@@ -237,7 +310,7 @@ static double walk(const or_graph* G, const or_query* Q, int method, uint64_t se
     }
     for (int d = 0; d < stop && valid; ++d) {
         depth_reached = d;
-        valid = step_at(G, Q, method, seed, sid, d, C0, C0_len, inC, S, refine, M, &W, rec);
+        valid = step_at(G, Q, method, select, seed, sid, d, C0, C0_len, inC, S, refine, M, &W, rec);
     }
     if (rec) {
         rec->valid = (uint8_t)valid;
@@ -249,10 +322,10 @@ static double walk(const or_graph* G, const or_query* Q, int method, uint64_t se
     return valid ? W : 0.0;
 }
 
-static double one_sample(const or_graph* G, const or_query* Q, int method, uint64_t seed, uint64_t sid,
+static double one_sample(const or_graph* G, const or_query* Q, int method, int select, uint64_t seed, uint64_t sid,
                          const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
                          or_record* rec) {
-    return walk(G, Q, method, seed, sid, Q->nq, C0, C0_len, inC, S, refine, rec, NULL, NULL);
+    return walk(G, Q, method, select, seed, sid, Q->nq, C0, C0_len, inC, S, refine, rec, NULL, NULL);
 }
 
 static int load_query(or_query* Q, int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col,
@@ -303,11 +376,25 @@ int or_sample_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const
                              count, y_out, rec_out, 0);
 }
 
+int or_sample_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                      int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                      const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
+                      double* y_out, or_record* rec_out, int filter, int select);
+
 /* Run samples [first, first + count) with the candidate sets of `filter`. */
 int or_sample_range_f(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
                       int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
                       const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
                       double* y_out, or_record* rec_out, int filter) {
+    return or_sample_range_v(n, row_ptr, col, labels, nq, q_row_ptr, q_col, q_labels, order, method, seed, first,
+                             count, y_out, rec_out, filter, 0);
+}
+
+/* ... and the Alley selection rule `select` (0 count-then-index, 1 warp streaming, A25). */
+int or_sample_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                      int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                      const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
+                      double* y_out, or_record* rec_out, int filter, int select) {
     or_graph G = {n, row_ptr, col, labels};
     or_query Q;
     int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
@@ -330,7 +417,7 @@ int or_sample_range_f(int64_t n, const int64_t* row_ptr, const int32_t* col, con
     for (int b = 0; b < OR_MAX_QV; ++b) S[b] = buf + (size_t)b * (size_t)(maxdeg + 1);
     int32_t* refine = buf + (size_t)OR_MAX_QV * (size_t)(maxdeg + 1);
     for (uint64_t i = 0; i < count; ++i) {
-        double y = one_sample(&G, &Q, method, seed, first + i, C0, C0_len, inC, S, refine,
+        double y = one_sample(&G, &Q, method, select, seed, first + i, C0, C0_len, inC, S, refine,
                               rec_out ? &rec_out[i] : NULL);
         if (y_out) y_out[i] = y;
     }
@@ -514,7 +601,7 @@ int or_trawl_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const 
         trawl_state st;
         memset(&st, 0, sizeof(st));
         double W = 0.0;
-        double y = walk(&G, &Q, method, seed, sid, d, C0, C0_len, inC, S, refine, &r, st.M, &W);
+        double y = walk(&G, &Q, method, 0, seed, sid, d, C0, C0_len, inC, S, refine, &r, st.M, &W);
         uint8_t status = 0;
         double t = 0.0;
         if (r.valid) {
@@ -560,10 +647,24 @@ int or_trawl_record_size(void) { return (int)sizeof(or_trawl_record); }
  * parent and its k copies all carry W / (k + 1) (the push-down of the recursive estimator,
  * P:L902-L910).  A copy keeps drawing with its own sample id.  group_out[g] = the sum of
  * the weights of the complete instances of group g; *n_complete counts those instances. */
+int or_inherit_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int32_t nq,
+                       const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels, const int32_t* order,
+                       int method, uint64_t seed, uint64_t first, uint64_t count, int filter, double* group_out,
+                       uint64_t* n_complete, int select);
+
 int or_inherit_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int32_t nq,
                      const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels, const int32_t* order,
                      int method, uint64_t seed, uint64_t first, uint64_t count, int filter, double* group_out,
                      uint64_t* n_complete) {
+    return or_inherit_range_v(n, row_ptr, col, labels, nq, q_row_ptr, q_col, q_labels, order, method, seed, first,
+                              count, filter, group_out, n_complete, 0);
+}
+
+/* ... with the Alley selection rule `select` (inheritance + warp streaming = the paper's O2). */
+int or_inherit_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int32_t nq,
+                       const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels, const int32_t* order,
+                       int method, uint64_t seed, uint64_t first, uint64_t count, int filter, double* group_out,
+                       uint64_t* n_complete, int select) {
     or_graph G = {n, row_ptr, col, labels};
     or_query Q;
     int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
@@ -597,7 +698,7 @@ int or_inherit_range(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
             int any = 0;
             for (int l = 0; l < L; ++l) {
                 if (!alive[l]) continue;
-                alive[l] = step_at(&G, &Q, method, seed, first + g0 + (uint64_t)l, d, C0, C0_len, inC, S, refine,
+                alive[l] = step_at(&G, &Q, method, select, seed, first + g0 + (uint64_t)l, d, C0, C0_len, inC, S, refine,
                                    M[l], &W[l], NULL);
                 any |= alive[l];
             }
