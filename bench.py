@@ -374,9 +374,13 @@ def run_ours(args):
     if world == 1 and not args.no_cpu_baseline:
         cores = host_cores()
         rate, per_method, dt = oracle_rate(g, q, args.cpu_seconds, cores, args.seed)
+        rate1, per1, dt1 = oracle_rate(g, q, min(5.0, args.cpu_seconds / 3), 1, args.seed)
         cpu_base = {"value": rate, "unit": UNIT, "cores": cores, "kind": "oracle",
                     "sample": f"{per_method} WanderJoin + {per_method} Alley samples (ids [0,{per_method})), "
-                              f"same graph/query/seed, {dt:.1f} s on {cores} threads ({cpu_model()})"}
+                              f"same graph/query/seed, {dt:.1f} s on {cores} threads ({cpu_model()})",
+                    # SURVEY §8(d) oracle timing (i): the same oracle on one thread
+                    "single_thread": {"value": rate1, "cores": 1,
+                                      "sample": f"{per1} + {per1} samples, {dt1:.1f} s"}}
 
     info = ctx.launch_info()
     name = {G.WJ: "wj", G.ALLEY: "alley"}

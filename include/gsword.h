@@ -153,6 +153,12 @@ typedef enum {
                                    /* keeps the fastest; results are unaffected       */
     GSWORD_OPT_BLOOM_BITS = 11,    /* edge filter bits per undirected edge (2..64,    */
                                    /* default 16), applied at the next graph load     */
+    GSWORD_OPT_STREAMING = 12,     /* 1 = Alley draws by warp streaming (Alg. 3,      */
+                                   /* P:L914-L968, NEXT-3 comparison mode, reading    */
+                                   /* A25): same C_d and weights, a different vertex  */
+                                   /* of C_d than count-then-index; 0 (default) off.  */
+                                   /* Applies to estimates and traces with every      */
+                                   /* schedule; WanderJoin and count_sectors ignore it */
     GSWORD_OPT_FILTER = 7          /* candidate filter applied by the next            */
                                    /* gsword_load_query: 0 label only, 1 LDF, 2 NLF   */
                                    /* (1-2 build the candidate graph, reading A21)    */

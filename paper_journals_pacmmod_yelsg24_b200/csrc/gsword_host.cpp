@@ -256,6 +256,7 @@ struct gsword_ctx {
     int opt_sched = 0;
     int opt_refill_min = 16;
     int opt_autotune = 1;         // pick the refill threshold per method with pilots at query load
+    int opt_streaming = 0;        // Alley by warp streaming (Alg. 3, NEXT-3 comparison mode)
     int tuned_refill[2] = {0, 0}; // 0 = not tuned  // measured: 1.2-1.35x over refilling every round on C1, neutral on C2/C3
     int opt_eset = 1;
     // last launch
@@ -370,6 +371,7 @@ DeviceGraph device_graph(const gsword_ctx* ctx) {
 int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, uint64_t seed, double* d_out4,
         gsword_sample_record* d_records, double* d_sectors) {
     if (ctx->q_filter) mode |= gsword::kModeCG;
+    if (method == GSWORD_ALLEY && ctx->opt_streaming && (mode & 3) != gsword::kModeCount) mode |= gsword::kModeStream;
     LaunchCfg cfg;
     int rc = launch_config(ctx, method, mode, &cfg);
     if (rc) return rc;
@@ -716,6 +718,9 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
             return GSWORD_OK;
         case GSWORD_OPT_EDGE_SET:
             ctx->opt_eset = value ? 1 : 0;
+            return GSWORD_OK;
+        case GSWORD_OPT_STREAMING:
+            ctx->opt_streaming = value ? 1 : 0;
             return GSWORD_OK;
         case GSWORD_OPT_COOP_THRESHOLD:
             if (value < 0 || value > 128) return fail(GSWORD_EINVAL, "coop threshold must be 0..128");

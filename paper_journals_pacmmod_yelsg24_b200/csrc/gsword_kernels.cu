@@ -28,8 +28,10 @@ constexpr unsigned kFull = 0xffffffffu;
 // Alley drivers longer than the coop threshold (<= 64) are refined by the whole warp.
 
 // ---------------------------------------------------------------- Philox4x32-10 (A6)
-__device__ __forceinline__ uint64_t philox_r(uint64_t seed, uint64_t sid, uint32_t d) {
-    uint32_t c0 = (uint32_t)sid, c1 = (uint32_t)(sid >> 32), c2 = d, c3 = 0u;
+// counter = (sid, d, c3): c3 = 0 for the plain draws; warp streaming (reading A25) uses
+// c3 = 1 + element index (reservoir keys) and 0x80000000 | chunk (chunk merges)
+__device__ __forceinline__ uint64_t philox_rc(uint64_t seed, uint64_t sid, uint32_t d, uint32_t c3) {
+    uint32_t c0 = (uint32_t)sid, c1 = (uint32_t)(sid >> 32), c2 = d;
     uint32_t k0 = (uint32_t)seed, k1 = (uint32_t)(seed >> 32);
 #pragma unroll
     for (int i = 0; i < 10; ++i) {
@@ -45,6 +47,10 @@ __device__ __forceinline__ uint64_t philox_r(uint64_t seed, uint64_t sid, uint32
         k1 += 0xBB67AE85u;
     }
     return ((uint64_t)c1 << 32) | (uint64_t)c0;
+}
+
+__device__ __forceinline__ uint64_t philox_r(uint64_t seed, uint64_t sid, uint32_t d) {
+    return philox_rc(seed, sid, d, 0u);
 }
 
 __device__ __forceinline__ int32_t ldg_i32(const int32_t* p) { return __ldg(p); }
@@ -771,6 +777,288 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
     }
 }
 
+// ---------------------------------------------------------------- warp streaming (NEXT-3)
+// Alg. 3 (reading A25) as a comparison mode for Alley: each position's
+// Refine + Sample is streamed over the driver list.  Collaborative phase (l.5-17): while
+// some lane has >= 32 unprocessed candidates, the lowest such lane leads, every lane
+// refines one candidate of the leader's sample, the survivor with the largest reservoir
+// key (r(sid, d, 1 + i)) is the chunk's pick (warp max, ties -> lowest lane), and the
+// leader replaces its pick with probability total / curTotal (mulhi64 of the chunk draw
+// r(sid, d, 0x80000000 | c)).  Independent phase (l.18-22): each lane streams its last
+// < 32 candidates alone.  |C_d| = curTotal, so W, records and the estimator are those of
+// Alley; only the drawn vertex differs from count-then-index.  Scheduling (refill /
+// sample synchronisation / inheritance) and the epilogue mirror sample_kernel.
+template <bool CG>
+__device__ __forceinline__ bool stream_keep(const DeviceGraph& g, const uint32_t* Ms, int T, int col_of,
+                                            const PlanStep& ps, int p, int32_t x) {
+    double sec = 0.0;
+    return not_matched(Ms, T, col_of, ps.dup, x) &&
+           member_all<false>(g, Ms, T, col_of, ps.back & ~(1u << p), ps.label, x, sec);
+}
+
+template <int MODE, bool CG>
+__global__ void __launch_bounds__(256) stream_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
+                                                     const uint64_t count, const uint64_t seed, const int chunk,
+                                                     const uint32_t /*coop_threshold*/, const int sched,
+                                                     const uint32_t refill_min,
+                                                     unsigned long long* __restrict__ queue,
+                                                     Partial* __restrict__ partials,
+                                                     gsword_sample_record* __restrict__ records,
+                                                     unsigned long long* __restrict__ /*phase_out*/) {
+    __shared__ PlanStep plan_s[kMaxQV];
+    __shared__ uint8_t eidx_s[kMaxQV][kMaxQV];
+    __shared__ Partial warp_part[32];
+    extern __shared__ uint32_t Ms[];  // Ms[j * blockDim.x + tid] = M[j] of this lane
+
+    const int tid = threadIdx.x;
+    const int T = blockDim.x;
+    const int lane = tid & 31;
+    const int wbase = tid - lane;
+    const unsigned lt_mask = (1u << lane) - 1u;
+    if (tid < kMaxQV) plan_s[tid] = plan_in.step[tid];
+    if (tid < kMaxQV * kMaxQV) eidx_s[tid / kMaxQV][tid % kMaxQV] = plan_in.eidx[tid / kMaxQV][tid % kMaxQV];
+    __syncthreads();
+    const int nq = plan_in.nq;
+
+    bool has = false;
+    uint64_t sid = 0;
+    int d = 0;
+    double W = 0.0;
+    double s_sum = 0.0, c_sum = 0.0, s_sq = 0.0, c_sq = 0.0;
+    unsigned long long n_valid = 0, n_done = 0;
+    uint64_t q_next = 0, q_end = 0;
+    bool exhausted = false;
+    bool member = false;
+    double g_acc = 0.0;
+    bool group_open = false;
+
+    while (true) {
+        // ---------------- A1: refill (as sample_kernel) ----------------
+        unsigned need = __ballot_sync(kFull, !has);
+        if (sched == 2 && need == kFull && group_open) {
+            double gsum = g_acc;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) gsum = __dadd_rn(gsum, shfl_xor_d(gsum, o));
+            if (lane == 0) {
+                nsum(s_sum, c_sum, gsum);
+                nsum(s_sq, c_sq, __dmul_rn(gsum, gsum));
+            }
+            g_acc = 0.0;
+            group_open = false;
+        }
+        if (sched != 0 && need != kFull) need = 0u;
+        if (sched == 0 && (uint32_t)__popc(need) < refill_min) need = 0u;
+        if (need == kFull) member = false;
+        while (need && !exhausted) {
+            if (q_next == q_end) {
+                unsigned long long base = 0;
+                if (lane == 0) base = atomicAdd(queue, (unsigned long long)chunk);
+                base = __shfl_sync(kFull, base, 0);
+                if (base >= count) {
+                    exhausted = true;
+                    break;
+                }
+                q_next = base;
+                q_end = ((uint64_t)base + (uint64_t)chunk < count) ? (uint64_t)base + (uint64_t)chunk : count;
+            }
+            const uint32_t avail = (q_end - q_next) < 32 ? (uint32_t)(q_end - q_next) : 32u;
+            const uint32_t rank = __popc(need & lt_mask);
+            if (!has && rank < avail) {
+                has = true;
+                member = true;
+                n_done += 1;
+                sid = first + q_next + rank;
+                d = 0;
+                W = 1.0;
+                if (MODE == kModeTrace) {
+                    gsword_sample_record* rec = records + (sid - first);
+                    rec->sample_id = sid;
+#pragma unroll
+                    for (int i = 0; i < kMaxQV; ++i) {
+                        rec->path[i] = -1;
+                        rec->csize[i] = 0;
+                    }
+                }
+            }
+            q_next += min((uint32_t)__popc(need), avail);
+            need = __ballot_sync(kFull, !has);
+            group_open = true;
+            if (sched != 0) break;
+        }
+        if (!__any_sync(kFull, has)) break;
+        __syncwarp();
+
+        // ---------------- seed, or GetMinCandidate (the driver list) ----------------
+        PlanStep ps = {0, 0u, 0u, 0};
+        uint32_t lo_p = 0, len_p = 0, cnt = 0, it = 0, chunk_no = 0;
+        int p = 0;
+        int32_t v = -1;
+        if (has) {
+            ps = plan_s[d];
+            if (d == 0) {
+                cnt = plan_in.seed_len;
+                if (cnt > 0) {
+                    const uint64_t k = __umul64hi(philox_r(seed, sid, 0u), (uint64_t)cnt);
+                    v = plan_in.seed_identity ? (int32_t)(plan_in.seed_lo + k) : ldg_i32(g.bucket + plan_in.seed_lo + k);
+                }
+            } else {
+                uint32_t bm = ps.back;
+                len_p = 0xFFFFFFFFu;
+                while (bm) {
+                    const int j = __ffs(bm) - 1;
+                    bm &= bm - 1;
+                    uint32_t a, b;
+                    local_run<CG>(g, eidx_s[d][j], Ms[j * T + tid], ps.label, &a, &b);
+                    if (b - a < len_p) {
+                        len_p = b - a;
+                        lo_p = a;
+                        p = j;
+                    }
+                }
+            }
+        }
+
+        // ---------------- collaborative phase (Alg. 3 l.5-17) ----------------
+        while (true) {
+            const unsigned wm = __ballot_sync(kFull, has && d > 0 && len_p - it >= 32u);
+            if (!wm) break;
+            const int L = __ffs(wm) - 1;
+            const uint32_t Llo = __shfl_sync(kFull, lo_p, L);
+            const uint32_t Lit = __shfl_sync(kFull, it, L);
+            const int Ld = __shfl_sync(kFull, d, L);
+            const int Lp = __shfl_sync(kFull, p, L);
+            const uint64_t Lsid = __shfl_sync(kFull, (unsigned long long)sid, L);
+            const PlanStep Lps = plan_s[Ld];
+            const uint32_t i = Lit + (uint32_t)lane;
+            const int32_t x = ldg_i32(g.clist + Llo + i);
+            const bool keep = stream_keep<CG>(g, Ms, T, wbase + L, Lps, Lp, x);
+            uint64_t bkey = keep ? philox_rc(seed, Lsid, (uint32_t)Ld, 1u + i) : 0ull;  // A-Res key (l.11)
+            int best = keep ? lane : -1;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {  // reduce_max (l.12), ties -> lowest lane
+                const int ob = __shfl_xor_sync(kFull, best, o);
+                const uint64_t okey = __shfl_xor_sync(kFull, (unsigned long long)bkey, o);
+                if (ob >= 0 && (best < 0 || okey > bkey || (okey == bkey && ob < best))) {
+                    best = ob;
+                    bkey = okey;
+                }
+            }
+            const uint32_t total = (uint32_t)__popc(__ballot_sync(kFull, keep));  // reduce_sum (l.13)
+            const int32_t xb = __shfl_sync(kFull, x, best < 0 ? 0 : best);
+            if (lane == L) {  // l.14-17
+                cnt += total;
+                if (total > 0 &&
+                    __umul64hi(philox_rc(seed, sid, (uint32_t)d, 0x80000000u | chunk_no), (uint64_t)cnt) < total)
+                    v = xb;
+                it += 32u;
+                chunk_no += 1u;
+            }
+        }
+
+        // ---------------- independent phase (Alg. 3 l.18-22) ----------------
+        if (has && d > 0) {
+            for (; it < len_p; ++it) {
+                const int32_t x = ldg_i32(g.clist + lo_p + it);
+                if (stream_keep<CG>(g, Ms, T, tid, ps, p, x)) {
+                    cnt += 1u;
+                    if (__umul64hi(philox_rc(seed, sid, (uint32_t)d, 1u + it), (uint64_t)cnt) == 0ull) v = x;
+                }
+            }
+        }
+
+        // ---------------- epilogue (as sample_kernel) ----------------
+        if (has) {
+            W = (d == 0) ? (double)cnt : __dmul_rn(W, (double)cnt);
+            if (MODE == kModeTrace) {
+                gsword_sample_record* rec = records + (sid - first);
+                rec->csize[d] = cnt;
+                rec->path[d] = (cnt > 0) ? v : -1;
+            }
+            const bool dead = cnt == 0;
+            bool complete = false;
+            if (!dead) {
+                Ms[d * T + tid] = (uint32_t)v;
+                if (d + 1 == nq) complete = true;
+            }
+            if (dead || complete) {
+                if (complete) {
+                    n_valid += 1;
+                    if (sched == 2) {
+                        g_acc = __dadd_rn(g_acc, W);
+                    } else {
+                        nsum(s_sum, c_sum, W);
+                        nsum(s_sq, c_sq, __dmul_rn(W, W));
+                    }
+                }
+                if (MODE == kModeTrace) {
+                    gsword_sample_record* rec = records + (sid - first);
+                    rec->valid = complete ? 1 : 0;
+                    rec->depth_reached = (uint8_t)d;
+                    rec->weight = W;
+                }
+                has = false;
+            } else {
+                d += 1;
+            }
+        }
+        __syncwarp();
+        if (sched == 2) {
+            const unsigned alive_m = __ballot_sync(kFull, has);
+            const unsigned idle_m = __ballot_sync(kFull, member && !has);
+            if (alive_m != 0u && idle_m != 0u) {
+                const int par = __ffs(alive_m) - 1;
+                const double Wn = __ddiv_rn(__shfl_sync(kFull, W, par), (double)(__popc(idle_m) + 1));
+                const int dp = __shfl_sync(kFull, d, par);
+                __syncwarp();
+                if (lane == par) W = Wn;
+                if ((idle_m >> lane) & 1u) {
+                    for (int j = 0; j < dp; ++j) Ms[j * T + tid] = Ms[j * T + wbase + par];
+                    d = dp;
+                    W = Wn;
+                    has = true;
+                }
+                __syncwarp();
+            }
+        }
+    }
+    if (sched == 2 && group_open) {
+        double gsum = g_acc;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) gsum = __dadd_rn(gsum, shfl_xor_d(gsum, o));
+        if (lane == 0) {
+            nsum(s_sum, c_sum, gsum);
+            nsum(s_sq, c_sq, __dmul_rn(gsum, gsum));
+        }
+    }
+
+    // ---------------- A10: warp -> CTA partial, fixed order ----------------
+    double sh = __dadd_rn(s_sum, c_sum), sl = __dsub_rn(c_sum, __dsub_rn(sh, s_sum));
+    double qh = __dadd_rn(s_sq, c_sq), ql = __dsub_rn(c_sq, __dsub_rn(qh, s_sq));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const double bh = shfl_xor_d(sh, o), bl = shfl_xor_d(sl, o);
+        const double ch = shfl_xor_d(qh, o), cl = shfl_xor_d(ql, o);
+        dd_add(sh, sl, bh, bl);
+        dd_add(qh, ql, ch, cl);
+        n_valid += __shfl_xor_sync(kFull, n_valid, o);
+        n_done += __shfl_xor_sync(kFull, n_done, o);
+    }
+    const int warp = tid >> 5;
+    if (lane == 0) warp_part[warp] = Partial{sh, sl, qh, ql, n_valid, n_done, 0.0, 0.0};
+    __syncthreads();
+    if (tid == 0) {
+        Partial acc = warp_part[0];
+        for (int w = 1; w < (T >> 5); ++w) {
+            const Partial& o = warp_part[w];
+            dd_add(acc.sum_hi, acc.sum_lo, o.sum_hi, o.sum_lo);
+            dd_add(acc.sq_hi, acc.sq_lo, o.sq_hi, o.sq_lo);
+            acc.valid += o.valid;
+            acc.n += o.n;
+        }
+        partials[blockIdx.x] = acc;
+    }
+}
+
 // ---------------------------------------------------------------- trawling (NEXT-2)
 // Alg. 4 (reading A23): per sample, d ~ P(d = j) proportional to 2^-j,
 // j in [3, |V_q|], drawn exactly in integers from r(sid, 31); the first d
@@ -1226,6 +1514,10 @@ const void* kernel_ptr() {
 
 template <bool CG>
 const void* select_kernel_cg(int method, int mode) {
+    if (mode & kModeStream) {  // warp streaming (Alley only; the host never asks for WJ or count)
+        return (mode & 3) == kModeTrace ? reinterpret_cast<const void*>(&stream_kernel<kModeTrace, CG>)
+                                        : reinterpret_cast<const void*>(&stream_kernel<kModeEstimate, CG>);
+    }
     if (method == GSWORD_WJ) {
         if (mode == kModeTrace) return kernel_ptr<GSWORD_WJ, kModeTrace, CG>();
         if (mode == kModeCount) return kernel_ptr<GSWORD_WJ, kModeCount, CG>();

@@ -160,6 +160,12 @@ cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int
                                uint64_t mask, cudaStream_t stream);
 int max_blocks_per_sm(int method, int mode, int threads, size_t* smem_bytes);
 
-enum Mode { kModeEstimate = 0, kModeTrace = 1, kModeCount = 2, kModeCG = 4 /* flag: candidate graph */ };
+enum Mode {
+    kModeEstimate = 0,
+    kModeTrace = 1,
+    kModeCount = 2,
+    kModeCG = 4,     // flag: candidate graph
+    kModeStream = 8  // flag: Alley by warp streaming (Alg. 3, NEXT-3)
+};
 
 }  // namespace gsword

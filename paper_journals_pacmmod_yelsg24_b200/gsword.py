@@ -34,6 +34,7 @@ OPT_SCHEDULE = 8
 OPT_REFILL_MIN = 9
 OPT_AUTOTUNE = 10
 OPT_BLOOM_BITS = 11
+OPT_STREAMING = 12  # Alley by warp streaming (Alg. 3, reading A25)
 SCHED_REFILL, SCHED_SAMPLE_SYNC, SCHED_INHERIT = 0, 1, 2
 FILTER_LABEL, FILTER_LDF, FILTER_NLF = 0, 1, 2
 CUDA_STREAM_LEGACY = 0x1  # cudaStreamLegacy
