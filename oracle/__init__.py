@@ -140,6 +140,9 @@ FILTER_NLF = 2
 # Alley selection rule: count-then-index (default) or warp streaming (Alg. 3, reading A25)
 SELECT_INDEX = 0
 SELECT_STREAM = 1
+# comparison variants of readings A3 / A5 (bit flags, combined with the selection rule)
+VARIANT_WJ_PARENT_FIRST = 2
+VARIANT_ALLEY_DUPCHECK_POST = 4
 
 
 def candidate_sets(g, q, filter: int) -> np.ndarray:
@@ -155,11 +158,11 @@ def candidate_sets(g, q, filter: int) -> np.ndarray:
 
 
 def sample_range(g, q, method: int, seed: int, first: int, count: int, records: bool = True,
-                 threads: int = 1, filter: int = FILTER_LABEL,
-                 select: int = SELECT_INDEX) -> Tuple[np.ndarray, Optional[np.ndarray]]:
+                 threads: int = 1, filter: int = FILTER_LABEL, select: int = SELECT_INDEX,
+                 variant: int = 0) -> Tuple[np.ndarray, Optional[np.ndarray]]:
     """Y values (and records) of samples [first, first+count), in sample-id order.
     select: Alley's selection rule, SELECT_INDEX (count-then-index) or SELECT_STREAM (warp
-    streaming, Alg. 3, reading A25)."""
+    streaming, Alg. 3, reading A25).  variant: VARIANT_* bits (readings A3, A5)."""
     lib = _load()
     pr = _Prepared(g, q)
     y = np.zeros(count, np.float64)
@@ -171,7 +174,7 @@ def sample_range(g, q, method: int, seed: int, first: int, count: int, records: 
         return lib.or_sample_range_v(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq,
                                      _ptr(pr.qrp), _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order),
                                      int(method), int(seed), int(first + a), int(b - a), yp, rp, int(filter),
-                                     int(select))
+                                     int(select) | int(variant))
 
     if threads <= 1 or count < 2 * threads:
         rc = run(0, count) if count else 0
@@ -217,7 +220,7 @@ def trawl_range(g, q, method: int, seed: int, first: int, count: int, budget: in
 
 
 def inherit_range(g, q, method: int, seed: int, first: int, count: int, filter: int = 0,
-                  select: int = 0) -> Dict[str, float]:
+                  select: int = 0, variant: int = 0) -> Dict[str, float]:
     """Sample inheritance (Alg. 2) over groups of 32 consecutive ids (reading A24).
     estimate = sum of group totals / count; variance from the group totals (the groups are
     the independent units): m (sum G^2 - (sum G)^2 / m) / ((m - 1) count^2)."""
@@ -228,7 +231,7 @@ def inherit_range(g, q, method: int, seed: int, first: int, count: int, filter: 
     nc = np.zeros(1, np.uint64)
     rc = lib.or_inherit_range_v(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq, _ptr(pr.qrp),
                                 _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order), int(method), int(seed), int(first),
-                                int(count), int(filter), _ptr(groups), _ptr(nc), int(select))
+                                int(count), int(filter), _ptr(groups), _ptr(nc), int(select) | int(variant))
     if rc != 0:
         raise ValueError(f"oracle rejected input (rc={rc})")
     groups = groups[:m]
@@ -263,9 +266,9 @@ def aggregate(y: np.ndarray) -> Dict[str, float]:
 
 
 def estimate(g, q, method: int, seed: int, n_samples: int, first: int = 0, threads: int = 1,
-             filter: int = FILTER_LABEL, select: int = 0) -> Dict[str, float]:
+             filter: int = FILTER_LABEL, select: int = 0, variant: int = 0) -> Dict[str, float]:
     y, _ = sample_range(g, q, method, seed, first, n_samples, records=False, threads=threads, filter=filter,
-                        select=select)
+                        select=select, variant=variant)
     return aggregate(y)
 
 

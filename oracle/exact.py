@@ -72,9 +72,13 @@ def embeddings(g, q):
             if all(lab[f[u]] == int(q.labels[u]) for u in range(q.nq)) and all(f[b] in adj[f[a]] for a, b in edges)]
 
 
-def tree_walk(g, q, method: int, filter: int = 0) -> Tuple[Fraction, Fraction, Dict[tuple, Tuple[int, ...]]]:
+def tree_walk(g, q, method: int, filter: int = 0,
+              variant: int = 0) -> Tuple[Fraction, Fraction, Dict[tuple, Tuple[int, ...]]]:
     """Returns (E[Y], E[Y^2], cand) where cand[prefix] = the candidate list C_d the
-    sampler draws from after matching `prefix` (len(prefix) = d)."""
+    sampler draws from after matching `prefix` (len(prefix) = d).
+    variant bits (readings A3 / A5): 2 = WanderJoin walks from the first backward
+    position's list; 4 = Alley keeps matched vertices in C_d and a drawn one ends the sample
+    (Fig. 19 DupCheck after Sample)."""
     adj = _adjacency_sets(g)
     order = [int(x) for x in q.order]
     nq = q.nq
@@ -92,10 +96,12 @@ def tree_walk(g, q, method: int, filter: int = 0) -> Tuple[Fraction, Fraction, D
         back = [j for j in range(d) if q.adj[order[j], u]]
         lists = [local(prefix[j], u) for j in back]
         p = min(range(len(back)), key=lambda b: (len(lists[b]), b))
-        if method == 0:  # WanderJoin: the smallest local list, unfiltered
+        if method == 0:  # WanderJoin: the smallest local list (or the first one), unfiltered
+            if variant & 2:
+                p = 0
             return lists[p], (back, lists, p)
         inter = [x for x in lists[p] if all(x in set(lists[b]) for b in range(len(back)))
-                 and x not in prefix]
+                 and (variant & 4 or x not in prefix)]
         return inter, None
 
     ey = Fraction(0)
@@ -121,6 +127,8 @@ def tree_walk(g, q, method: int, filter: int = 0) -> Tuple[Fraction, Fraction, D
                     continue
                 if any(v not in set(lists[b]) for b in range(len(back)) if b != p):
                     continue
+            if method == 1 and variant & 4 and v in prefix:
+                continue  # the post-sampling DupCheck kills the sample
             stack.append((prefix + (v,), p2, w2))
     return ey, ey2, cand
 

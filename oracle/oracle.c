@@ -154,15 +154,28 @@ static int64_t local_candidates(const or_graph* G, int32_t v, const uint8_t* inC
  * matched prefix M[0..d-1], draws M[d] with r(sid, d), multiplies *W by |C_d| (the running
  * product of Eq. 1 in depth order, reading A7; *W starts as |C_0| at d = 0) and validates.
  * Returns 1 if M[0..d] is still a valid partial instance, 0 if the sample died here. */
+/* Per-call flags of the sampler (readings A3, A5, A25):
+ *   OR_SELECT_STREAM        Alley draws by warp streaming (Alg. 3) instead of count-then-index
+ *   OR_WJ_PARENT_FIRST      WanderJoin walks from the FIRST backward position's list instead
+ *                           of the smallest (the "previously selected vertex" of P:L538)
+ *   OR_ALLEY_DUPCHECK_POST  Alley's refine keeps matched vertices; a drawn matched vertex
+ *                           kills the sample (Fig. 19 AL Validate/DupCheck) */
+#define OR_SELECT_STREAM 1
+#define OR_WJ_PARENT_FIRST 2
+#define OR_ALLEY_DUPCHECK_POST 4
+
 /* Alley refine predicate (Fig. 19 AL; reading A5): x of the driver list S[p]
- * lies in every other local list and is not an already-matched vertex. */
-static int alley_keep(int32_t x, int32_t** S, const int64_t* len, int nb, int p, const int32_t* M, int d) {
+ * lies in every other local list and (unless the DupCheck is deferred to after sampling) is
+ * not an already-matched vertex. */
+static int alley_keep(int32_t x, int32_t** S, const int64_t* len, int nb, int p, const int32_t* M, int d,
+                      int check_matched) {
     for (int b = 0; b < nb; ++b) {
         if (b == p) continue;
         if (!contains(S[b], len[b], x)) return 0;
     }
-    for (int j = 0; j < d; ++j)
-        if (M[j] == x) return 0;
+    if (check_matched)
+        for (int j = 0; j < d; ++j)
+            if (M[j] == x) return 0;
     return 1;
 }
 
@@ -177,7 +190,7 @@ static int alley_keep(int32_t x, int32_t** S, const int64_t* len, int nb, int p,
  * mulhi64(u, b) < a for a fresh draw u.  Returns curTotalW (= |C_d|, Theorem 2) and the
  * pick in *v (-1 when curTotalW = 0). */
 static int64_t stream_select(uint64_t seed, uint64_t sid, int d, const int32_t* cand, int64_t clen, int32_t** S,
-                             const int64_t* len, int nb, int p, const int32_t* M, int32_t* v) {
+                             const int64_t* len, int nb, int p, const int32_t* M, int check_matched, int32_t* v) {
     int64_t cur_iter = 0;         /* l.1 */
     int32_t cur_v = -1;           /* l.2 (dummy) */
     uint64_t cur_total = 0;       /* l.4 (curW is 1 for every pick: the weights are 0/1) */
@@ -187,7 +200,7 @@ static int64_t stream_select(uint64_t seed, uint64_t sid, int d, const int32_t* 
         uint64_t best_key = 0, total = 0;
         for (int t = 0; t < 32; ++t) {                       /* worker t: cand[cur_iter + t] (l.8) */
             int32_t x = cand[cur_iter + t];
-            if (!alley_keep(x, S, len, nb, p, M, d)) continue;  /* l.9-10: w = 0, key 0 */
+            if (!alley_keep(x, S, len, nb, p, M, d, check_matched)) continue;  /* l.9-10: w = 0 */
             total += 1;
             uint64_t key = draw_rc(seed, sid, (uint32_t)d, (uint32_t)(1 + cur_iter + t));  /* l.11 */
             if (best < 0 || key > best_key) { best = t; best_key = key; }                 /* l.12 */
@@ -201,7 +214,7 @@ static int64_t stream_select(uint64_t seed, uint64_t sid, int d, const int32_t* 
     }
     while (cur_iter < clen) {                                 /* l.18 */
         int32_t x = cand[cur_iter];
-        if (alley_keep(x, S, len, nb, p, M, d)) {             /* l.19-20: w = 1 */
+        if (alley_keep(x, S, len, nb, p, M, d, check_matched)) {  /* l.19-20: w = 1 */
             cur_total += 1;                                   /* l.21 */
             if (uniform_index(draw_rc(seed, sid, (uint32_t)d, (uint32_t)(1 + cur_iter)), cur_total) < 1)
                 cur_v = x;                                    /* l.22: with probability 1 / curTotalW */
@@ -212,9 +225,12 @@ static int64_t stream_select(uint64_t seed, uint64_t sid, int d, const int32_t* 
     return (int64_t)cur_total;
 }
 
-/* select: 0 = count-then-index (the default sampler), 1 = Alley by warp streaming (Alg. 3).
- * WanderJoin has no refine stage, so `select` does not change it. */
-static int step_at(const or_graph* G, const or_query* Q, int method, int select, uint64_t seed, uint64_t sid,
+/* One position d of a sample (method 0 = WanderJoin, 1 = Alley): forms C_d from the
+ * matched prefix M[0..d-1], draws M[d] with r(sid, d), multiplies *W by |C_d| (the running
+ * product of Eq. 1 in depth order, reading A7; *W starts as |C_0| at d = 0) and validates.
+ * `flags`: OR_* above (0 = the default sampler).  Returns 1 if M[0..d] is still a valid
+ * partial instance, 0 if the sample died here. */
+static int step_at(const or_graph* G, const or_query* Q, int method, int flags, uint64_t seed, uint64_t sid,
                    int d, const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
                    int32_t* M, double* W, or_record* rec) {
     if (d == 0) {
@@ -239,6 +255,7 @@ static int step_at(const or_graph* G, const or_query* Q, int method, int select,
         len[b] = local_candidates(G, M[B[b]], inC + (int64_t)u * G->n, S[b]);
         if (len[b] < len[p]) p = b;
     }
+    if (method == 0 && (flags & OR_WJ_PARENT_FIRST)) p = 0; /* variant: first backward position */
     int64_t clen;
     const int32_t* cand = S[p];
     if (method == 0) {
@@ -261,43 +278,35 @@ static int step_at(const or_graph* G, const or_query* Q, int method, int select,
         }
         return 1;
     }
-    if (select == 1) {
-        int32_t v = -1;
-        clen = stream_select(seed, sid, d, cand, len[p], S, len, nb, p, M, &v);
-        *W = *W * (double)clen;
-        if (clen == 0) return 0;
-        M[d] = v;
-        if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
-        return 1;
-    }
-    /* Alley Refine: keep each x of cand that lies in every other local list and is not
-     * already matched (Fig. 19 AL; reading A5) */
-    clen = 0;
-    for (int64_t i = 0; i < len[p]; ++i) {
-        int32_t x = cand[i];
-        int keep = 1;
-        for (int b = 0; b < nb && keep; ++b) {
-            if (b == p) continue;
-            if (!contains(S[b], len[b], x)) keep = 0;
+    const int post = (flags & OR_ALLEY_DUPCHECK_POST) != 0;
+    int32_t v = -1;
+    if (flags & OR_SELECT_STREAM) {
+        clen = stream_select(seed, sid, d, cand, len[p], S, len, nb, p, M, !post, &v);
+    } else {
+        /* Alley Refine: keep each x of cand that lies in every other local list and is not
+         * already matched (Fig. 19 AL; reading A5) */
+        clen = 0;
+        for (int64_t i = 0; i < len[p]; ++i) {
+            int32_t x = cand[i];
+            if (alley_keep(x, S, len, nb, p, M, d, !post)) refine[clen++] = x;
         }
-        for (int j = 0; j < d && keep; ++j)
-            if (M[j] == x) keep = 0;
-        if (keep) refine[clen++] = x;
+        if (clen > 0) v = refine[uniform_index(draw_r(seed, sid, (uint32_t)d), (uint64_t)clen)];
     }
     *W = *W * (double)clen;
     /* empty refined set: the sample stops */
     if (clen == 0) return 0;
-    uint64_t k = uniform_index(draw_r(seed, sid, (uint32_t)d), (uint64_t)clen);
-    int32_t v = refine[k];
     M[d] = v;
     if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
+    if (post) /* Fig. 19 AL Validate: DupCheck of the drawn vertex */
+        for (int j = 0; j < d; ++j)
+            if (M[j] == v) return 0;
     return 1;
 }
 
 /* Samples positions 0 .. stop-1 (stop = |V_q| for the plain estimator; the trawling
  * prefix length d otherwise).  Returns Y = W if all `stop` positions were matched, else 0;
  * M and W are left in *Mout / *Wout. */
-static double walk(const or_graph* G, const or_query* Q, int method, int select, uint64_t seed, uint64_t sid, int stop,
+static double walk(const or_graph* G, const or_query* Q, int method, int flags, uint64_t seed, uint64_t sid, int stop,
                    const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
                    or_record* rec, int32_t* Mout, double* Wout) {
     int32_t M[OR_MAX_QV] = {0};
@@ -310,7 +319,7 @@ static double walk(const or_graph* G, const or_query* Q, int method, int select,
     }
     for (int d = 0; d < stop && valid; ++d) {
         depth_reached = d;
-        valid = step_at(G, Q, method, select, seed, sid, d, C0, C0_len, inC, S, refine, M, &W, rec);
+        valid = step_at(G, Q, method, flags, seed, sid, d, C0, C0_len, inC, S, refine, M, &W, rec);
     }
     if (rec) {
         rec->valid = (uint8_t)valid;
@@ -322,10 +331,10 @@ static double walk(const or_graph* G, const or_query* Q, int method, int select,
     return valid ? W : 0.0;
 }
 
-static double one_sample(const or_graph* G, const or_query* Q, int method, int select, uint64_t seed, uint64_t sid,
+static double one_sample(const or_graph* G, const or_query* Q, int method, int flags, uint64_t seed, uint64_t sid,
                          const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
                          or_record* rec) {
-    return walk(G, Q, method, select, seed, sid, Q->nq, C0, C0_len, inC, S, refine, rec, NULL, NULL);
+    return walk(G, Q, method, flags, seed, sid, Q->nq, C0, C0_len, inC, S, refine, rec, NULL, NULL);
 }
 
 static int load_query(or_query* Q, int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col,
@@ -379,7 +388,7 @@ int or_sample_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const
 int or_sample_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
                       int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
                       const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
-                      double* y_out, or_record* rec_out, int filter, int select);
+                      double* y_out, or_record* rec_out, int filter, int flags);
 
 /* Run samples [first, first + count) with the candidate sets of `filter`. */
 int or_sample_range_f(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
@@ -390,11 +399,11 @@ int or_sample_range_f(int64_t n, const int64_t* row_ptr, const int32_t* col, con
                              count, y_out, rec_out, filter, 0);
 }
 
-/* ... and the Alley selection rule `select` (0 count-then-index, 1 warp streaming, A25). */
+/* ... and the sampler flags OR_* (streaming selection, readings A3/A5 variants). */
 int or_sample_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
                       int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
                       const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
-                      double* y_out, or_record* rec_out, int filter, int select) {
+                      double* y_out, or_record* rec_out, int filter, int flags) {
     or_graph G = {n, row_ptr, col, labels};
     or_query Q;
     int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
@@ -417,7 +426,7 @@ int or_sample_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, con
     for (int b = 0; b < OR_MAX_QV; ++b) S[b] = buf + (size_t)b * (size_t)(maxdeg + 1);
     int32_t* refine = buf + (size_t)OR_MAX_QV * (size_t)(maxdeg + 1);
     for (uint64_t i = 0; i < count; ++i) {
-        double y = one_sample(&G, &Q, method, select, seed, first + i, C0, C0_len, inC, S, refine,
+        double y = one_sample(&G, &Q, method, flags, seed, first + i, C0, C0_len, inC, S, refine,
                               rec_out ? &rec_out[i] : NULL);
         if (y_out) y_out[i] = y;
     }
@@ -650,7 +659,7 @@ int or_trawl_record_size(void) { return (int)sizeof(or_trawl_record); }
 int or_inherit_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int32_t nq,
                        const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels, const int32_t* order,
                        int method, uint64_t seed, uint64_t first, uint64_t count, int filter, double* group_out,
-                       uint64_t* n_complete, int select);
+                       uint64_t* n_complete, int flags);
 
 int or_inherit_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int32_t nq,
                      const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels, const int32_t* order,
@@ -660,11 +669,11 @@ int or_inherit_range(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
                               count, filter, group_out, n_complete, 0);
 }
 
-/* ... with the Alley selection rule `select` (inheritance + warp streaming = the paper's O2). */
+/* ... with the sampler flags OR_* (inheritance + warp streaming = the paper's O2). */
 int or_inherit_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int32_t nq,
                        const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels, const int32_t* order,
                        int method, uint64_t seed, uint64_t first, uint64_t count, int filter, double* group_out,
-                       uint64_t* n_complete, int select) {
+                       uint64_t* n_complete, int flags) {
     or_graph G = {n, row_ptr, col, labels};
     or_query Q;
     int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
@@ -698,7 +707,7 @@ int or_inherit_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, co
             int any = 0;
             for (int l = 0; l < L; ++l) {
                 if (!alive[l]) continue;
-                alive[l] = step_at(&G, &Q, method, select, seed, first + g0 + (uint64_t)l, d, C0, C0_len, inC, S, refine,
+                alive[l] = step_at(&G, &Q, method, flags, seed, first + g0 + (uint64_t)l, d, C0, C0_len, inC, S, refine,
                                    M[l], &W[l], NULL);
                 any |= alive[l];
             }

@@ -22,8 +22,9 @@ ap.add_argument("--filter", type=int, default=0)
 args = ap.parse_args()
 OPT = {"coop": G.OPT_COOP_THRESHOLD, "threads": G.OPT_THREADS, "chunk": G.OPT_CHUNK, "bps": G.OPT_BLOCKS_PER_SM,
        "l2": G.OPT_L2_PERSIST, "bloom": G.OPT_BLOOM, "eset": G.OPT_EDGE_SET,
-       "sched": G.OPT_SCHEDULE, "rmin": G.OPT_REFILL_MIN}
-DEF = {"coop": 64, "threads": 256, "chunk": 256, "bps": 0, "l2": 2, "bloom": 1, "eset": 1, "sched": 0, "rmin": 16}
+       "sched": G.OPT_SCHEDULE, "rmin": G.OPT_REFILL_MIN, "stream": G.OPT_STREAMING}
+DEF = {"coop": 64, "threads": 256, "chunk": 256, "bps": 0, "l2": 2, "bloom": 1, "eset": 1, "sched": 0, "rmin": 16,
+       "stream": 0}
 grid = json.loads(args.grid)
 g, qs = gen.CONFIGS[args.config]()
 queries = qs if args.query < 0 else [qs[args.query]]
