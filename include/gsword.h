@@ -34,6 +34,18 @@ typedef struct gsword_ctx gsword_ctx; /* opaque */
 /* Random-walk estimators (P:L538 WanderJoin, P:L540 Alley). */
 typedef enum { GSWORD_WJ = 0, GSWORD_ALLEY = 1 } gsword_method;
 
+/* Comparison variants (GSWORD_OPT_VARIANT bits) of the two passages the paper leaves open:
+ *  WJ_PARENT_FIRST (reading A3; "a vertex that has been previously selected"):
+ *      WanderJoin draws from the label-filtered list of the FIRST backward position
+ *      j = min B(d) instead of the smallest list (GetMinCandidate, Alg. 1 l.8);
+ *      the other backward neighbours are validated as usual.
+ *  ALLEY_DUPCHECK_POST (reading A5; Fig. 19 AL Validate): Alley's refined
+ *      set keeps matched vertices (|C_d| counts them) and a drawn vertex equal to a
+ *      matched one kills the sample after the draw (recorded like a WanderJoin
+ *      validation failure: path[d] = v, csize[d] = |C_d|, valid = 0).
+ * Both variants are unbiased; the per-sample results differ from the default. */
+typedef enum { GSWORD_VARIANT_WJ_PARENT_FIRST = 2, GSWORD_VARIANT_ALLEY_DUPCHECK_POST = 4 } gsword_variant;
+
 typedef enum {
     GSWORD_OK = 0,
     GSWORD_EINVAL = -1,   /* bad argument (NULL pointer, unknown method, label out of range) */
@@ -159,6 +171,11 @@ typedef enum {
                                    /* of C_d than count-then-index; 0 (default) off.  */
                                    /* Applies to estimates and traces with every      */
                                    /* schedule; WanderJoin and count_sectors ignore it */
+    GSWORD_OPT_VARIANT = 13,       /* comparison variants of the sampler (bit flags,  */
+                                   /* gsword_variant; default 0 = readings A3/A5 as   */
+                                   /* in SURVEY R3-R5).  Applies to estimates and     */
+                                   /* traces (every schedule, streaming included);    */
+                                   /* trawling ignores it                             */
     GSWORD_OPT_FILTER = 7          /* candidate filter applied by the next            */
                                    /* gsword_load_query: 0 label only, 1 LDF, 2 NLF   */
                                    /* (1-2 build the candidate graph, reading A21)    */

@@ -257,6 +257,7 @@ struct gsword_ctx {
     int opt_refill_min = 16;
     int opt_autotune = 1;         // pick the refill threshold per method with pilots at query load
     int opt_streaming = 0;        // Alley by warp streaming (Alg. 3, NEXT-3 comparison mode)
+    int opt_variant = 0;          // GSWORD_VARIANT_* bits (readings A3/A5 comparison variants)
     int tuned_refill[2] = {0, 0}; // 0 = not tuned  // measured: 1.2-1.35x over refilling every round on C1, neutral on C2/C3
     int opt_eset = 1;
     // last launch
@@ -378,7 +379,8 @@ int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, u
     CUDA_TRY(cudaEventRecord(ctx->evk0, ctx->stream));
     const bool counting = (mode & 3) == gsword::kModeCount;
     if (counting) CUDA_TRY(cudaMemsetAsync(ctx->d_phase, 0, 8 * sizeof(unsigned long long), ctx->stream));
-    cudaError_t e = gsword::launch_sample(method, mode, device_graph(ctx), ctx->plan, cfg, first, count, seed,
+    cudaError_t e = gsword::launch_sample(method, mode, device_graph(ctx),
+                                          gsword::plan_variant(ctx->plan, method, ctx->opt_variant), cfg, first, count, seed,
                                           ctx->d_queue, ctx->d_partials, d_records,
                                           counting ? ctx->d_phase : nullptr, ctx->stream);
     if (e != cudaSuccess) return cuda_fail(e, "launch sample kernel");
@@ -721,6 +723,11 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
             return GSWORD_OK;
         case GSWORD_OPT_STREAMING:
             ctx->opt_streaming = value ? 1 : 0;
+            return GSWORD_OK;
+        case GSWORD_OPT_VARIANT:
+            if (value & ~(int64_t)(GSWORD_VARIANT_WJ_PARENT_FIRST | GSWORD_VARIANT_ALLEY_DUPCHECK_POST))
+                return fail(GSWORD_EINVAL, "unknown variant bits 0x%llx", (unsigned long long)value);
+            ctx->opt_variant = (int)value;
             return GSWORD_OK;
         case GSWORD_OPT_COOP_THRESHOLD:
             if (value < 0 || value > 128) return fail(GSWORD_EINVAL, "coop threshold must be 0..128");

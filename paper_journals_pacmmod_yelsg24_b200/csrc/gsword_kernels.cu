@@ -245,6 +245,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
     __shared__ uint32_t qadj_s[kMaxQV];
     __shared__ uint8_t eidx_s[kMaxQV][kMaxQV];
     __shared__ uint8_t uq_s[kMaxQV];
+    __shared__ uint32_t pdup_s[kMaxQV];  // variant A5: post-draw DupCheck positions
     __shared__ uint32_t res_s[256];   // Alley task-pool results per lane (adjacent matched vertices)
     __shared__ uint32_t rm_s[4][256];  // Alley task-pool results per lane: refine-mask removals (128 bits)
     __shared__ Partial warp_part[32];
@@ -259,6 +260,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
         plan_s[tid] = plan_in.step[tid];
         qadj_s[tid] = plan_in.qadj[tid];
         uq_s[tid] = plan_in.uq[tid];
+        pdup_s[tid] = plan_in.pdup[tid];
     }
     if (tid < kMaxQV * kMaxQV) eidx_s[tid / kMaxQV][tid % kMaxQV] = plan_in.eidx[tid / kMaxQV][tid % kMaxQV];
     __syncthreads();
@@ -382,7 +384,9 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 if (MODE == kModeCount) sectors += 1.0;
             } else {
                 // GetMinCandidate (Alg. 1 l.8): the smallest N_l(M[j]) over j in B(d)
+                // (variant A3: WanderJoin takes the first backward position's list)
                 uint32_t bm = ps.back;
+                if (METHOD == GSWORD_WJ && plan_in.wj_parent_first) bm &= 0u - bm;
                 len_p = 0xFFFFFFFFu;
                 while (bm) {
                     const int j = __ffs(bm) - 1;
@@ -395,7 +399,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                         p = j;
                     }
                 }
-                if (MODE == kModeCount) sectors += (double)ps.nback;
+                if (MODE == kModeCount) sectors += (METHOD == GSWORD_WJ && plan_in.wj_parent_first) ? 1.0 : (double)ps.nback;
             }
         }
 
@@ -682,6 +686,9 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 rec->path[d] = (cnt > 0) ? v : -1;
             }
             bool dead = (cnt == 0) || reject;
+            // variant A5 (Fig. 19 AL Validate): DupCheck of the drawn vertex
+            if (METHOD == GSWORD_ALLEY && !dead && pdup_s[d] != 0u && !not_matched(Ms + tid, T, 0, pdup_s[d], v))
+                dead = true;
             bool complete = false;
             if (!dead) {
                 Ms[d * T + tid] = (uint32_t)v;
@@ -807,6 +814,7 @@ __global__ void __launch_bounds__(256) stream_kernel(const DeviceGraph g, const 
                                                      unsigned long long* __restrict__ /*phase_out*/) {
     __shared__ PlanStep plan_s[kMaxQV];
     __shared__ uint8_t eidx_s[kMaxQV][kMaxQV];
+    __shared__ uint32_t pdup_s[kMaxQV];
     __shared__ Partial warp_part[32];
     extern __shared__ uint32_t Ms[];  // Ms[j * blockDim.x + tid] = M[j] of this lane
 
@@ -815,7 +823,10 @@ __global__ void __launch_bounds__(256) stream_kernel(const DeviceGraph g, const 
     const int lane = tid & 31;
     const int wbase = tid - lane;
     const unsigned lt_mask = (1u << lane) - 1u;
-    if (tid < kMaxQV) plan_s[tid] = plan_in.step[tid];
+    if (tid < kMaxQV) {
+        plan_s[tid] = plan_in.step[tid];
+        pdup_s[tid] = plan_in.pdup[tid];
+    }
     if (tid < kMaxQV * kMaxQV) eidx_s[tid / kMaxQV][tid % kMaxQV] = plan_in.eidx[tid / kMaxQV][tid % kMaxQV];
     __syncthreads();
     const int nq = plan_in.nq;
@@ -974,7 +985,7 @@ __global__ void __launch_bounds__(256) stream_kernel(const DeviceGraph g, const 
                 rec->csize[d] = cnt;
                 rec->path[d] = (cnt > 0) ? v : -1;
             }
-            const bool dead = cnt == 0;
+            const bool dead = cnt == 0 || (pdup_s[d] != 0u && !not_matched(Ms + tid, T, 0, pdup_s[d], v));  // A5
             bool complete = false;
             if (!dead) {
                 Ms[d * T + tid] = (uint32_t)v;

@@ -32,6 +32,9 @@ struct Plan {
     uint32_t qadj[kMaxQV];  // bit j: (phi[j], phi[d]) is a query edge, any j != d
     uint8_t uq[kMaxQV];     // phi[d] (query vertex at depth d: row of cbits)
     uint8_t eidx[kMaxQV][kMaxQV];  // directed query edge (phi[j] -> phi[d]) index, j in B(d)
+    // comparison variants (GSWORD_OPT_VARIANT, readings A3/A5), applied per launch:
+    int32_t wj_parent_first;  // A3: WanderJoin draws from the first backward position's list
+    uint32_t pdup[kMaxQV];    // A5: Alley DupCheck after the draw (step[d].dup is then 0)
 };
 
 // Candidate filter of one query vertex (NEXT-1): label, degree, and the per-label
@@ -102,6 +105,19 @@ struct LaunchCfg {
     int sched;  // 0 refill, 1 sample synchronisation, 2 + inheritance (NEXT-3)
     uint32_t refill_min;  // sched 0: refill when at least this many lanes are free (1..32)
 };
+
+// Applies the GSWORD_OPT_VARIANT bits to a copy of the loaded plan (readings A3, A5).
+inline Plan plan_variant(const Plan& base, int method, int variant) {
+    Plan p = base;
+    p.wj_parent_first = (method == GSWORD_WJ && (variant & GSWORD_VARIANT_WJ_PARENT_FIRST)) ? 1 : 0;
+    for (int d = 0; d < kMaxQV; ++d) p.pdup[d] = 0u;
+    if (method == GSWORD_ALLEY && (variant & GSWORD_VARIANT_ALLEY_DUPCHECK_POST))
+        for (int d = 0; d < kMaxQV; ++d) {
+            p.pdup[d] = p.step[d].dup;
+            p.step[d].dup = 0u;
+        }
+    return p;
+}
 
 // Per-CTA partial aggregate (written by the sampling kernel, reduced in CTA order).
 struct Partial {

@@ -35,6 +35,9 @@ OPT_REFILL_MIN = 9
 OPT_AUTOTUNE = 10
 OPT_BLOOM_BITS = 11
 OPT_STREAMING = 12  # Alley by warp streaming (Alg. 3, reading A25)
+OPT_VARIANT = 13  # comparison variants of readings A3/A5 (bit flags below)
+VARIANT_WJ_PARENT_FIRST = 2
+VARIANT_ALLEY_DUPCHECK_POST = 4
 SCHED_REFILL, SCHED_SAMPLE_SYNC, SCHED_INHERIT = 0, 1, 2
 FILTER_LABEL, FILTER_LDF, FILTER_NLF = 0, 1, 2
 CUDA_STREAM_LEGACY = 0x1  # cudaStreamLegacy
