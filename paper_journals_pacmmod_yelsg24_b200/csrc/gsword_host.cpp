@@ -373,6 +373,7 @@ int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, u
         gsword_sample_record* d_records, double* d_sectors) {
     if (ctx->q_filter) mode |= gsword::kModeCG;
     if (method == GSWORD_ALLEY && ctx->opt_streaming && (mode & 3) != gsword::kModeCount) mode |= gsword::kModeStream;
+    if (ctx->opt_sched != 0) mode |= gsword::kModeSync;
     LaunchCfg cfg;
     int rc = launch_config(ctx, method, mode, &cfg);
     if (rc) return rc;

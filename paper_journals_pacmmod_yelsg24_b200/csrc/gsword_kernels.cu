@@ -112,6 +112,12 @@ __device__ __forceinline__ uint32_t fns32(uint32_t m, uint32_t k) {
     return pos;
 }
 
+// the same for masks of query positions (<= 16 bits, k usually 0-2): clear k low bits
+__device__ __forceinline__ int fns_small(uint32_t m, uint32_t k) {
+    while (k--) m &= m - 1;
+    return __ffs(m) - 1;
+}
+
 __device__ __forceinline__ uint32_t fns64(uint64_t m, uint32_t k) {
     const uint32_t lo = (uint32_t)m;
     const uint32_t c = __popc(lo);
@@ -215,6 +221,11 @@ __device__ __forceinline__ bool member_all(const DeviceGraph& g, const uint32_t*
     return true;
 }
 
+// One-word signature of a lane's matched vertices: bit sig_bit(v) is set for every M[j].
+// A clear bit proves x is not matched, so the exact scan of M is skipped (~80 % of the
+// DupChecks of an 8-vertex query).
+__device__ __forceinline__ uint32_t sig_bit(int32_t v) { return 1u << (((uint32_t)v * 0x9E3779B1u) >> 27); }
+
 __device__ __forceinline__ bool not_matched(const uint32_t* Ms, int stride, int col_of, uint32_t dup, int32_t x) {
     while (dup) {
         const int j = __ffs(dup) - 1;
@@ -224,6 +235,11 @@ __device__ __forceinline__ bool not_matched(const uint32_t* Ms, int stride, int 
     return true;
 }
 
+__device__ __forceinline__ bool not_matched_sig(const uint32_t* Ms, int stride, int col_of, uint32_t dup, uint32_t sig,
+                                                int32_t x) {
+    return !(sig & sig_bit(x)) || not_matched(Ms, stride, col_of, dup, x);
+}
+
 #ifndef GSWORD_WJ_MIN_BLOCKS
 #define GSWORD_WJ_MIN_BLOCKS 6  // 42 registers: 48 warps per SM (measured best)
 #endif
@@ -231,11 +247,13 @@ __device__ __forceinline__ bool not_matched(const uint32_t* Ms, int stride, int 
 #define GSWORD_AL_MIN_BLOCKS 5  // 51 registers: 40 warps per SM (measured best)
 #endif
 
-template <int METHOD, int MODE, bool CG>
+// SYNC: false = the default refill scheduler only (sched 0, the scheduling-mode logic
+// compiled out); true = any GSWORD_OPT_SCHEDULE (NEXT-3 comparison modes)
+template <int METHOD, int MODE, bool CG, bool SYNC>
 __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLOCKS : GSWORD_AL_MIN_BLOCKS)
     sample_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
                                                      const uint64_t count, const uint64_t seed, const int chunk,
-                                                     const uint32_t coop_threshold, const int sched,
+                                                     const uint32_t coop_threshold, const int sched_arg,
                                                      const uint32_t refill_min,
                                                      unsigned long long* __restrict__ queue,
                                                      Partial* __restrict__ partials,
@@ -266,9 +284,11 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
     __syncthreads();
 
     const int nq = plan_in.nq;
+    const int sched = SYNC ? sched_arg : 0;
 
     // lane state
     bool has = false;
+    uint32_t msig = 0u;  // signature of M[0..d-1] (sig_bit)
     uint64_t sid = 0;
     int d = 0;
     double W = 0.0;
@@ -342,6 +362,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 sid = first + q_next + rank;
                 d = 0;
                 W = 1.0;
+                msig = 0u;
                 if (MODE == kModeTrace) {
                     gsword_sample_record* rec = records + (sid - first);
                     rec->sample_id = sid;
@@ -419,7 +440,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                         if (MODE == kModeCount) sectors += 1.0;
                         // Validate: DupCheck, then IsEdge for the other matched neighbours.
                         // v in N_l(M[j]) <=> M[j] in N_{L(phi[j])}(v): search the shorter run.
-                        reject = !not_matched(Ms + tid, T, 0, ps.dup, v);
+                        reject = !not_matched_sig(Ms + tid, T, 0, ps.dup, msig, v);
                         uint32_t bm = ps.back & ~(1u << p);
                         while (bm && !reject) {
                             const int j = __ffs(bm) - 1;
@@ -497,7 +518,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 const int32_t olab = __shfl_sync(kFull, ps.label, o);
                 if (valid) {
                     const int ocol = wbase + o;
-                    const int j = (int)fns32(omask, k);
+                    const int j = fns_small(omask, k);
                     if (is_edge<MODE == kModeCount>(g, Ms[op * T + ocol], Ms[j * T + ocol], olab, sectors))
                         atomicOr(&res_s[ocol], 1u << j);
                 }
@@ -535,9 +556,13 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 if (valid) {
                     const int ocol = wbase + o;
                     // is S_p[i] (label l_d) in N_l(M[j]), i.e. is {M[j], S_p[i]} an edge?
-                    const uint32_t nth = k / olen;
-                    const uint32_t i = k - nth * olen;
-                    const int j = (int)fns32(omask, nth);
+                    // task k = (list nth, element i); one other list is the common case
+                    uint32_t nth = 0u, i = k;
+                    if (omask & (omask - 1u)) {
+                        nth = k / olen;
+                        i = k - nth * olen;
+                    }
+                    const int j = fns_small(omask, nth);
                     const int32_t x = ldg_i32(g.clist + olo + i);
                     if (!is_edge<MODE == kModeCount>(g, Ms[j * T + ocol], (uint32_t)x, olab, sectors))
                         atomicOr(&rm_s[i >> 5][ocol], 1u << (i & 31));
@@ -579,7 +604,8 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     while (mm) {
                         const int i = __ffs(mm) - 1;
                         mm &= mm - 1;
-                        if (!not_matched(Ms + tid, T, 0, dup, ldg_i32(g.clist + lo_p + 32u * w + i))) m &= ~(1u << i);
+                        if (!not_matched_sig(Ms + tid, T, 0, dup, msig, ldg_i32(g.clist + lo_p + 32u * w + i)))
+                            m &= ~(1u << i);
                     }
                     keep[w] = m;
                     cnt += __popc(m);
@@ -613,6 +639,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 const PlanStep Lps = plan_s[Ld];
                 const uint32_t others = Lps.back & ~(1u << Lp);
                 const int colL = wbase + L;
+                const uint32_t Lsig = __shfl_sync(kFull, msig, L);
                 uint32_t total = 0, my_bal = 0;
                 for (uint32_t base = 0; base < Llen; base += 32) {
                     const uint32_t i = base + lane;
@@ -621,7 +648,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                     if (keep) {
                         x = ldg_i32(g.clist + Llo + i);
                         keep = member_all<MODE == kModeCount>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
-                               not_matched(Ms, T, colL, Lps.dup, x);
+                               not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x);
                     }
                     const unsigned bal = __ballot_sync(kFull, keep);
                     if ((base >> 5) == (uint32_t)lane) my_bal = bal;
@@ -656,7 +683,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                             if (keep) {
                                 x = ldg_i32(g.clist + Llo + i);
                                 keep = member_all<MODE == kModeCount>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
-                                       not_matched(Ms, T, colL, Lps.dup, x);
+                                       not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x);
                             }
                             const unsigned bal = __ballot_sync(kFull, keep);
                             const uint32_t c = __popc(bal);
@@ -687,11 +714,13 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             }
             bool dead = (cnt == 0) || reject;
             // variant A5 (Fig. 19 AL Validate): DupCheck of the drawn vertex
-            if (METHOD == GSWORD_ALLEY && !dead && pdup_s[d] != 0u && !not_matched(Ms + tid, T, 0, pdup_s[d], v))
+            if (METHOD == GSWORD_ALLEY && !dead && pdup_s[d] != 0u &&
+                !not_matched_sig(Ms + tid, T, 0, pdup_s[d], msig, v))
                 dead = true;
             bool complete = false;
             if (!dead) {
                 Ms[d * T + tid] = (uint32_t)v;
+                msig |= sig_bit(v);
                 if (d + 1 == nq) complete = true;
             }
             if (dead || complete) {
@@ -724,10 +753,12 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 const int par = __ffs(alive_m) - 1;
                 const double Wn = __ddiv_rn(__shfl_sync(kFull, W, par), (double)(__popc(idle_m) + 1));
                 const int dp = __shfl_sync(kFull, d, par);
+                const uint32_t psig = __shfl_sync(kFull, msig, par);
                 __syncwarp();
                 if (lane == par) W = Wn;
                 if ((idle_m >> lane) & 1u) {
                     for (int j = 0; j < dp; ++j) Ms[j * T + tid] = Ms[j * T + wbase + par];
+                    msig = psig;
                     d = dp;
                     W = Wn;
                     has = true;
@@ -741,9 +772,9 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) gsum = __dadd_rn(gsum, shfl_xor_d(gsum, o));
         if (lane == 0) {
-            nsum(s_sum, c_sum, gsum);
-            nsum(s_sq, c_sq, __dmul_rn(gsum, gsum));
-        }
+                nsum(s_sum, c_sum, gsum);
+                nsum(s_sq, c_sq, __dmul_rn(gsum, gsum));
+            }
     }
 
     mark(7);
@@ -1519,8 +1550,9 @@ __global__ void scan_add_kernel(uint32_t* __restrict__ data, int64_t n, const ui
 }
 
 template <int METHOD, int MODE, bool CG>
-const void* kernel_ptr() {
-    return reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE, CG>);
+const void* kernel_ptr(bool sync) {
+    return sync ? reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE, CG, true>)
+                : reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE, CG, false>);
 }
 
 template <bool CG>
@@ -1529,14 +1561,16 @@ const void* select_kernel_cg(int method, int mode) {
         return (mode & 3) == kModeTrace ? reinterpret_cast<const void*>(&stream_kernel<kModeTrace, CG>)
                                         : reinterpret_cast<const void*>(&stream_kernel<kModeEstimate, CG>);
     }
+    const bool sync = (mode & kModeSync) != 0;
+    mode &= ~kModeSync;
     if (method == GSWORD_WJ) {
-        if (mode == kModeTrace) return kernel_ptr<GSWORD_WJ, kModeTrace, CG>();
-        if (mode == kModeCount) return kernel_ptr<GSWORD_WJ, kModeCount, CG>();
-        return kernel_ptr<GSWORD_WJ, kModeEstimate, CG>();
+        if (mode == kModeTrace) return kernel_ptr<GSWORD_WJ, kModeTrace, CG>(sync);
+        if (mode == kModeCount) return kernel_ptr<GSWORD_WJ, kModeCount, CG>(sync);
+        return kernel_ptr<GSWORD_WJ, kModeEstimate, CG>(sync);
     }
-    if (mode == kModeTrace) return kernel_ptr<GSWORD_ALLEY, kModeTrace, CG>();
-    if (mode == kModeCount) return kernel_ptr<GSWORD_ALLEY, kModeCount, CG>();
-    return kernel_ptr<GSWORD_ALLEY, kModeEstimate, CG>();
+    if (mode == kModeTrace) return kernel_ptr<GSWORD_ALLEY, kModeTrace, CG>(sync);
+    if (mode == kModeCount) return kernel_ptr<GSWORD_ALLEY, kModeCount, CG>(sync);
+    return kernel_ptr<GSWORD_ALLEY, kModeEstimate, CG>(sync);
 }
 
 // mode: kMode* | kModeCG when the query was loaded with a candidate filter
