@@ -1126,28 +1126,52 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
         // schedule autotune (no effect on any result): time pilot runs of each method with
         // refill thresholds 8/16/24/32 and keep the fastest (samples of long-lived walks
         // favour depth-synchronous warps, short-lived ones frequent refills)
-        static const int cand[4] = {8, 16, 24, 32};
+        // All pilots are queued back to back on the context stream and timed by events,
+        // with one host synchronisation for the whole tune (a warm-up launch per method
+        // first).
+        static const int cand[4] = {16, 8, 24, 32};
         const uint64_t pilot = 2000000;
-        for (int m = 0; m < 2; ++m) {
-            double best = 0.0;
-            int best_r = ctx->opt_refill_min;
-            for (int rep = 0; rep < 2; ++rep)
-                for (int c = 0; c < 4; ++c) {
-                    ctx->tuned_refill[m] = cand[c];
-                    gsword_result r;
-                    int rc2 = gsword_estimate_range(ctx, (gsword_method)m, 0, pilot, 0x5EEDull, &r);
-                    if (rc2) {
-                        ctx->tuned_refill[0] = ctx->tuned_refill[1] = 0;
-                        return rc2;
-                    }
-                    double t = 0.0;
-                    if (gsword_last_kernel_seconds(ctx, &t) != GSWORD_OK) t = r.seconds;
-                    if ((rep == 0 && c == 0) || t < best) {
-                        best = t;
-                        best_r = cand[c];
-                    }
+        cudaEvent_t ev[2][5];
+        int made = 0;
+        cudaError_t e = cudaSuccess;
+        for (; made < 10 && e == cudaSuccess; ++made) e = cudaEventCreate(&ev[made / 5][made % 5]);
+        auto destroy = [&]() {
+            for (int i = 0; i < made; ++i) cudaEventDestroy(ev[i / 5][i % 5]);
+        };
+        if (e != cudaSuccess) {
+            made -= 1;
+            destroy();
+            return cuda_fail(e, "autotune events");
+        }
+        int rc2 = GSWORD_OK;
+        for (int m = 0; m < 2 && rc2 == GSWORD_OK; ++m) {
+            ctx->tuned_refill[m] = cand[0];
+            rc2 = run(ctx, m, gsword::kModeEstimate, 0, pilot / 2, 0x5EEDull, ctx->d_out4, nullptr, nullptr);
+            for (int c = 0; c < 4 && rc2 == GSWORD_OK; ++c) {
+                ctx->tuned_refill[m] = cand[c];
+                if ((e = cudaEventRecord(ev[m][c], ctx->stream)) != cudaSuccess) break;
+                rc2 = run(ctx, m, gsword::kModeEstimate, 0, pilot, 0x5EEDull, ctx->d_out4, nullptr, nullptr);
+            }
+            if (rc2 == GSWORD_OK && e == cudaSuccess) e = cudaEventRecord(ev[m][4], ctx->stream);
+        }
+        if (rc2 == GSWORD_OK && e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+        for (int m = 0; m < 2 && rc2 == GSWORD_OK && e == cudaSuccess; ++m) {
+            float best = 0.f;
+            int best_r = cand[0];
+            for (int c = 0; c < 4 && e == cudaSuccess; ++c) {
+                float ms = 0.f;
+                e = cudaEventElapsedTime(&ms, ev[m][c], ev[m][c + 1]);
+                if (c == 0 || ms < best) {
+                    best = ms;
+                    best_r = cand[c];
                 }
+            }
             ctx->tuned_refill[m] = best_r;
+        }
+        destroy();
+        if (rc2 != GSWORD_OK || e != cudaSuccess) {
+            ctx->tuned_refill[0] = ctx->tuned_refill[1] = 0;
+            return rc2 != GSWORD_OK ? rc2 : cuda_fail(e, "autotune");
         }
     }
     return GSWORD_OK;

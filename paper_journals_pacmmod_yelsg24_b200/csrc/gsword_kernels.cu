@@ -641,12 +641,14 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 const int colL = wbase + L;
                 const uint32_t Lsig = __shfl_sync(kFull, msig, L);
                 uint32_t total = 0, my_bal = 0;
+                // the next chunk's driver elements are loaded while this chunk is tested
+                int32_t xn = ((uint32_t)lane < Llen) ? ldg_i32(g.clist + Llo + lane) : 0;
                 for (uint32_t base = 0; base < Llen; base += 32) {
                     const uint32_t i = base + lane;
                     bool keep = i < Llen;
-                    int32_t x = 0;
+                    const int32_t x = xn;
+                    if (i + 32u < Llen) xn = ldg_i32(g.clist + Llo + i + 32u);
                     if (keep) {
-                        x = ldg_i32(g.clist + Llo + i);
                         keep = member_all<MODE == kModeCount>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
                                not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x);
                     }
