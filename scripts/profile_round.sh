@@ -18,6 +18,7 @@ timeout 900 ncu --set full --import-source on --clock-control none -k regex:samp
     -o gpurun_out/${TAG}_full python scripts/profile_driver.py --samples 1e8 > gpurun_out/${TAG}_full.log 2>&1
 python scripts/ncu_summary.py gpurun_out/${TAG}_full.ncu-rep profiles/${TAG}_ncu_details.json 1e8 \
     > gpurun_out/${TAG}_summary.log 2>&1
+python scripts/launch_summary.py gpurun_out/${TAG}_launches.csv > gpurun_out/${TAG}_launches_summary.md 2>&1
 python scripts/ncu_lines.py gpurun_out/${TAG}_full.ncu-rep "" 30 > gpurun_out/${TAG}_ncu_lines.txt 2>&1
 cp profiles/${TAG}_ncu_details.json profiles/traffic_latest.json gpurun_out/ 2>/dev/null
 timeout 900 python bench.py > gpurun_out/${TAG}_bench.jsonl 2> gpurun_out/${TAG}_bench.err
