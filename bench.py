@@ -415,7 +415,9 @@ def run_ours(args):
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": 32 * len(methods), "graph_load_s": graph_load_s,
                 "note": "per step: gsword_load_query from host arrays + gsword_estimate per method "
-                        "(synchronous, host result); graph loaded once (P:L1057 excludes it)"},
+                        "(synchronous, host result); graph loaded once (P:L1057 excludes it); the "
+                        "refill-threshold autotune runs at the first load of the query and is cached "
+                        "per (query, options) afterwards"},
         "qerror": qerr,
         "gpu_launches": 2 * len(methods) * args.steps,
         "clocks": clocks.summary(),

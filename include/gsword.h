@@ -135,6 +135,9 @@ typedef struct {
     uint64_t cg_entries;
     double build_seconds;
     int32_t refill_min[2]; /* refill threshold in use per method (after autotune) */
+    int32_t occupancy[2];  /* resident CTAs per SM of the estimate kernel in use   */
+                           /* per method (after autotune; GSWORD_OPT_BLOCKS_PER_SM */
+                           /* may lower it further)                               */
 } gsword_query_stats;
 
 /* Tunables for gsword_set_option (defaults chosen by measurement). */
@@ -162,7 +165,13 @@ typedef enum {
                                    /* results                                         */
     GSWORD_OPT_AUTOTUNE = 10,      /* 1 (default): gsword_load_query times pilots of   */
                                    /* refill thresholds 8/16/24/32 per method and     */
-                                   /* keeps the fastest; results are unaffected       */
+                                   /* keeps the fastest, then times the estimate      */
+                                   /* kernel compiled for one CTA/SM less and one     */
+                                   /* more (register budget vs occupancy) at that     */
+                                   /* threshold; results are unaffected.              */
+                                   /* Results are cached per (query arrays, options)  */
+                                   /* until the next graph load: reloading the same   */
+                                   /* query runs no pilots                            */
     GSWORD_OPT_BLOOM_BITS = 11,    /* edge filter bits per undirected edge (2..64,    */
                                    /* default 16), applied at the next graph load     */
     GSWORD_OPT_STREAMING = 12,     /* 1 = Alley draws by warp streaming (Alg. 3,      */

@@ -12,6 +12,7 @@
 #include <cstdio>
 #include <cstring>
 #include <limits>
+#include <map>
 #include <string>
 #include <thread>
 #include <vector>
@@ -259,6 +260,13 @@ struct gsword_ctx {
     int opt_streaming = 0;        // Alley by warp streaming (Alg. 3, NEXT-3 comparison mode)
     int opt_variant = 0;          // GSWORD_VARIANT_* bits (readings A3/A5 comparison variants)
     int tuned_refill[2] = {0, 0}; // 0 = not tuned  // measured: 1.2-1.35x over refilling every round on C1, neutral on C2/C3
+    // autotune results per (query, options) since the last graph load: reloading a query
+    // (a serving loop re-issuing the same query) reuses them instead of re-running pilots
+    int tuned_occ[2] = {0, 0};    // occupancy variant of the estimate kernel (kModeOccShift)
+    struct Tuned {
+        int refill[2], occ[2];
+    };
+    std::map<std::string, Tuned> tune_cache;
     int opt_eset = 1;
     // last launch
     int last_grid = 0, last_threads = 0;
@@ -282,6 +290,7 @@ struct gsword_ctx {
         d_seg = nullptr;
         d_bucket = nullptr;
         graph_loaded = false;
+        tune_cache.clear();
         query_loaded = false;
     }
 };
@@ -374,6 +383,8 @@ int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, u
     if (ctx->q_filter) mode |= gsword::kModeCG;
     if (method == GSWORD_ALLEY && ctx->opt_streaming && (mode & 3) != gsword::kModeCount) mode |= gsword::kModeStream;
     if (ctx->opt_sched != 0) mode |= gsword::kModeSync;
+    if ((mode & (3 | gsword::kModeSync | gsword::kModeStream)) == gsword::kModeEstimate && ctx->opt_autotune)
+        mode |= ctx->tuned_occ[method & 1] << gsword::kModeOccShift;
     LaunchCfg cfg;
     int rc = launch_config(ctx, method, mode, &cfg);
     if (rc) return rc;
@@ -1122,57 +1133,91 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
     ctx->plan = p;
     ctx->query_loaded = true;
     ctx->tuned_refill[0] = ctx->tuned_refill[1] = 0;
+    ctx->tuned_occ[0] = ctx->tuned_occ[1] = 0;
+    std::string tkey;
     if (ctx->opt_autotune && ctx->opt_sched == 0) {
-        // schedule autotune (no effect on any result): time pilot runs of each method with
-        // refill thresholds 8/16/24/32 and keep the fastest (samples of long-lived walks
-        // favour depth-synchronous warps, short-lived ones frequent refills)
-        // All pilots are queued back to back on the context stream and timed by events,
-        // with one host synchronisation for the whole tune (a warm-up launch per method
-        // first).
+        // the query exactly as given plus every option that changes the kernels' schedule
+        const int opts[] = {n_qv, ctx->opt_blocks_per_sm, ctx->opt_threads, ctx->opt_chunk, ctx->opt_l2,
+                            ctx->opt_coop, ctx->opt_bloom, ctx->opt_eset, ctx->opt_filter, ctx->opt_streaming,
+                            ctx->opt_variant};
+        tkey.append(reinterpret_cast<const char*>(opts), sizeof(opts));
+        tkey.append(reinterpret_cast<const char*>(q_row_ptr), sizeof(int32_t) * (size_t)(n_qv + 1));
+        tkey.append(reinterpret_cast<const char*>(q_col), sizeof(int32_t) * (size_t)q_row_ptr[n_qv]);
+        tkey.append(reinterpret_cast<const char*>(q_labels), sizeof(int32_t) * (size_t)n_qv);
+        tkey.append(reinterpret_cast<const char*>(order), sizeof(int32_t) * (size_t)n_qv);
+        const auto it = ctx->tune_cache.find(tkey);
+        if (it != ctx->tune_cache.end()) {
+            for (int m = 0; m < 2; ++m) {
+                ctx->tuned_refill[m] = it->second.refill[m];
+                ctx->tuned_occ[m] = it->second.occ[m];
+            }
+        }
+    }
+    if (ctx->opt_autotune && ctx->opt_sched == 0 && ctx->tuned_refill[0] == 0) {
+        // schedule autotune (no effect on any result).  Phase 1: refill thresholds
+        // 16/8/24/32 (samples of long-lived walks favour depth-synchronous warps, short-lived
+        // ones frequent refills).  Phase 2, at the chosen threshold: the
+        // estimate kernel compiled for one CTA/SM less (more registers, fewer spills) and one
+        // more.  Every candidate is timed over the same id range of `big` samples, preceded
+        // by a warm-up over a range of its own (short or repeated pilots favour whichever
+        // candidate profits from the tail or from a warm L2); each phase queues its runs back
+        // to back on the context stream, timed by events, with one host synchronisation.
         static const int cand[4] = {16, 8, 24, 32};
-        const uint64_t pilot = 2000000;
-        cudaEvent_t ev[2][5];
-        int made = 0;
-        cudaError_t e = cudaSuccess;
-        for (; made < 10 && e == cudaSuccess; ++made) e = cudaEventCreate(&ev[made / 5][made % 5]);
-        auto destroy = [&]() {
-            for (int i = 0; i < made; ++i) cudaEventDestroy(ev[i / 5][i % 5]);
-        };
-        if (e != cudaSuccess) {
-            made -= 1;
-            destroy();
-            return cuda_fail(e, "autotune events");
-        }
+        const uint64_t big = 8000000, warm = 1000000, range0 = 1ull << 40;
         int rc2 = GSWORD_OK;
-        for (int m = 0; m < 2 && rc2 == GSWORD_OK; ++m) {
-            ctx->tuned_refill[m] = cand[0];
-            rc2 = run(ctx, m, gsword::kModeEstimate, 0, pilot / 2, 0x5EEDull, ctx->d_out4, nullptr, nullptr);
-            for (int c = 0; c < 4 && rc2 == GSWORD_OK; ++c) {
-                ctx->tuned_refill[m] = cand[c];
-                if ((e = cudaEventRecord(ev[m][c], ctx->stream)) != cudaSuccess) break;
-                rc2 = run(ctx, m, gsword::kModeEstimate, 0, pilot, 0x5EEDull, ctx->d_out4, nullptr, nullptr);
-            }
-            if (rc2 == GSWORD_OK && e == cudaSuccess) e = cudaEventRecord(ev[m][4], ctx->stream);
-        }
-        if (rc2 == GSWORD_OK && e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
-        for (int m = 0; m < 2 && rc2 == GSWORD_OK && e == cudaSuccess; ++m) {
-            float best = 0.f;
-            int best_r = cand[0];
-            for (int c = 0; c < 4 && e == cudaSuccess; ++c) {
-                float ms = 0.f;
-                e = cudaEventElapsedTime(&ms, ev[m][c], ev[m][c + 1]);
-                if (c == 0 || ms < best) {
-                    best = ms;
-                    best_r = cand[c];
+        cudaError_t e = cudaSuccess;
+        std::vector<cudaEvent_t> evs;
+        auto event = [&](cudaEvent_t* out) {
+            if (e == cudaSuccess) e = cudaEventCreate(out);
+            if (e == cudaSuccess) evs.push_back(*out);
+        };
+        // times[m][c] for candidate c of method m; sets tuned_* before each run
+        auto time_phase = [&](int ncand, auto&& apply, float (*times)[4]) {
+            cudaEvent_t ev[2][4][2];
+            for (int m = 0; m < 2 && rc2 == GSWORD_OK && e == cudaSuccess; ++m)
+                for (int c = 0; c < ncand && rc2 == GSWORD_OK && e == cudaSuccess; ++c) {
+                    apply(m, c);
+                    rc2 = run(ctx, m, gsword::kModeEstimate, range0 + big + warm * (uint64_t)(4 * m + c), warm,
+                              0x5EEDull, ctx->d_out4, nullptr, nullptr);
+                    event(&ev[m][c][0]);
+                    event(&ev[m][c][1]);
+                    if (rc2 == GSWORD_OK && e == cudaSuccess) e = cudaEventRecord(ev[m][c][0], ctx->stream);
+                    if (rc2 == GSWORD_OK && e == cudaSuccess)
+                        rc2 = run(ctx, m, gsword::kModeEstimate, range0, big, 0x5EEDull, ctx->d_out4, nullptr, nullptr);
+                    if (rc2 == GSWORD_OK && e == cudaSuccess) e = cudaEventRecord(ev[m][c][1], ctx->stream);
                 }
-            }
-            ctx->tuned_refill[m] = best_r;
+            if (rc2 == GSWORD_OK && e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+            for (int m = 0; m < 2 && rc2 == GSWORD_OK && e == cudaSuccess; ++m)
+                for (int c = 0; c < ncand && e == cudaSuccess; ++c)
+                    e = cudaEventElapsedTime(&times[m][c], ev[m][c][0], ev[m][c][1]);
+        };
+        float t1[2][4] = {}, t2[2][4] = {};
+        time_phase(4, [&](int m, int c) { ctx->tuned_refill[m] = cand[c]; }, t1);
+        float best[2] = {0.f, 0.f};
+        for (int m = 0; m < 2; ++m) {
+            int bc = 0;
+            for (int c = 1; c < 4; ++c)
+                if (t1[m][c] < t1[m][bc]) bc = c;
+            ctx->tuned_refill[m] = cand[bc];
+            best[m] = t1[m][bc];
         }
-        destroy();
+        time_phase(2, [&](int m, int c) { ctx->tuned_occ[m] = 1 + c; }, t2);
+        for (int m = 0; m < 2; ++m) {
+            ctx->tuned_occ[m] = 0;
+            for (int c = 0; c < 2; ++c)
+                if (t2[m][c] < 0.97f * best[m]) {  // a variant must win by 3 % (pilot noise)
+                    best[m] = t2[m][c];
+                    ctx->tuned_occ[m] = 1 + c;
+                }
+        }
+        for (cudaEvent_t x : evs) cudaEventDestroy(x);
         if (rc2 != GSWORD_OK || e != cudaSuccess) {
             ctx->tuned_refill[0] = ctx->tuned_refill[1] = 0;
+            ctx->tuned_occ[0] = ctx->tuned_occ[1] = 0;
             return rc2 != GSWORD_OK ? rc2 : cuda_fail(e, "autotune");
         }
+        if (ctx->tune_cache.size() >= 4096) ctx->tune_cache.clear();
+        ctx->tune_cache[tkey] = {{ctx->tuned_refill[0], ctx->tuned_refill[1]}, {ctx->tuned_occ[0], ctx->tuned_occ[1]}};
     }
     return GSWORD_OK;
 }
@@ -1188,6 +1233,15 @@ int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out) {
     out->build_seconds = ctx->cg_seconds;
     out->refill_min[0] = ctx->tuned_refill[0] ? ctx->tuned_refill[0] : ctx->opt_refill_min;
     out->refill_min[1] = ctx->tuned_refill[1] ? ctx->tuned_refill[1] : ctx->opt_refill_min;
+    for (int m = 0; m < 2; ++m) {
+        int mode = gsword::kModeEstimate | (ctx->q_filter ? gsword::kModeCG : 0);
+        if (ctx->opt_autotune && ctx->opt_sched == 0 && !(m == GSWORD_ALLEY && ctx->opt_streaming))
+            mode |= ctx->tuned_occ[m] << gsword::kModeOccShift;
+        if (m == GSWORD_ALLEY && ctx->opt_streaming) mode |= gsword::kModeStream;
+        if (ctx->opt_sched != 0) mode |= gsword::kModeSync;
+        const int occ = gsword::max_blocks_per_sm(m, mode, ctx->opt_threads, nullptr);
+        out->occupancy[m] = ctx->opt_blocks_per_sm > 0 ? std::min(ctx->opt_blocks_per_sm, occ) : occ;
+    }
     return GSWORD_OK;
 }
 

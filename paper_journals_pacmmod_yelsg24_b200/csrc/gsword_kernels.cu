@@ -18,6 +18,7 @@
 // The graph is read through the read-only path; candidate order is ascending vertex
 // id everywhere, so results are bit-identical to the CPU oracle.
 #include <cstdint>
+#include <type_traits>
 
 #include "internal.h"
 
@@ -25,6 +26,13 @@ namespace gsword {
 namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
+
+#ifndef GSWORD_SELECT_WINDOW
+#define GSWORD_SELECT_WINDOW 1  // Alley single-list select: window load + register fixed point
+#endif
+#ifndef GSWORD_POOL_DEFER
+#define GSWORD_POOL_DEFER 0  // 1: Alley task pool batches exact edge probes 32 at a time (measured 4-10 % slower)
+#endif
 // Alley drivers longer than the coop threshold (<= 64) are refined by the whole warp.
 
 // ---------------------------------------------------------------- Philox4x32-10 (A6)
@@ -209,6 +217,38 @@ __device__ __forceinline__ bool is_edge(const DeviceGraph& g, uint32_t a, uint32
     return in_run(g.col, lo, hi, (int32_t)b);
 }
 
+// The two halves of is_edge for callers that batch the exact step (the Alley task pool):
+// bloom_maybe = the filter's verdict (false is final), edge_exact = the edge-set probe
+// (or the binary search when the edge set is off).
+template <bool COUNT>
+__device__ __forceinline__ bool bloom_maybe(const DeviceGraph& g, uint32_t a, uint32_t b, double& sec) {
+    if (!g.bloom) return true;
+    if (COUNT) sec += 1.0;
+    const uint64_t h = edge_hash(a, b);
+    const uint64_t m = bloom_bits(h);
+    return (__ldg(g.bloom + (h & g.bloom_mask)) & m) == m;
+}
+
+template <bool COUNT>
+__device__ __forceinline__ bool edge_exact(const DeviceGraph& g, uint32_t a, uint32_t b, int32_t lb, double& sec) {
+    if (g.eset) {
+        const unsigned long long key = edge_key(a, b);
+        uint64_t bk = edge_hash(a, b) & g.eset_mask;
+        while (true) {
+            if (COUNT) sec += 1.0;
+            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(g.eset + 4 * bk);
+            const ulonglong2 x0 = __ldg(p), x1 = __ldg(p + 1);
+            if (x0.x == key || x0.y == key || x1.x == key || x1.y == key) return true;
+            if (x0.x == kEmptyKey || x0.y == kEmptyKey || x1.x == kEmptyKey || x1.y == kEmptyKey) return false;
+            bk = (bk + 1) & g.eset_mask;
+        }
+    }
+    uint32_t lo, hi;
+    segment(g, a, lb, &lo, &hi);
+    if (COUNT) sec += 1.0 + (double)bs_sectors(hi - lo);
+    return in_run(g.col, lo, hi, (int32_t)b);
+}
+
 // Is x in every N_l(M[j]) for j in `mask`?  M column `col_of` in shared memory.
 template <bool COUNT>
 __device__ __forceinline__ bool member_all(const DeviceGraph& g, const uint32_t* Ms, int stride, int col_of,
@@ -247,10 +287,17 @@ __device__ __forceinline__ bool not_matched_sig(const uint32_t* Ms, int stride, 
 #define GSWORD_AL_MIN_BLOCKS 5  // 51 registers: 40 warps per SM (measured best)
 #endif
 
+// Launch bounds per occupancy variant: 0 = the measured default, 1 = one CTA/SM less
+// (more registers, fewer spills: better where samples die early, e.g. C3 Alley), 2 = one
+// more.  The autotune in gsword_load_query picks per method and query.
+__host__ __device__ constexpr int kOccBlocks(int method, int occ) {
+    return (method == GSWORD_WJ ? GSWORD_WJ_MIN_BLOCKS : GSWORD_AL_MIN_BLOCKS) + (occ == 1 ? -1 : occ == 2 ? 1 : 0);
+}
+
 // SYNC: false = the default refill scheduler only (sched 0, the scheduling-mode logic
 // compiled out); true = any GSWORD_OPT_SCHEDULE (NEXT-3 comparison modes)
-template <int METHOD, int MODE, bool CG, bool SYNC>
-__global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLOCKS : GSWORD_AL_MIN_BLOCKS)
+template <int METHOD, int MODE, bool CG, bool SYNC, int OCC = 0>
+__global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     sample_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
                                                      const uint64_t count, const uint64_t seed, const int chunk,
                                                      const uint32_t coop_threshold, const int sched_arg,
@@ -264,8 +311,13 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
     __shared__ uint8_t eidx_s[kMaxQV][kMaxQV];
     __shared__ uint8_t uq_s[kMaxQV];
     __shared__ uint32_t pdup_s[kMaxQV];  // variant A5: post-draw DupCheck positions
-    __shared__ uint32_t res_s[256];   // Alley task-pool results per lane (adjacent matched vertices)
-    __shared__ uint32_t rm_s[4][256];  // Alley task-pool results per lane: refine-mask removals (128 bits)
+    // Alley task-pool results per lane: pool_s[0] = adjacent matched vertices (pool 1),
+    // pool_s[1..4] = refine-mask removals (pool 2, 128 bits)
+    __shared__ uint32_t pool_s[5][256];
+#if GSWORD_POOL_DEFER
+    // per-warp ring of edge tests the filter could not settle: (a, b, target, label)
+    __shared__ uint32_t dq_s[8][4][64];
+#endif
     __shared__ Partial warp_part[32];
     extern __shared__ uint32_t Ms[];  // Ms[j * blockDim.x + tid] = M[j] of this lane
 
@@ -461,7 +513,14 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             // exclusive scan of per-lane counts, owner found by shuffle bisection), so every
             // lane is busy whichever lanes generated the work (the refine imbalance).
             // test(o, k) runs task k of owner lane o; every lane calls it (it shuffles).
-            auto pool = [&](uint32_t ntask, auto&& test) {
+            // test(o, k, valid, a, b, tgt, lb) names the edge {a, b} of task k of owner lane o
+            // (label lb = L(b)) and the result bit tgt = (word << 5) | bit in pool_s; the bit
+            // is set when the edge's presence equals SET_ON_EDGE.  Every lane calls it (it
+            // shuffles).  GSWORD_POOL_DEFER: a "maybe" of the filter is queued and the exact
+            // probes run 32 at a time, so the filter loads of successive rounds are not
+            // serialised behind divergent edge-set probes.
+            auto pool = [&](uint32_t ntask, auto set_on_edge, auto&& test) {
+                constexpr bool SET_ON_EDGE = decltype(set_on_edge)::value;
                 if (!__any_sync(kFull, ntask != 0u)) return;
                 uint32_t incl = ntask;
 #pragma unroll
@@ -471,6 +530,22 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 }
                 const uint32_t total = __shfl_sync(kFull, incl, 31);
                 const uint32_t excl = incl - ntask;
+#if GSWORD_POOL_DEFER
+                uint32_t(*dq)[64] = dq_s[tid >> 5];
+                uint32_t qh = 0, qn = 0;  // ring head and length (warp-uniform)
+                auto flush = [&](uint32_t n) {
+                    __syncwarp();
+                    if ((uint32_t)lane < n) {
+                        const uint32_t e = (qh + lane) & 63u;
+                        const uint32_t tg = dq[2][e];
+                        const bool is = edge_exact<MODE == kModeCount>(g, dq[0][e], dq[1][e], (int32_t)dq[3][e], sectors);
+                        if (is == SET_ON_EDGE) atomicOr(&pool_s[0][0] + (tg >> 5), 1u << (tg & 31u));
+                    }
+                    __syncwarp();
+                    qh = (qh + n) & 63u;
+                    qn -= n;
+                };
+#endif
                 for (uint32_t base = 0; base < total; base += 32) {
                     const uint32_t t = base + (uint32_t)lane;
                     const uint32_t tt = t < total ? t : total - 1;
@@ -480,15 +555,37 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                         const uint32_t y = __shfl_sync(kFull, incl, o + s2 - 1);
                         if (y <= tt) o += s2;
                     }
-                    test(o, tt - __shfl_sync(kFull, excl, o), t < total);
+                    uint32_t ea = 0, eb = 0, tg = 0;
+                    int32_t lb = 0;
+                    const bool valid = t < total;
+                    test(o, tt - __shfl_sync(kFull, excl, o), valid, ea, eb, tg, lb);
+#if GSWORD_POOL_DEFER
+                    const bool maybe = valid && bloom_maybe<MODE == kModeCount>(g, ea, eb, sectors);
+                    if (valid && !maybe && !SET_ON_EDGE) atomicOr(&pool_s[0][0] + (tg >> 5), 1u << (tg & 31u));
+                    const unsigned mb = __ballot_sync(kFull, maybe);
+                    if (maybe) {
+                        const uint32_t e = (qh + qn + __popc(mb & lt_mask)) & 63u;
+                        dq[0][e] = ea;
+                        dq[1][e] = eb;
+                        dq[2][e] = tg;
+                        dq[3][e] = (uint32_t)lb;
+                    }
+                    qn += __popc(mb);
+                    if (qn >= 32u) flush(32u);
+#else
+                    if (valid && is_edge<MODE == kModeCount>(g, ea, eb, lb, sectors) == SET_ON_EDGE)
+                        atomicOr(&pool_s[0][0] + (tg >> 5), 1u << (tg & 31u));
+#endif
                 }
+#if GSWORD_POOL_DEFER
+                if (qn) flush(qn);
+#endif
                 __syncwarp();
             };
             int kind = 0;
             uint32_t unk = 0, known = 0, others = 0;
-            res_s[tid] = 0u;
 #pragma unroll
-            for (int w = 0; w < 4; ++w) rm_s[w][tid] = 0u;
+            for (int w = 0; w < 5; ++w) pool_s[w][tid] = 0u;
             if (has && deferred) {
                 // M[j] (same label) with (phi[j], phi[p]) a query edge lies in S_p by the
                 // Alley invariant (every drawn prefix is a partial instance); M[p] never does
@@ -512,15 +609,18 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             }
             __syncwarp();
             // pool 1: exclusion tests, overlapping the in-flight segment loads
-            pool((kind == 1) ? (uint32_t)__popc(unk) : 0u, [&](int o, uint32_t k, bool valid) {
+            pool((kind == 1) ? (uint32_t)__popc(unk) : 0u, std::true_type{},
+                 [&](int o, uint32_t k, bool valid, uint32_t& ea, uint32_t& eb, uint32_t& tg, int32_t& lb) {
                 const uint32_t omask = __shfl_sync(kFull, unk, o);
                 const int op = __shfl_sync(kFull, p, o);
                 const int32_t olab = __shfl_sync(kFull, ps.label, o);
                 if (valid) {
                     const int ocol = wbase + o;
                     const int j = fns_small(omask, k);
-                    if (is_edge<MODE == kModeCount>(g, Ms[op * T + ocol], Ms[j * T + ocol], olab, sectors))
-                        atomicOr(&res_s[ocol], 1u << j);
+                    ea = Ms[op * T + ocol];
+                    eb = Ms[j * T + ocol];
+                    lb = olab;
+                    tg = ((uint32_t)ocol << 5) | (uint32_t)j;  // pool_s[0][ocol], bit j
                 }
             });
             if (deferred) {
@@ -548,7 +648,8 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
             }
             mark(3);
             // pool 2: membership tests of short refine masks
-            pool((kind == 2) ? len_p * (uint32_t)__popc(others) : 0u, [&](int o, uint32_t k, bool valid) {
+            pool((kind == 2) ? len_p * (uint32_t)__popc(others) : 0u, std::false_type{},
+                 [&](int o, uint32_t k, bool valid, uint32_t& ea, uint32_t& eb, uint32_t& tg, int32_t& lb) {
                 const uint32_t omask = __shfl_sync(kFull, others, o);
                 const uint32_t olo = __shfl_sync(kFull, lo_p, o);
                 const uint32_t olen = __shfl_sync(kFull, len_p, o);
@@ -563,20 +664,41 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                         i = k - nth * olen;
                     }
                     const int j = fns_small(omask, nth);
-                    const int32_t x = ldg_i32(g.clist + olo + i);
-                    if (!is_edge<MODE == kModeCount>(g, Ms[j * T + ocol], (uint32_t)x, olab, sectors))
-                        atomicOr(&rm_s[i >> 5][ocol], 1u << (i & 31));
+                    ea = Ms[j * T + ocol];
+                    eb = (uint32_t)ldg_i32(g.clist + olo + i);
+                    lb = olab;
+                    tg = ((uint32_t)((1u + (i >> 5)) * 256u + (uint32_t)ocol) << 5) | (i & 31u);  // pool_s[1 + i/32][ocol]
                 }
             });
             mark(4);
             if (kind == 1) {
-                const uint32_t in_sp = known | res_s[tid];  // matched vertices inside S_p
+                const uint32_t in_sp = known | pool_s[0][tid];  // matched vertices inside S_p
                 cnt = len_p - __popc(in_sp);
                 if (cnt > 0) {
                     const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
                     // smallest idx with idx = k + #{x in X : x <= S_p[idx]}: the k-th survivor
-                    uint32_t idx = k;
-                    while (true) {
+                    const int nx = __popc(in_sp);
+#if GSWORD_SELECT_WINDOW
+                    if (nx <= 2) {
+                        // idx lies in [k, k + nx] (inside S_p since cnt = len_p - nx > k): load
+                        // that window at once and find the fixed point in registers (one
+                        // memory round trip instead of up to nx + 1 dependent ones)
+                        const int32_t* wb = g.clist + lo_p + k;
+                        const int32_t w0 = ldg_i32(wb);
+                        const int32_t w1 = nx >= 1 ? ldg_i32(wb + 1) : 0;
+                        const int32_t w2 = nx >= 2 ? ldg_i32(wb + 2) : 0;
+                        const int32_t x0 = nx >= 1 ? (int32_t)Ms[(__ffs(in_sp) - 1) * T + tid] : INT32_MAX;
+                        const int32_t x1 = nx >= 2 ? (int32_t)Ms[(31 - __clz(in_sp)) * T + tid] : INT32_MAX;
+                        uint32_t i = 0;
+#pragma unroll
+                        for (int it = 0; it < 2; ++it) {
+                            const int32_t wi = i == 0 ? w0 : (i == 1 ? w1 : w2);
+                            i = (uint32_t)(x0 <= wi) + (uint32_t)(x1 <= wi);
+                        }
+                        v = i == 0 ? w0 : (i == 1 ? w1 : w2);
+                    } else
+#endif
+                    for (uint32_t idx = k;;) {
                         v = ldg_i32(g.clist + lo_p + idx);
                         uint32_t c = 0, xm = in_sp;
                         while (xm) {
@@ -599,7 +721,7 @@ __global__ void __launch_bounds__(256, (METHOD == GSWORD_WJ) ? GSWORD_WJ_MIN_BLO
                 for (int w = 0; w < 4; ++w) {
                     const uint32_t n_w = (len_p > 32u * w) ? min(len_p - 32u * w, 32u) : 0u;
                     uint32_t m = (n_w == 32u) ? 0xFFFFFFFFu : ((1u << n_w) - 1u);
-                    m &= ~rm_s[w][tid];
+                    m &= ~pool_s[1 + w][tid];
                     uint32_t mm = dup ? m : 0u;
                     while (mm) {
                         const int i = __ffs(mm) - 1;
@@ -1552,7 +1674,11 @@ __global__ void scan_add_kernel(uint32_t* __restrict__ data, int64_t n, const ui
 }
 
 template <int METHOD, int MODE, bool CG>
-const void* kernel_ptr(bool sync) {
+const void* kernel_ptr(bool sync, int occ = 0) {
+    if (MODE == kModeEstimate && !sync && occ == 1)
+        return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 1>);
+    if (MODE == kModeEstimate && !sync && occ == 2)
+        return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 2>);
     return sync ? reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE, CG, true>)
                 : reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE, CG, false>);
 }
@@ -1564,15 +1690,16 @@ const void* select_kernel_cg(int method, int mode) {
                                         : reinterpret_cast<const void*>(&stream_kernel<kModeEstimate, CG>);
     }
     const bool sync = (mode & kModeSync) != 0;
-    mode &= ~kModeSync;
+    const int occ = (mode >> kModeOccShift) & 3;
+    mode &= 3;
     if (method == GSWORD_WJ) {
         if (mode == kModeTrace) return kernel_ptr<GSWORD_WJ, kModeTrace, CG>(sync);
         if (mode == kModeCount) return kernel_ptr<GSWORD_WJ, kModeCount, CG>(sync);
-        return kernel_ptr<GSWORD_WJ, kModeEstimate, CG>(sync);
+        return kernel_ptr<GSWORD_WJ, kModeEstimate, CG>(sync, occ);
     }
     if (mode == kModeTrace) return kernel_ptr<GSWORD_ALLEY, kModeTrace, CG>(sync);
     if (mode == kModeCount) return kernel_ptr<GSWORD_ALLEY, kModeCount, CG>(sync);
-    return kernel_ptr<GSWORD_ALLEY, kModeEstimate, CG>(sync);
+    return kernel_ptr<GSWORD_ALLEY, kModeEstimate, CG>(sync, occ);
 }
 
 // mode: kMode* | kModeCG when the query was loaded with a candidate filter
@@ -1582,6 +1709,8 @@ const void* select_kernel(int method, int mode) {
 }
 
 }  // namespace
+
+int occ_blocks(int method, int occ_variant) { return kOccBlocks(method, occ_variant); }
 
 int max_blocks_per_sm(int method, int mode, int threads, size_t* smem_bytes) {
     const size_t smem = (size_t)kMaxQV * (size_t)threads * sizeof(uint32_t);

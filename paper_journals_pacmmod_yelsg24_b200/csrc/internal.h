@@ -194,6 +194,8 @@ cudaError_t launch_build_eset(const int64_t* d_row_ptr, const int32_t* col, int6
 cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* bloom,
                                uint64_t mask, cudaStream_t stream);
 int max_blocks_per_sm(int method, int mode, int threads, size_t* smem_bytes);
+// minimum resident CTAs per SM the sampling kernel is compiled for (launch bounds)
+int occ_blocks(int method, int occ_variant);
 
 enum Mode {
     kModeEstimate = 0,
@@ -201,7 +203,9 @@ enum Mode {
     kModeCount = 2,
     kModeCG = 4,     // flag: candidate graph
     kModeStream = 8,  // flag: Alley by warp streaming (Alg. 3, NEXT-3)
-    kModeSync = 16    // flag: a scheduling mode other than refill (GSWORD_OPT_SCHEDULE != 0)
+    kModeSync = 16,   // flag: a scheduling mode other than refill (GSWORD_OPT_SCHEDULE != 0)
+    kModeOccShift = 5  // bits 5-6: occupancy variant of the estimate kernel (0 default, 1 one
+                       // CTA/SM less, 2 one more; refill schedule only), see occ_blocks()
 };
 
 }  // namespace gsword

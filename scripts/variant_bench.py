@@ -35,7 +35,7 @@ with G.Context(0) as ctx:
                 ts.append(ctx.last_kernel_seconds())
             print(json.dumps({"lib": os.path.basename(G.gsword.LIB_PATH), "config": cfg, "query": int(qi), "method": m,
                               "kernel_ms": 1e3 * min(ts), "samples_per_s": N / min(ts), "est": r["estimate"],
-                              "valid": r["n_valid"]}), flush=True)
+                              "valid": r["n_valid"], "tuned": ctx.query_info()}), flush=True)
 """ % HERE
 
 for lib in sys.argv[1:]:

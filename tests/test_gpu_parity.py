@@ -519,8 +519,27 @@ def test_autotune_does_not_change_results(ctx, G, c0):
     ctx.load_query_obj(q)
     info = ctx.query_info()
     assert all(r in (8, 16, 24, 32) for r in info["refill_min"])
+    assert info["occupancy"][0] in (5, 6, 7) and info["occupancy"][1] in (4, 5, 6)
     for m in (0, 1):
         assert ctx.trace_samples(m, 0, 30_000, 4).tobytes() == ref[m].tobytes()
+    # reloading the same query reuses the tuned thresholds (no pilots); a graph reload
+    # forgets them
+    ctx.load_query_obj(q)
+    assert ctx.query_info()["refill_min"] == info["refill_min"]
+    assert ctx.query_info()["occupancy"] == info["occupancy"]
+    # every occupancy variant of the estimate kernel gives the same aggregate
+    for m in (0, 1):
+        ref_agg = ctx.estimate(m, 50_000, 9)
+        for bps in (3, 4):
+            ctx.set_option(G.OPT_BLOCKS_PER_SM, bps)
+            try:
+                agg = ctx.estimate(m, 50_000, 9)
+            finally:
+                ctx.set_option(G.OPT_BLOCKS_PER_SM, 0)
+            assert agg["n_valid"] == ref_agg["n_valid"] and agg["sum"] == pytest.approx(ref_agg["sum"], rel=REL)
+    ctx.load_graph_obj(g)
+    ctx.load_query_obj(q)
+    assert all(r in (8, 16, 24, 32) for r in ctx.query_info()["refill_min"])
 
 
 def test_estimate_until(ctx, G, c0):
