@@ -30,6 +30,9 @@ constexpr unsigned kFull = 0xffffffffu;
 #ifndef GSWORD_SELECT_WINDOW
 #define GSWORD_SELECT_WINDOW 1  // Alley single-list select: window load + register fixed point
 #endif
+#ifndef GSWORD_COOP_WIDE
+#define GSWORD_COOP_WIDE 0  // 1: occupancy variant 1 runs two coop chunks per round (measured 0-7 % slower: spills)
+#endif
 #ifndef GSWORD_POOL_DEFER
 #define GSWORD_POOL_DEFER 0  // 1: Alley task pool batches exact edge probes 32 at a time (measured 4-10 % slower)
 #endif
@@ -259,6 +262,54 @@ __device__ __forceinline__ bool member_all(const DeviceGraph& g, const uint32_t*
         if (!is_edge<COUNT>(g, Ms[j * stride + col_of], (uint32_t)x, l, sec)) return false;
     }
     return true;
+}
+
+// Two membership tests at once (x0, x1 each in every N_l(M[j]), j in `mask`): the filter
+// words of both, then the first edge-set buckets of both, are loaded before either is
+// used, so the two tests cost one dependent chain.  k0/k1 enter as "still a candidate".
+__device__ __forceinline__ bool eset_first(const DeviceGraph& g, unsigned long long key, uint64_t bk, bool& done) {
+    const ulonglong2* p = reinterpret_cast<const ulonglong2*>(g.eset + 4 * bk);
+    const ulonglong2 x0 = __ldg(p), x1 = __ldg(p + 1);
+    const bool hit = x0.x == key || x0.y == key || x1.x == key || x1.y == key;
+    done = hit || x0.x == kEmptyKey || x0.y == kEmptyKey || x1.x == kEmptyKey || x1.y == kEmptyKey;
+    return hit;
+}
+
+__device__ __forceinline__ void member_all2(const DeviceGraph& g, const uint32_t* Ms, int stride, int col_of,
+                                            uint32_t mask, int32_t l, int32_t x0, int32_t x1, bool& k0, bool& k1) {
+    double sec = 0.0;
+    if (!g.bloom || !g.eset) {
+        k0 = k0 && member_all<false>(g, Ms, stride, col_of, mask, l, x0, sec);
+        k1 = k1 && member_all<false>(g, Ms, stride, col_of, mask, l, x1, sec);
+        return;
+    }
+    while (mask && (k0 || k1)) {
+        const int j = __ffs(mask) - 1;
+        mask &= mask - 1;
+        const uint32_t a = Ms[j * stride + col_of];
+        const uint64_t h0 = edge_hash(a, (uint32_t)x0), h1 = edge_hash(a, (uint32_t)x1);
+        const unsigned long long w0 = k0 ? __ldg(g.bloom + (h0 & g.bloom_mask)) : 0ull;
+        const unsigned long long w1 = k1 ? __ldg(g.bloom + (h1 & g.bloom_mask)) : 0ull;
+        const uint64_t m0 = bloom_bits(h0), m1 = bloom_bits(h1);
+        k0 = k0 && (w0 & m0) == m0;
+        k1 = k1 && (w1 & m1) == m1;
+        if (!(k0 || k1)) return;
+        bool d0 = !k0, d1 = !k1, e0 = false, e1 = false;
+        uint64_t b0 = h0 & g.eset_mask, b1 = h1 & g.eset_mask;
+        const unsigned long long y0 = edge_key(a, (uint32_t)x0), y1 = edge_key(a, (uint32_t)x1);
+        if (k0) e0 = eset_first(g, y0, b0, d0);
+        if (k1) e1 = eset_first(g, y1, b1, d1);
+        while (!d0) {  // bucket overflow (rare): continue linear probing
+            b0 = (b0 + 1) & g.eset_mask;
+            e0 = eset_first(g, y0, b0, d0);
+        }
+        while (!d1) {
+            b1 = (b1 + 1) & g.eset_mask;
+            e1 = eset_first(g, y1, b1, d1);
+        }
+        k0 = k0 && e0;
+        k1 = k1 && e1;
+    }
 }
 
 // One-word signature of a lane's matched vertices: bit sig_bit(v) is set for every M[j].
@@ -763,6 +814,22 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 const int colL = wbase + L;
                 const uint32_t Lsig = __shfl_sync(kFull, msig, L);
                 uint32_t total = 0, my_bal = 0;
+                if (OCC == 1 && GSWORD_COOP_WIDE) {
+                    // register-rich build: two chunks per round, both tests in one chain
+                    for (uint32_t base = 0; base < Llen; base += 64) {
+                        const uint32_t i0 = base + lane, i1 = i0 + 32u;
+                        bool k0 = i0 < Llen, k1 = i1 < Llen;
+                        const int32_t x0 = k0 ? ldg_i32(g.clist + Llo + i0) : 0;
+                        const int32_t x1 = k1 ? ldg_i32(g.clist + Llo + i1) : 0;
+                        member_all2(g, Ms, T, colL, others, Lps.label, x0, x1, k0, k1);
+                        k0 = k0 && not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x0);
+                        k1 = k1 && not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x1);
+                        const unsigned bal0 = __ballot_sync(kFull, k0), bal1 = __ballot_sync(kFull, k1);
+                        if ((base >> 5) == (uint32_t)lane) my_bal = bal0;
+                        if ((base >> 5) + 1u == (uint32_t)lane) my_bal = bal1;
+                        total += __popc(bal0) + __popc(bal1);
+                    }
+                } else {
                 // the next chunk's driver elements are loaded while this chunk is tested
                 int32_t xn = ((uint32_t)lane < Llen) ? ldg_i32(g.clist + Llo + lane) : 0;
                 for (uint32_t base = 0; base < Llen; base += 32) {
@@ -777,6 +844,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     const unsigned bal = __ballot_sync(kFull, keep);
                     if ((base >> 5) == (uint32_t)lane) my_bal = bal;
                     total += __popc(bal);
+                }
                 }
                 int32_t chosen = -1;
                 if (total > 0) {
