@@ -254,6 +254,31 @@ def test_c3_parity_sampled(ctx, G):
                 _records_equal(rec, ref, f"C3/{q.name}/m{m}@{first}")
 
 
+def test_c4_full_size_sampled(ctx, G):
+    """BASELINE configs[4] at full size (Kronecker scale 23, 1e8 undirected edges, 16
+    labels; budgets up to 1e11 in the sweep): 4-, 8- and 16-vertex queries and a star,
+    both methods, label-only and NLF candidate filtering, a prefix checked record by
+    record and in aggregate, and windows deep in the 1e11 id range."""
+    g, qs = gen.config_c4()
+    ctx.load_graph_obj(g)
+    pick = [q for q in qs if q.name in ("dense4_s5004", "sparse8_s4008", "dense8_s5008", "dense16_s5016", "star4_s6004")]
+    assert len(pick) == 5
+    for filt in (0, 2):
+        ctx.set_option(G.OPT_FILTER, filt)
+        try:
+            for q in pick if filt == 0 else pick[2:4]:
+                for m in (0, 1):
+                    ctx.load_query_obj(q)
+                    for first, count in ((0, 10_000), (50_000_000_000, 2000), (100_000_000_000 - 2000, 2000)):
+                        rec = ctx.trace_samples(m, first, count, 11)
+                        y, ref = oracle.sample_range(g, q, m, 11, first, count, records=True, threads=1, filter=filt)
+                        _records_equal(rec, ref, f"C4/{q.name}/f{filt}/m{m}@{first}")
+                        if first == 0:
+                            _agg_close(ctx.estimate(m, count, 11), oracle.aggregate(y), G)
+        finally:
+            ctx.set_option(G.OPT_FILTER, 0)
+
+
 def test_scheduling_invariance(ctx, G, c0):
     g, qs = c0
     ctx.load_graph_obj(g)
