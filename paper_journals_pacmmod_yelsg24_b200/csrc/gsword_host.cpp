@@ -336,6 +336,13 @@ int apply_l2_window(gsword_ctx* ctx) {
     return GSWORD_OK;
 }
 
+// every position d >= 1 has exactly one backward neighbour (spanning-tree order)
+bool plan_is_tree(const Plan& p) {
+    for (int d = 1; d < p.nq; ++d)
+        if (p.step[d].nback != 1) return false;
+    return true;
+}
+
 int launch_config(gsword_ctx* ctx, int method, int mode, LaunchCfg* cfg) {
     size_t smem = 0;
     const int occ = gsword::max_blocks_per_sm(method, mode, ctx->opt_threads, &smem);
@@ -383,8 +390,10 @@ int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, u
     if (ctx->q_filter) mode |= gsword::kModeCG;
     if (method == GSWORD_ALLEY && ctx->opt_streaming && (mode & 3) != gsword::kModeCount) mode |= gsword::kModeStream;
     if (ctx->opt_sched != 0) mode |= gsword::kModeSync;
-    if ((mode & (3 | gsword::kModeSync | gsword::kModeStream)) == gsword::kModeEstimate && ctx->opt_autotune)
-        mode |= ctx->tuned_occ[method & 1] << gsword::kModeOccShift;
+    if ((mode & (3 | gsword::kModeSync | gsword::kModeStream)) == gsword::kModeEstimate) {
+        if (ctx->opt_autotune) mode |= ctx->tuned_occ[method & 1] << gsword::kModeOccShift;
+        if (plan_is_tree(ctx->plan)) mode |= gsword::kModeTree;
+    }
     LaunchCfg cfg;
     int rc = launch_config(ctx, method, mode, &cfg);
     if (rc) return rc;
@@ -1235,8 +1244,10 @@ int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out) {
     out->refill_min[1] = ctx->tuned_refill[1] ? ctx->tuned_refill[1] : ctx->opt_refill_min;
     for (int m = 0; m < 2; ++m) {
         int mode = gsword::kModeEstimate | (ctx->q_filter ? gsword::kModeCG : 0);
-        if (ctx->opt_autotune && ctx->opt_sched == 0 && !(m == GSWORD_ALLEY && ctx->opt_streaming))
-            mode |= ctx->tuned_occ[m] << gsword::kModeOccShift;
+        if (ctx->opt_sched == 0 && !(m == GSWORD_ALLEY && ctx->opt_streaming)) {
+            if (ctx->opt_autotune) mode |= ctx->tuned_occ[m] << gsword::kModeOccShift;
+            if (plan_is_tree(ctx->plan)) mode |= gsword::kModeTree;
+        }
         if (m == GSWORD_ALLEY && ctx->opt_streaming) mode |= gsword::kModeStream;
         if (ctx->opt_sched != 0) mode |= gsword::kModeSync;
         const int occ = gsword::max_blocks_per_sm(m, mode, ctx->opt_threads, nullptr);

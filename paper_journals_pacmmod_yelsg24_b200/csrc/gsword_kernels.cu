@@ -33,8 +33,8 @@ constexpr unsigned kFull = 0xffffffffu;
 #ifndef GSWORD_COOP_WIDE
 #define GSWORD_COOP_WIDE 0  // 1: occupancy variant 1 runs two coop chunks per round (measured 0-7 % slower: spills)
 #endif
-#ifndef GSWORD_POOL_DEFER
-#define GSWORD_POOL_DEFER 0  // 1: Alley task pool batches exact edge probes 32 at a time (measured 4-10 % slower)
+#ifndef GSWORD_POOL_MERGED
+#define GSWORD_POOL_MERGED 1  // Alley exclusion and membership tests in one task pool
 #endif
 // Alley drivers longer than the coop threshold (<= 64) are refined by the whole warp.
 
@@ -220,38 +220,6 @@ __device__ __forceinline__ bool is_edge(const DeviceGraph& g, uint32_t a, uint32
     return in_run(g.col, lo, hi, (int32_t)b);
 }
 
-// The two halves of is_edge for callers that batch the exact step (the Alley task pool):
-// bloom_maybe = the filter's verdict (false is final), edge_exact = the edge-set probe
-// (or the binary search when the edge set is off).
-template <bool COUNT>
-__device__ __forceinline__ bool bloom_maybe(const DeviceGraph& g, uint32_t a, uint32_t b, double& sec) {
-    if (!g.bloom) return true;
-    if (COUNT) sec += 1.0;
-    const uint64_t h = edge_hash(a, b);
-    const uint64_t m = bloom_bits(h);
-    return (__ldg(g.bloom + (h & g.bloom_mask)) & m) == m;
-}
-
-template <bool COUNT>
-__device__ __forceinline__ bool edge_exact(const DeviceGraph& g, uint32_t a, uint32_t b, int32_t lb, double& sec) {
-    if (g.eset) {
-        const unsigned long long key = edge_key(a, b);
-        uint64_t bk = edge_hash(a, b) & g.eset_mask;
-        while (true) {
-            if (COUNT) sec += 1.0;
-            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(g.eset + 4 * bk);
-            const ulonglong2 x0 = __ldg(p), x1 = __ldg(p + 1);
-            if (x0.x == key || x0.y == key || x1.x == key || x1.y == key) return true;
-            if (x0.x == kEmptyKey || x0.y == kEmptyKey || x1.x == kEmptyKey || x1.y == kEmptyKey) return false;
-            bk = (bk + 1) & g.eset_mask;
-        }
-    }
-    uint32_t lo, hi;
-    segment(g, a, lb, &lo, &hi);
-    if (COUNT) sec += 1.0 + (double)bs_sectors(hi - lo);
-    return in_run(g.col, lo, hi, (int32_t)b);
-}
-
 // Is x in every N_l(M[j]) for j in `mask`?  M column `col_of` in shared memory.
 template <bool COUNT>
 __device__ __forceinline__ bool member_all(const DeviceGraph& g, const uint32_t* Ms, int stride, int col_of,
@@ -347,7 +315,10 @@ __host__ __device__ constexpr int kOccBlocks(int method, int occ) {
 
 // SYNC: false = the default refill scheduler only (sched 0, the scheduling-mode logic
 // compiled out); true = any GSWORD_OPT_SCHEDULE (NEXT-3 comparison modes)
-template <int METHOD, int MODE, bool CG, bool SYNC, int OCC = 0>
+// TREE: every position d >= 1 has exactly one backward neighbour (a spanning-tree query
+// order, e.g. paths and stars): WanderJoin has no IsEdge validation and Alley only the
+// single-list refine, so the multi-list code is compiled out (estimate kernels only).
+template <int METHOD, int MODE, bool CG, bool SYNC, int OCC = 0, bool TREE = false>
 __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     sample_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
                                                      const uint64_t count, const uint64_t seed, const int chunk,
@@ -365,10 +336,6 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     // Alley task-pool results per lane: pool_s[0] = adjacent matched vertices (pool 1),
     // pool_s[1..4] = refine-mask removals (pool 2, 128 bits)
     __shared__ uint32_t pool_s[5][256];
-#if GSWORD_POOL_DEFER
-    // per-warp ring of edge tests the filter could not settle: (a, b, target, label)
-    __shared__ uint32_t dq_s[8][4][64];
-#endif
     __shared__ Partial warp_part[32];
     extern __shared__ uint32_t Ms[];  // Ms[j * blockDim.x + tid] = M[j] of this lane
 
@@ -388,6 +355,9 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
 
     const int nq = plan_in.nq;
     const int sched = SYNC ? sched_arg : 0;
+    bool multi_back = false;  // some position has |B(d)| >= 2 (Alley refine kinds 2/3 can occur)
+    if (!TREE)
+        for (int dd = 1; dd < nq; ++dd) multi_back |= plan_s[dd].nback >= 2;
 
     // lane state
     bool has = false;
@@ -499,13 +469,19 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 lo_p = plan_in.seed_lo;
                 len_p = plan_in.seed_len;
                 if (MODE == kModeCount) sectors += plan_in.seed_identity ? 0.0 : 1.0;
-            } else if (METHOD == GSWORD_ALLEY && ps.nback == 1) {
+            } else if (METHOD == GSWORD_ALLEY && (TREE || ps.nback == 1)) {
                 // one backward neighbour: p is fixed by the plan; the segment load is left
                 // in flight and consumed after the exclusion tests (which need only M)
                 p = __ffs(ps.back) - 1;
                 local_run<CG>(g, eidx_s[d][p], Ms[p * T + tid], ps.label, &seg_a, &seg_b);
                 deferred = true;
                 if (MODE == kModeCount) sectors += 1.0;
+            } else if (TREE) {
+                p = __ffs(ps.back) - 1;
+                uint32_t a, b;
+                local_run<CG>(g, eidx_s[d][p], Ms[p * T + tid], ps.label, &a, &b);
+                lo_p = a;
+                len_p = b - a;
             } else {
                 // GetMinCandidate (Alg. 1 l.8): the smallest N_l(M[j]) over j in B(d)
                 // (variant A3: WanderJoin takes the first backward position's list)
@@ -544,7 +520,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                         // Validate: DupCheck, then IsEdge for the other matched neighbours.
                         // v in N_l(M[j]) <=> M[j] in N_{L(phi[j])}(v): search the shorter run.
                         reject = !not_matched_sig(Ms + tid, T, 0, ps.dup, msig, v);
-                        uint32_t bm = ps.back & ~(1u << p);
+                        uint32_t bm = TREE ? 0u : ps.back & ~(1u << p);
                         while (bm && !reject) {
                             const int j = __ffs(bm) - 1;
                             bm &= bm - 1;
@@ -564,14 +540,11 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
             // exclusive scan of per-lane counts, owner found by shuffle bisection), so every
             // lane is busy whichever lanes generated the work (the refine imbalance).
             // test(o, k) runs task k of owner lane o; every lane calls it (it shuffles).
-            // test(o, k, valid, a, b, tgt, lb) names the edge {a, b} of task k of owner lane o
-            // (label lb = L(b)) and the result bit tgt = (word << 5) | bit in pool_s; the bit
-            // is set when the edge's presence equals SET_ON_EDGE.  Every lane calls it (it
-            // shuffles).  GSWORD_POOL_DEFER: a "maybe" of the filter is queued and the exact
-            // probes run 32 at a time, so the filter loads of successive rounds are not
-            // serialised behind divergent edge-set probes.
-            auto pool = [&](uint32_t ntask, auto set_on_edge, auto&& test) {
-                constexpr bool SET_ON_EDGE = decltype(set_on_edge)::value;
+            // test(o, k, valid, a, b, tgt, lb, soe) names the edge {a, b} of task k of owner
+            // lane o (label lb = L(b)), the result bit tgt = (word << 5) | bit in pool_s, and
+            // whether the bit is set on an edge (soe) or on a non-edge.  Every lane calls it
+            // (it shuffles).
+            auto pool = [&](uint32_t ntask, auto&& test) {
                 if (!__any_sync(kFull, ntask != 0u)) return;
                 uint32_t incl = ntask;
 #pragma unroll
@@ -581,22 +554,6 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 }
                 const uint32_t total = __shfl_sync(kFull, incl, 31);
                 const uint32_t excl = incl - ntask;
-#if GSWORD_POOL_DEFER
-                uint32_t(*dq)[64] = dq_s[tid >> 5];
-                uint32_t qh = 0, qn = 0;  // ring head and length (warp-uniform)
-                auto flush = [&](uint32_t n) {
-                    __syncwarp();
-                    if ((uint32_t)lane < n) {
-                        const uint32_t e = (qh + lane) & 63u;
-                        const uint32_t tg = dq[2][e];
-                        const bool is = edge_exact<MODE == kModeCount>(g, dq[0][e], dq[1][e], (int32_t)dq[3][e], sectors);
-                        if (is == SET_ON_EDGE) atomicOr(&pool_s[0][0] + (tg >> 5), 1u << (tg & 31u));
-                    }
-                    __syncwarp();
-                    qh = (qh + n) & 63u;
-                    qn -= n;
-                };
-#endif
                 for (uint32_t base = 0; base < total; base += 32) {
                     const uint32_t t = base + (uint32_t)lane;
                     const uint32_t tt = t < total ? t : total - 1;
@@ -608,30 +565,39 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     }
                     uint32_t ea = 0, eb = 0, tg = 0;
                     int32_t lb = 0;
+                    bool soe = false;
                     const bool valid = t < total;
-                    test(o, tt - __shfl_sync(kFull, excl, o), valid, ea, eb, tg, lb);
-#if GSWORD_POOL_DEFER
-                    const bool maybe = valid && bloom_maybe<MODE == kModeCount>(g, ea, eb, sectors);
-                    if (valid && !maybe && !SET_ON_EDGE) atomicOr(&pool_s[0][0] + (tg >> 5), 1u << (tg & 31u));
-                    const unsigned mb = __ballot_sync(kFull, maybe);
-                    if (maybe) {
-                        const uint32_t e = (qh + qn + __popc(mb & lt_mask)) & 63u;
-                        dq[0][e] = ea;
-                        dq[1][e] = eb;
-                        dq[2][e] = tg;
-                        dq[3][e] = (uint32_t)lb;
-                    }
-                    qn += __popc(mb);
-                    if (qn >= 32u) flush(32u);
-#else
-                    if (valid && is_edge<MODE == kModeCount>(g, ea, eb, lb, sectors) == SET_ON_EDGE)
+                    test(o, tt - __shfl_sync(kFull, excl, o), valid, ea, eb, tg, lb, soe);
+                    if (valid && is_edge<MODE == kModeCount>(g, ea, eb, lb, sectors) == soe)
                         atomicOr(&pool_s[0][0] + (tg >> 5), 1u << (tg & 31u));
-#endif
                 }
-#if GSWORD_POOL_DEFER
-                if (qn) flush(qn);
-#endif
                 __syncwarp();
+            };
+            // task of a kind-1 owner: exclusion test {M[p], M[j]} for the k-th j of `omask`,
+            // result bit j of pool_s[0] on an edge
+            auto excl_task = [&](int ocol, uint32_t omask, int op, uint32_t k, uint32_t& ea, uint32_t& eb,
+                                 uint32_t& tg, bool& soe) {
+                const int j = fns_small(omask, k);
+                ea = Ms[op * T + ocol];
+                eb = Ms[j * T + ocol];
+                tg = ((uint32_t)ocol << 5) | (uint32_t)j;  // pool_s[0][ocol], bit j
+                soe = true;
+            };
+            // task of a kind-2 owner: is S_p[i] (label l_d) in N_l(M[j]), i.e. is {M[j], S_p[i]}
+            // an edge?  task k = (list nth of `omask`, element i); result bit i of
+            // pool_s[1 + i/32] on a non-edge
+            auto memb_task = [&](int ocol, uint32_t omask, uint32_t olo, uint32_t olen, uint32_t k, uint32_t& ea,
+                                 uint32_t& eb, uint32_t& tg, bool& soe) {
+                uint32_t nth = 0u, i = k;
+                if (omask & (omask - 1u)) {  // one other list is the common case
+                    nth = k / olen;
+                    i = k - nth * olen;
+                }
+                const int j = fns_small(omask, nth);
+                ea = Ms[j * T + ocol];
+                eb = (uint32_t)ldg_i32(g.clist + olo + i);
+                tg = ((uint32_t)((1u + (i >> 5)) * 256u + (uint32_t)ocol) << 5) | (i & 31u);
+                soe = false;
             };
             int kind = 0;
             uint32_t unk = 0, known = 0, others = 0;
@@ -659,21 +625,53 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 unk = cdup & ~qa;
             }
             __syncwarp();
+#if GSWORD_POOL_MERGED
+            // kind 2 is known before the pool for lanes that waited on GetMinCandidate, so the
+            // exclusion tests (kind 1) and the membership tests (kind 2) share one pool: one
+            // pass of rounds instead of two
+            if (!TREE && has && !deferred && d > 0 && len_p > 0 && len_p <= coop_threshold) {
+                kind = 2;
+                others = ps.back & ~(1u << p);
+                if (MODE == kModeCount) sectors += (double)scan_sectors(len_p);
+            }
+            if (multi_back) {
+                const uint32_t ntask = kind == 1 ? (uint32_t)__popc(unk) : kind == 2 ? len_p * (uint32_t)__popc(others) : 0u;
+                // owner state in three words: kind | task mask (positions < 16), p or lo_p, len_p
+                const uint32_t kmask = ((uint32_t)kind << 16) | (kind == 1 ? unk : others);
+                const uint32_t pl = kind == 1 ? (uint32_t)p : lo_p;
+                pool(ntask, [&](int o, uint32_t k, bool valid, uint32_t& ea, uint32_t& eb, uint32_t& tg, int32_t& lb,
+                                bool& soe) {
+                    const uint32_t okm = __shfl_sync(kFull, kmask, o);
+                    const uint32_t opl = __shfl_sync(kFull, pl, o);
+                    const uint32_t olen = __shfl_sync(kFull, len_p, o);
+                    lb = __shfl_sync(kFull, ps.label, o);
+                    if (valid) {
+                        if ((okm >> 16) == 1u)
+                            excl_task(wbase + o, okm & 0xFFFFu, (int)opl, k, ea, eb, tg, soe);
+                        else
+                            memb_task(wbase + o, okm & 0xFFFFu, opl, olen, k, ea, eb, tg, soe);
+                    }
+                });
+            } else {
+                // no position has two backward neighbours: exclusion tests only
+                pool((kind == 1) ? (uint32_t)__popc(unk) : 0u,
+                     [&](int o, uint32_t k, bool valid, uint32_t& ea, uint32_t& eb, uint32_t& tg, int32_t& lb, bool& soe) {
+                    const uint32_t omask = __shfl_sync(kFull, unk, o);
+                    const int op = __shfl_sync(kFull, p, o);
+                    lb = __shfl_sync(kFull, ps.label, o);
+                    if (valid) excl_task(wbase + o, omask, op, k, ea, eb, tg, soe);
+                });
+            }
+#else
             // pool 1: exclusion tests, overlapping the in-flight segment loads
-            pool((kind == 1) ? (uint32_t)__popc(unk) : 0u, std::true_type{},
-                 [&](int o, uint32_t k, bool valid, uint32_t& ea, uint32_t& eb, uint32_t& tg, int32_t& lb) {
+            pool((kind == 1) ? (uint32_t)__popc(unk) : 0u,
+                 [&](int o, uint32_t k, bool valid, uint32_t& ea, uint32_t& eb, uint32_t& tg, int32_t& lb, bool& soe) {
                 const uint32_t omask = __shfl_sync(kFull, unk, o);
                 const int op = __shfl_sync(kFull, p, o);
-                const int32_t olab = __shfl_sync(kFull, ps.label, o);
-                if (valid) {
-                    const int ocol = wbase + o;
-                    const int j = fns_small(omask, k);
-                    ea = Ms[op * T + ocol];
-                    eb = Ms[j * T + ocol];
-                    lb = olab;
-                    tg = ((uint32_t)ocol << 5) | (uint32_t)j;  // pool_s[0][ocol], bit j
-                }
+                lb = __shfl_sync(kFull, ps.label, o);
+                if (valid) excl_task(wbase + o, omask, op, k, ea, eb, tg, soe);
             });
+#endif
             if (deferred) {
                 lo_p = seg_a;
                 len_p = seg_b - seg_a;
@@ -687,40 +685,28 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     }
                 } else if (len_p == 0) {
                     kind = 0;
-                } else if (!deferred) {
-                    if (len_p <= coop_threshold) {
+                } else if (!TREE && !deferred) {
+                    if (len_p > coop_threshold) {
+                        kind = 3;
+                    } else if (!GSWORD_POOL_MERGED) {
                         kind = 2;
                         others = ps.back & ~(1u << p);
                         if (MODE == kModeCount) sectors += (double)scan_sectors(len_p);
-                    } else {
-                        kind = 3;
                     }
                 }
             }
             mark(3);
+#if !GSWORD_POOL_MERGED
             // pool 2: membership tests of short refine masks
-            pool((kind == 2) ? len_p * (uint32_t)__popc(others) : 0u, std::false_type{},
-                 [&](int o, uint32_t k, bool valid, uint32_t& ea, uint32_t& eb, uint32_t& tg, int32_t& lb) {
+            pool((kind == 2) ? len_p * (uint32_t)__popc(others) : 0u,
+                 [&](int o, uint32_t k, bool valid, uint32_t& ea, uint32_t& eb, uint32_t& tg, int32_t& lb, bool& soe) {
                 const uint32_t omask = __shfl_sync(kFull, others, o);
                 const uint32_t olo = __shfl_sync(kFull, lo_p, o);
                 const uint32_t olen = __shfl_sync(kFull, len_p, o);
-                const int32_t olab = __shfl_sync(kFull, ps.label, o);
-                if (valid) {
-                    const int ocol = wbase + o;
-                    // is S_p[i] (label l_d) in N_l(M[j]), i.e. is {M[j], S_p[i]} an edge?
-                    // task k = (list nth, element i); one other list is the common case
-                    uint32_t nth = 0u, i = k;
-                    if (omask & (omask - 1u)) {
-                        nth = k / olen;
-                        i = k - nth * olen;
-                    }
-                    const int j = fns_small(omask, nth);
-                    ea = Ms[j * T + ocol];
-                    eb = (uint32_t)ldg_i32(g.clist + olo + i);
-                    lb = olab;
-                    tg = ((uint32_t)((1u + (i >> 5)) * 256u + (uint32_t)ocol) << 5) | (i & 31u);  // pool_s[1 + i/32][ocol]
-                }
+                lb = __shfl_sync(kFull, ps.label, o);
+                if (valid) memb_task(wbase + o, omask, olo, olen, k, ea, eb, tg, soe);
             });
+#endif
             mark(4);
             if (kind == 1) {
                 const uint32_t in_sp = known | pool_s[0][tid];  // matched vertices inside S_p
@@ -762,7 +748,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     }
                     if (MODE == kModeCount) sectors += 1.0;
                 }
-            } else if (kind == 2) {
+            } else if (!TREE && kind == 2) {
                 // refine mask over S_p (<= 128 elements, 4 words): not removed by a membership
                 // test and not a matched same-label vertex (injectivity)
                 const uint32_t dup = ps.dup & ~(1u << p);
@@ -795,12 +781,12 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     v = ldg_i32(g.clist + lo_p + pos - 1u);
                 }
             }
-            const bool coop = (kind == 3);
+            const bool coop = !TREE && (kind == 3);
             mark(5);
 
             // ---------------- warp-cooperative refine for long drivers ----------------
-            unsigned cm = __ballot_sync(kFull, coop);
-            while (cm) {
+            unsigned cm = TREE ? 0u : __ballot_sync(kFull, coop);
+            while (!TREE && cm) {
                 const int L = __ffs(cm) - 1;
                 cm &= cm - 1;
                 const uint32_t Llo = __shfl_sync(kFull, lo_p, L);
@@ -1741,12 +1727,17 @@ __global__ void scan_add_kernel(uint32_t* __restrict__ data, int64_t n, const ui
     if (i0 + 1 < n) data[i0 + 1] += add;
 }
 
+template <int METHOD, bool CG, bool TREE>
+const void* estimate_ptr(int occ) {
+    if (occ == 1) return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 1, TREE>);
+    if (occ == 2) return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 2, TREE>);
+    return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 0, TREE>);
+}
+
 template <int METHOD, int MODE, bool CG>
-const void* kernel_ptr(bool sync, int occ = 0) {
-    if (MODE == kModeEstimate && !sync && occ == 1)
-        return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 1>);
-    if (MODE == kModeEstimate && !sync && occ == 2)
-        return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 2>);
+const void* kernel_ptr(bool sync, int occ = 0, bool tree = false) {
+    if (MODE == kModeEstimate && !sync)
+        return tree ? estimate_ptr<METHOD, CG, true>(occ) : estimate_ptr<METHOD, CG, false>(occ);
     return sync ? reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE, CG, true>)
                 : reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE, CG, false>);
 }
@@ -1759,15 +1750,16 @@ const void* select_kernel_cg(int method, int mode) {
     }
     const bool sync = (mode & kModeSync) != 0;
     const int occ = (mode >> kModeOccShift) & 3;
+    const bool tree = (mode & kModeTree) != 0;
     mode &= 3;
     if (method == GSWORD_WJ) {
         if (mode == kModeTrace) return kernel_ptr<GSWORD_WJ, kModeTrace, CG>(sync);
         if (mode == kModeCount) return kernel_ptr<GSWORD_WJ, kModeCount, CG>(sync);
-        return kernel_ptr<GSWORD_WJ, kModeEstimate, CG>(sync, occ);
+        return kernel_ptr<GSWORD_WJ, kModeEstimate, CG>(sync, occ, tree);
     }
     if (mode == kModeTrace) return kernel_ptr<GSWORD_ALLEY, kModeTrace, CG>(sync);
     if (mode == kModeCount) return kernel_ptr<GSWORD_ALLEY, kModeCount, CG>(sync);
-    return kernel_ptr<GSWORD_ALLEY, kModeEstimate, CG>(sync, occ);
+    return kernel_ptr<GSWORD_ALLEY, kModeEstimate, CG>(sync, occ, tree);
 }
 
 // mode: kMode* | kModeCG when the query was loaded with a candidate filter

@@ -204,8 +204,9 @@ enum Mode {
     kModeCG = 4,     // flag: candidate graph
     kModeStream = 8,  // flag: Alley by warp streaming (Alg. 3, NEXT-3)
     kModeSync = 16,   // flag: a scheduling mode other than refill (GSWORD_OPT_SCHEDULE != 0)
-    kModeOccShift = 5  // bits 5-6: occupancy variant of the estimate kernel (0 default, 1 one
-                       // CTA/SM less, 2 one more; refill schedule only), see occ_blocks()
+    kModeOccShift = 5,  // bits 5-6: occupancy variant of the estimate kernel (0 default, 1 one
+                        // CTA/SM less, 2 one more; refill schedule only), see occ_blocks()
+    kModeTree = 128     // flag: every position has one backward neighbour (estimate kernels)
 };
 
 }  // namespace gsword
