@@ -1,11 +1,15 @@
 """Short, fixed launch sequence for ncu captures (one GPU, never multi-rank):
 2 warm-up estimates (WanderJoin, Alley; 1e6 samples), then WanderJoin and Alley at
---samples each on the bench workload.  Use `ncu -k regex:sample_kernel -s 2 -c 2`."""
+--samples each on the bench workload, bracketed by cudaProfilerStart/Stop so that
+`ncu --profile-from-start off -k regex:sample_kernel` captures exactly those two launches
+(whatever the autotune at query load launched before)."""
 import argparse
 import os
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
 
 import paper_journals_pacmmod_yelsg24_b200 as G  # noqa: E402
 from workloads import gen  # noqa: E402
@@ -37,7 +41,10 @@ with G.Context(0) as ctx:
     ctx.load_query_obj(q)
     for m in (G.WJ, G.ALLEY):
         ctx.estimate(m, 1_000_000, 42)
-    for m in (G.WJ, G.ALLEY):
-        r = ctx.estimate(m, int(args.samples), 42)
+    torch.cuda.synchronize()
+    torch.cuda.profiler.start()
+    res = {m: ctx.estimate(m, int(args.samples), 42) for m in (G.WJ, G.ALLEY)}
+    torch.cuda.profiler.stop()
+    for m, r in res.items():
         print(f"method={m} samples={int(args.samples)} seconds={r['seconds']:.4f} "
               f"rate={args.samples / r['seconds']:.3e}/s est={r['estimate']:.4e} valid={r['n_valid']}")

@@ -13,8 +13,8 @@ mkdir -p gpurun_out profiles
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
     --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline \
     > gpurun_out/${TAG}_launches_bench.log 2>&1
-# profile_driver: 10 autotune launches + 2 warm-ups precede the two bench-size launches
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:sample_kernel -s 12 -c 2 \
+# profile_driver brackets the two bench-size launches with cudaProfilerStart/Stop
+timeout 900 ncu --set full --import-source on --clock-control none --profile-from-start off -k regex:sample_kernel -c 2 \
     -o gpurun_out/${TAG}_full python scripts/profile_driver.py --samples 1e8 > gpurun_out/${TAG}_full.log 2>&1
 python scripts/ncu_summary.py gpurun_out/${TAG}_full.ncu-rep profiles/${TAG}_ncu_details.json 1e8 \
     > gpurun_out/${TAG}_summary.log 2>&1
