@@ -1214,7 +1214,7 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
         for (int m = 0; m < 2; ++m) {
             ctx->tuned_occ[m] = 0;
             for (int c = 0; c < 2; ++c)
-                if (t2[m][c] < 0.97f * best[m]) {  // a variant must win by 3 % (pilot noise)
+                if (t2[m][c] < 0.985f * best[m]) {  // a variant must win by 1.5 % (pilot noise)
                     best[m] = t2[m][c];
                     ctx->tuned_occ[m] = 1 + c;
                 }

@@ -30,6 +30,9 @@ constexpr unsigned kFull = 0xffffffffu;
 #ifndef GSWORD_SELECT_WINDOW
 #define GSWORD_SELECT_WINDOW 1  // Alley single-list select: window load + register fixed point
 #endif
+#ifndef GSWORD_SMEM_ACC
+#define GSWORD_SMEM_ACC 1  // Alley: per-lane compensated sums in shared memory
+#endif
 #ifndef GSWORD_COOP_WIDE
 #define GSWORD_COOP_WIDE 0  // 1: occupancy variant 1 runs two coop chunks per round (measured 0-7 % slower: spills)
 #endif
@@ -368,6 +371,27 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     // lane accumulators
     double s_sum = 0.0, c_sum = 0.0, s_sq = 0.0, c_sq = 0.0;
     unsigned long long n_valid = 0, n_done = 0;
+    // Alley (GSWORD_SMEM_ACC): the compensated sums live in shared memory (touched only when
+    // a sample completes), freeing 8 registers for the refine paths
+    constexpr bool kSmemAcc = GSWORD_SMEM_ACC && METHOD == GSWORD_ALLEY;
+    __shared__ double acc_s[kSmemAcc ? 4 : 1][256];
+    if (kSmemAcc)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) acc_s[i][tid] = 0.0;
+    auto accumulate = [&](double y) {
+        if (kSmemAcc) {
+            double a = acc_s[0][tid], b = acc_s[1][tid], c = acc_s[2][tid], e = acc_s[3][tid];
+            nsum(a, b, y);
+            nsum(c, e, __dmul_rn(y, y));
+            acc_s[0][tid] = a;
+            acc_s[1][tid] = b;
+            acc_s[2][tid] = c;
+            acc_s[3][tid] = e;
+        } else {
+            nsum(s_sum, c_sum, y);
+            nsum(s_sq, c_sq, __dmul_rn(y, y));
+        }
+    };
     double sectors = 0.0;
 
     // warp chunk of the queue (warp-uniform)
@@ -403,10 +427,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
             double gsum = g_acc;
 #pragma unroll
             for (int o = 16; o > 0; o >>= 1) gsum = __dadd_rn(gsum, shfl_xor_d(gsum, o));
-            if (lane == 0) {
-                nsum(s_sum, c_sum, gsum);
-                nsum(s_sq, c_sq, __dmul_rn(gsum, gsum));
-            }
+            if (lane == 0) accumulate(gsum);
             g_acc = 0.0;
             group_open = false;
         }
@@ -907,8 +928,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     if (sched == 2) {
                         g_acc = __dadd_rn(g_acc, W);
                     } else {
-                        nsum(s_sum, c_sum, W);
-                        nsum(s_sq, c_sq, __dmul_rn(W, W));
+                        accumulate(W);
                     }
                 }
                 if (MODE == kModeTrace) {
@@ -949,10 +969,13 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
         double gsum = g_acc;
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) gsum = __dadd_rn(gsum, shfl_xor_d(gsum, o));
-        if (lane == 0) {
-                nsum(s_sum, c_sum, gsum);
-                nsum(s_sq, c_sq, __dmul_rn(gsum, gsum));
-            }
+        if (lane == 0) accumulate(gsum);
+    }
+    if (kSmemAcc) {
+        s_sum = acc_s[0][tid];
+        c_sum = acc_s[1][tid];
+        s_sq = acc_s[2][tid];
+        c_sq = acc_s[3][tid];
     }
 
     mark(7);
