@@ -345,7 +345,8 @@ bool plan_is_tree(const Plan& p) {
 
 int launch_config(gsword_ctx* ctx, int method, int mode, LaunchCfg* cfg) {
     size_t smem = 0;
-    const int occ = gsword::max_blocks_per_sm(method, mode, ctx->opt_threads, &smem);
+    const int rows = ctx->query_loaded ? std::max(1, ctx->plan.nq) : GSWORD_MAX_QV;
+    const int occ = gsword::max_blocks_per_sm(method, mode, ctx->opt_threads, rows, &smem);
     if (occ <= 0) return fail(GSWORD_ECUDA, "kernel does not fit on the device (threads=%d)", ctx->opt_threads);
     const int bps = ctx->opt_blocks_per_sm > 0 ? std::min(ctx->opt_blocks_per_sm, occ) : occ;
     cfg->grid = ctx->num_sms * bps;
@@ -353,6 +354,7 @@ int launch_config(gsword_ctx* ctx, int method, int mode, LaunchCfg* cfg) {
     cfg->chunk = ctx->opt_sched ? ((ctx->opt_chunk + 31) / 32) * 32 : ctx->opt_chunk;  // groups of 32 ids
     cfg->coop_threshold = ctx->opt_coop;
     cfg->sched = ctx->opt_sched;
+    cfg->ms_rows = rows;
     cfg->refill_min = (uint32_t)((ctx->opt_autotune && ctx->tuned_refill[method & 1] > 0) ? ctx->tuned_refill[method & 1]
                                                                                        : ctx->opt_refill_min);
     if (cfg->grid > ctx->partial_cap) {
@@ -1250,7 +1252,7 @@ int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out) {
         }
         if (m == GSWORD_ALLEY && ctx->opt_streaming) mode |= gsword::kModeStream;
         if (ctx->opt_sched != 0) mode |= gsword::kModeSync;
-        const int occ = gsword::max_blocks_per_sm(m, mode, ctx->opt_threads, nullptr);
+        const int occ = gsword::max_blocks_per_sm(m, mode, ctx->opt_threads, std::max(1, ctx->plan.nq), nullptr);
         out->occupancy[m] = ctx->opt_blocks_per_sm > 0 ? std::min(ctx->opt_blocks_per_sm, occ) : occ;
     }
     return GSWORD_OK;

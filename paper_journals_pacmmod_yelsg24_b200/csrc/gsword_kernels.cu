@@ -1795,8 +1795,8 @@ const void* select_kernel(int method, int mode) {
 
 int occ_blocks(int method, int occ_variant) { return kOccBlocks(method, occ_variant); }
 
-int max_blocks_per_sm(int method, int mode, int threads, size_t* smem_bytes) {
-    const size_t smem = (size_t)kMaxQV * (size_t)threads * sizeof(uint32_t);
+int max_blocks_per_sm(int method, int mode, int threads, int ms_rows, size_t* smem_bytes) {
+    const size_t smem = (size_t)ms_rows * (size_t)threads * sizeof(uint32_t);
     if (smem_bytes) *smem_bytes = smem;
     int blocks = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, select_kernel(method, mode), threads, smem) !=
@@ -1811,7 +1811,9 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
                           cudaStream_t stream) {
     cudaError_t e = cudaMemsetAsync(d_queue, 0, sizeof(unsigned long long), stream);
     if (e != cudaSuccess) return e;
-    const size_t smem = (size_t)kMaxQV * (size_t)cfg.threads * sizeof(uint32_t);
+    // Ms[j * threads + tid] for j < n_q only: sizing it by the query leaves the rest of the
+    // 256 KB L1/shared array to the L1 cache (spill slots, hot CSR entries)
+    const size_t smem = (size_t)cfg.ms_rows * (size_t)cfg.threads * sizeof(uint32_t);
     const uint32_t thr = (uint32_t)cfg.coop_threshold;
     void* args[] = {(void*)&g,      (void*)&plan,  (void*)&first,   (void*)&count,     (void*)&seed,
                     (void*)&cfg.chunk, (void*)&thr, (void*)&cfg.sched, (void*)&cfg.refill_min, (void*)&d_queue,

@@ -123,6 +123,7 @@ struct LaunchCfg {
     int coop_threshold;
     int sched;  // 0 refill, 1 sample synchronisation, 2 + inheritance (NEXT-3)
     uint32_t refill_min;  // sched 0: refill when at least this many lanes are free (1..32)
+    int ms_rows;          // rows of the per-lane matched-vertex array in shared memory (n_q)
 };
 
 // Applies the GSWORD_OPT_VARIANT bits to a copy of the loaded plan (readings A3, A5).
@@ -193,7 +194,8 @@ cudaError_t launch_build_eset(const int64_t* d_row_ptr, const int32_t* col, int6
                               uint64_t mask, cudaStream_t stream);
 cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* bloom,
                                uint64_t mask, cudaStream_t stream);
-int max_blocks_per_sm(int method, int mode, int threads, size_t* smem_bytes);
+// ms_rows = query vertices (rows of the dynamic shared-memory matched-vertex array)
+int max_blocks_per_sm(int method, int mode, int threads, int ms_rows, size_t* smem_bytes);
 // minimum resident CTAs per SM the sampling kernel is compiled for (launch bounds)
 int occ_blocks(int method, int occ_variant);
 
