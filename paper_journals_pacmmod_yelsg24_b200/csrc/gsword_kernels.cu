@@ -33,6 +33,9 @@ constexpr unsigned kFull = 0xffffffffu;
 #ifndef GSWORD_SMEM_ACC
 #define GSWORD_SMEM_ACC 1  // Alley: per-lane compensated sums in shared memory
 #endif
+#ifndef GSWORD_SMEM_QUEUE
+#define GSWORD_SMEM_QUEUE 1  // queue chunk and sample/valid counters in shared memory
+#endif
 #ifndef GSWORD_COOP_WIDE
 #define GSWORD_COOP_WIDE 0  // 1: occupancy variant 1 runs two coop chunks per round (measured 0-7 % slower: spills)
 #endif
@@ -374,6 +377,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     // Alley (GSWORD_SMEM_ACC): the compensated sums live in shared memory (touched only when
     // a sample completes), freeing 8 registers for the refine paths
     constexpr bool kSmemAcc = GSWORD_SMEM_ACC && METHOD == GSWORD_ALLEY;
+    constexpr bool kSmemQueue = GSWORD_SMEM_QUEUE != 0;
     __shared__ double acc_s[kSmemAcc ? 4 : 1][256];
     if (kSmemAcc)
 #pragma unroll
@@ -397,6 +401,16 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     // warp chunk of the queue (warp-uniform)
     uint64_t q_next = 0, q_end = 0;
     bool exhausted = false;
+    // GSWORD_SMEM_QUEUE: the warp's queue chunk, its sample count and the lanes' valid counts
+    // live in shared memory (touched at refill / completion only): 8 registers fewer in the
+    // sampling loop
+    __shared__ unsigned long long wq_s[kSmemQueue ? 8 : 1][3];  // q_next, q_end, n of the warp
+    __shared__ uint32_t nv_s[kSmemQueue ? 256 : 1];
+    if (kSmemQueue) {
+        if (lane == 0) wq_s[tid >> 5][0] = wq_s[tid >> 5][1] = wq_s[tid >> 5][2] = 0ull;
+        nv_s[tid] = 0u;
+        __syncwarp();
+    }
     // scheduling (NEXT-3 comparison modes): 0 refill free lanes every round; 1 sample
     // synchronisation (a warp refills only when all 32 lanes are free); 2 sample
     // synchronisation + sample inheritance (Alg. 2, reading A24)
@@ -436,6 +450,10 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
         if (sched == 0 && (uint32_t)__popc(need) < refill_min) need = 0u;
         if (need == kFull) member = false;
         while (need && !exhausted) {
+            if (kSmemQueue) {
+                q_next = wq_s[tid >> 5][0];
+                q_end = wq_s[tid >> 5][1];
+            }
             if (q_next == q_end) {
                 unsigned long long base = 0;
                 if (lane == 0) base = atomicAdd(queue, (unsigned long long)chunk);
@@ -452,7 +470,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
             if (!has && rank < avail) {
                 has = true;
                 member = true;
-                n_done += 1;  // every sample id counts in n (reading A8)
+                if (!kSmemQueue) n_done += 1;  // every sample id counts in n (reading A8)
                 sid = first + q_next + rank;
                 d = 0;
                 W = 1.0;
@@ -467,7 +485,17 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     }
                 }
             }
-            q_next += min((uint32_t)__popc(need), avail);
+            const uint32_t took = min((uint32_t)__popc(need), avail);
+            q_next += took;
+            if (kSmemQueue) {
+                __syncwarp();
+                if (lane == 0) {
+                    wq_s[tid >> 5][0] = q_next;
+                    wq_s[tid >> 5][1] = q_end;
+                    wq_s[tid >> 5][2] += took;  // every sample id counts in n (reading A8)
+                }
+                __syncwarp();
+            }
             need = __ballot_sync(kFull, !has);
             group_open = true;
             if (sched != 0) break;  // one group of <= 32 consecutive ids at a time
@@ -924,7 +952,10 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
             }
             if (dead || complete) {
                 if (complete) {
-                    n_valid += 1;
+                    if (kSmemQueue)
+                        nv_s[tid] += 1u;
+                    else
+                        n_valid += 1;
                     if (sched == 2) {
                         g_acc = __dadd_rn(g_acc, W);
                     } else {
@@ -984,6 +1015,11 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
         for (int i = 0; i < 8; ++i) atomicAdd(phase_out + i, ph[i]);
     }
 
+    if (kSmemQueue) {
+        __syncwarp();
+        n_valid = nv_s[tid];
+        n_done = (lane == 0) ? wq_s[tid >> 5][2] : 0ull;
+    }
     // ---------------- A10: warp -> CTA partial, fixed order ----------------
     double sh = __dadd_rn(s_sum, c_sum), sl = __dsub_rn(c_sum, __dsub_rn(sh, s_sum));
     double qh = __dadd_rn(s_sq, c_sq), ql = __dsub_rn(c_sq, __dsub_rn(qh, s_sq));
