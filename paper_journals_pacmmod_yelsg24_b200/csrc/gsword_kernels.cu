@@ -36,6 +36,9 @@ constexpr unsigned kFull = 0xffffffffu;
 #ifndef GSWORD_SMEM_QUEUE
 #define GSWORD_SMEM_QUEUE 1  // queue chunk and sample/valid counters in shared memory
 #endif
+#ifndef GSWORD_SMEM_LANE
+#define GSWORD_SMEM_LANE 1  // sample id and running weight in shared memory
+#endif
 #ifndef GSWORD_COOP_WIDE
 #define GSWORD_COOP_WIDE 0  // 1: occupancy variant 1 runs two coop chunks per round (measured 0-7 % slower: spills)
 #endif
@@ -368,9 +371,18 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     // lane state
     bool has = false;
     uint32_t msig = 0u;  // signature of M[0..d-1] (sig_bit)
-    uint64_t sid = 0;
+    // GSWORD_SMEM_LANE (Alley): the sample id and the running weight W live in shared memory (read
+    // once per step), 4 registers fewer in the sampling loop
+    constexpr bool kSmemLane = GSWORD_SMEM_LANE && METHOD == GSWORD_ALLEY;
+    __shared__ uint64_t sid_s[kSmemLane ? 256 : 1];
+    __shared__ double W_s[kSmemLane ? 256 : 1];
+    uint64_t sid_r = 0;
+    double W_r = 0.0;
+    uint64_t& sid = kSmemLane ? sid_s[tid] : sid_r;
+    double& W = kSmemLane ? W_s[tid] : W_r;
+    sid = 0;
     int d = 0;
-    double W = 0.0;
+    W = 0.0;
     // lane accumulators
     double s_sum = 0.0, c_sum = 0.0, s_sq = 0.0, c_sq = 0.0;
     unsigned long long n_valid = 0, n_done = 0;
