@@ -370,7 +370,11 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
 
     // lane state
     bool has = false;
-    uint32_t msig = 0u;  // signature of M[0..d-1] (sig_bit)
+    // signature of M[0..d-1] (sig_bit); Alley keeps it in shared memory with the sample id
+    __shared__ uint32_t msig_s[(GSWORD_SMEM_LANE && METHOD == GSWORD_ALLEY) ? 256 : 1];
+    uint32_t msig_r = 0u;
+    uint32_t& msig = (GSWORD_SMEM_LANE && METHOD == GSWORD_ALLEY) ? msig_s[tid] : msig_r;
+    msig = 0u;
     // GSWORD_SMEM_LANE (Alley): the sample id and the running weight W live in shared memory (read
     // once per step), 4 registers fewer in the sampling loop
     constexpr bool kSmemLane = GSWORD_SMEM_LANE && METHOD == GSWORD_ALLEY;
