@@ -19,6 +19,9 @@ flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 work = [w.split(":") for w in os.environ.get("VB_WORK", "C1:1,C1:0,C2:0").split(",")]
 cache = {}
 with G.Context(0) as ctx:
+    opts = [o.split("=") for o in os.environ.get("VB_OPTS", "").split(",") if o]
+    for k, v in opts:  # gsword_set_option(id, value) before any load, e.g. VB_OPTS=11=32
+        ctx.set_option(int(k), int(v))
     for cfg, qi in work:
         if cfg not in cache:
             cache[cfg] = gen.CONFIGS[cfg]()
@@ -33,7 +36,7 @@ with G.Context(0) as ctx:
                 torch.cuda.synchronize()
                 r = ctx.estimate(m, N, 42)
                 ts.append(ctx.last_kernel_seconds())
-            print(json.dumps({"lib": os.path.basename(G.gsword.LIB_PATH), "config": cfg, "query": int(qi), "method": m,
+            print(json.dumps({"lib": os.path.basename(G.gsword.LIB_PATH) + os.environ.get("VB_TAG", ""), "config": cfg, "query": int(qi), "method": m,
                               "kernel_ms": 1e3 * min(ts), "samples_per_s": N / min(ts), "est": r["estimate"],
                               "valid": r["n_valid"], "tuned": ctx.query_info()}), flush=True)
 """ % HERE
