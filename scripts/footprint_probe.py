@@ -18,10 +18,14 @@ from workloads import gen  # noqa: E402
 
 N = int(float(sys.argv[1])) if len(sys.argv) > 1 else 100_000_000
 scales = [float(x) for x in sys.argv[2].split(",")] if len(sys.argv) > 2 else [1.0, 0.5, 0.25, 0.125]
+# optional gsword_set_option pairs applied before the loads, e.g. "5=0" (filter off)
+opts = [tuple(int(v) for v in o.split("=")) for o in sys.argv[3].split(",")] if len(sys.argv) > 3 else []
 _, qs = gen.config_c1()
 q = qs[1]
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 with G.Context(0) as ctx:
+    for k, v in opts:
+        ctx.set_option(k, v)
     for s in scales:
         n, m = int(862_664 * s), int(16_138_468 * s)
         g = gen.chung_lu(n, m, gamma=2.1, max_over_mean=68_963 / 37.4, seed=2005, name=f"cl_{s}")
@@ -37,6 +41,6 @@ with G.Context(0) as ctx:
                 ts.append(ctx.last_kernel_seconds())
             sec = ctx.count_sectors(meth, 0, 1_000_000, 42) / 1_000_000
             t = min(ts)
-            print(json.dumps({"scale": s, "n": n, "m": m, "col_mb": 8 * m / 2**20, "method": meth, "kernel_ms": 1e3 * t,
+            print(json.dumps({"opts": opts, "scale": s, "n": n, "m": m, "col_mb": 8 * m / 2**20, "method": meth, "kernel_ms": 1e3 * t,
                               "samples_per_s": N / t, "sectors_per_sample": sec, "valid_fraction": r["n_valid"] / N,
                               "GBps_alg": sec * 32 * N / t / 1e9}), flush=True)
