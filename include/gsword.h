@@ -185,6 +185,10 @@ typedef enum {
                                    /* in SURVEY R3-R5).  Applies to estimates and     */
                                    /* traces (every schedule, streaming included);    */
                                    /* trawling ignores it                             */
+    GSWORD_OPT_OCCUPANCY = 14,     /* estimate-kernel occupancy variant: -1 (default) */
+                                   /* the autotuned one; 0 default launch bounds, 1   */
+                                   /* one CTA/SM less, 2 one more (forced; for A/B    */
+                                   /* and sanitizer runs).  Results are unaffected    */
     GSWORD_OPT_FILTER = 7          /* candidate filter applied by the next            */
                                    /* gsword_load_query: 0 label only, 1 LDF, 2 NLF   */
                                    /* (1-2 build the candidate graph, reading A21)    */

@@ -263,6 +263,7 @@ struct gsword_ctx {
     // autotune results per (query, options) since the last graph load: reloading a query
     // (a serving loop re-issuing the same query) reuses them instead of re-running pilots
     int tuned_occ[2] = {0, 0};    // occupancy variant of the estimate kernel (kModeOccShift)
+    int opt_occ = -1;             // GSWORD_OPT_OCCUPANCY: -1 autotuned, else forced
     struct Tuned {
         int refill[2], occ[2];
     };
@@ -336,6 +337,12 @@ int apply_l2_window(gsword_ctx* ctx) {
     return GSWORD_OK;
 }
 
+// occupancy variant of the estimate kernel in use for `method`
+int occ_variant(const gsword_ctx* ctx, int method) {
+    if (ctx->opt_occ >= 0) return ctx->opt_occ;
+    return ctx->opt_autotune ? ctx->tuned_occ[method & 1] : 0;
+}
+
 // every position d >= 1 has exactly one backward neighbour (spanning-tree order)
 bool plan_is_tree(const Plan& p) {
     for (int d = 1; d < p.nq; ++d)
@@ -393,7 +400,7 @@ int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, u
     if (method == GSWORD_ALLEY && ctx->opt_streaming && (mode & 3) != gsword::kModeCount) mode |= gsword::kModeStream;
     if (ctx->opt_sched != 0) mode |= gsword::kModeSync;
     if ((mode & (3 | gsword::kModeSync | gsword::kModeStream)) == gsword::kModeEstimate) {
-        if (ctx->opt_autotune) mode |= ctx->tuned_occ[method & 1] << gsword::kModeOccShift;
+        mode |= occ_variant(ctx, method) << gsword::kModeOccShift;
         if (plan_is_tree(ctx->plan)) mode |= gsword::kModeTree;
     }
     LaunchCfg cfg;
@@ -746,6 +753,10 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
             return GSWORD_OK;
         case GSWORD_OPT_STREAMING:
             ctx->opt_streaming = value ? 1 : 0;
+            return GSWORD_OK;
+        case GSWORD_OPT_OCCUPANCY:
+            if (value < -1 || value > 2) return fail(GSWORD_EINVAL, "occupancy variant must be -1..2");
+            ctx->opt_occ = (int)value;
             return GSWORD_OK;
         case GSWORD_OPT_VARIANT:
             if (value & ~(int64_t)(GSWORD_VARIANT_WJ_PARENT_FIRST | GSWORD_VARIANT_ALLEY_DUPCHECK_POST))
@@ -1212,10 +1223,10 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
             ctx->tuned_refill[m] = cand[bc];
             best[m] = t1[m][bc];
         }
-        time_phase(2, [&](int m, int c) { ctx->tuned_occ[m] = 1 + c; }, t2);
+        if (ctx->opt_occ < 0) time_phase(2, [&](int m, int c) { ctx->tuned_occ[m] = 1 + c; }, t2);
         for (int m = 0; m < 2; ++m) {
             ctx->tuned_occ[m] = 0;
-            for (int c = 0; c < 2; ++c)
+            for (int c = 0; c < 2 && ctx->opt_occ < 0; ++c)
                 if (t2[m][c] < 0.985f * best[m]) {  // a variant must win by 1.5 % (pilot noise)
                     best[m] = t2[m][c];
                     ctx->tuned_occ[m] = 1 + c;
@@ -1247,7 +1258,7 @@ int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out) {
     for (int m = 0; m < 2; ++m) {
         int mode = gsword::kModeEstimate | (ctx->q_filter ? gsword::kModeCG : 0);
         if (ctx->opt_sched == 0 && !(m == GSWORD_ALLEY && ctx->opt_streaming)) {
-            if (ctx->opt_autotune) mode |= ctx->tuned_occ[m] << gsword::kModeOccShift;
+            mode |= occ_variant(ctx, m) << gsword::kModeOccShift;
             if (plan_is_tree(ctx->plan)) mode |= gsword::kModeTree;
         }
         if (m == GSWORD_ALLEY && ctx->opt_streaming) mode |= gsword::kModeStream;

@@ -11,13 +11,19 @@ from workloads import gen  # noqa: E402
 g = gen.chung_lu(2000, 30_000, gamma=2.2, max_over_mean=40.0, seed=3, labels=gen.uniform_labels(2000, 2, 4),
                  n_labels=2)
 q = gen.extract_query(g, 6, seed=5, dense=True, require_dense=True)
+qt = gen.extract_query(g, 6, seed=6, dense=False)  # tree order: the TREE estimate kernels
 with G.Context(0) as ctx:
+    ctx.set_option(G.OPT_AUTOTUNE, 0)  # no pilots under the sanitizer; variants forced below
     ctx.load_graph_obj(g)
-    ctx.load_query_obj(q)
-    for coop in (0, 64):
-        ctx.set_option(G.OPT_COOP_THRESHOLD, coop)
-        for m in (G.WJ, G.ALLEY):
-            r = ctx.estimate(m, 20_000, 1)
-            rec = ctx.trace_samples(m, 0, 2000, 1)
-            s = ctx.count_sectors(m, 0, 2000, 1)
-            print(m, coop, r["n_valid"], int(rec["valid"].sum()), s)
+    for qq in (q, qt):
+        ctx.load_query_obj(qq)
+        for coop in (0, 64):
+            ctx.set_option(G.OPT_COOP_THRESHOLD, coop)
+            for m in (G.WJ, G.ALLEY):
+                for occ in (0, 1, 2):  # every occupancy variant of the estimate kernel
+                    ctx.set_option(G.OPT_OCCUPANCY, occ)
+                    r = ctx.estimate(m, 20_000, 1)
+                ctx.set_option(G.OPT_OCCUPANCY, -1)
+                rec = ctx.trace_samples(m, 0, 2000, 1)
+                s = ctx.count_sectors(m, 0, 2000, 1)
+                print(qq.name, m, coop, r["n_valid"], int(rec["valid"].sum()), s)

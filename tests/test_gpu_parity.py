@@ -552,16 +552,22 @@ def test_autotune_does_not_change_results(ctx, G, c0):
     ctx.load_query_obj(q)
     assert ctx.query_info()["refill_min"] == info["refill_min"]
     assert ctx.query_info()["occupancy"] == info["occupancy"]
-    # every occupancy variant of the estimate kernel gives the same aggregate
-    for m in (0, 1):
-        ref_agg = ctx.estimate(m, 50_000, 9)
-        for bps in (3, 4):
-            ctx.set_option(G.OPT_BLOCKS_PER_SM, bps)
-            try:
-                agg = ctx.estimate(m, 50_000, 9)
-            finally:
-                ctx.set_option(G.OPT_BLOCKS_PER_SM, 0)
-            assert agg["n_valid"] == ref_agg["n_valid"] and agg["sum"] == pytest.approx(ref_agg["sum"], rel=REL)
+    # every occupancy variant of the estimate kernel (forced), and a limited grid, gives the
+    # oracle's aggregate, for a tree order (TREE kernels) and a non-tree one
+    for qq in (q, gen.path_query(4, labels=[int(x) for x in q.labels[:4]]) if q.nq >= 4 else q):
+        ctx.load_query_obj(qq)
+        for m in (0, 1):
+            y, _ = oracle.sample_range(g, qq, m, 9, 0, 50_000, records=False, threads=8)
+            ref_agg = oracle.aggregate(y)
+            for occ, bps in ((0, 0), (1, 0), (2, 0), (-1, 3)):
+                ctx.set_option(G.OPT_OCCUPANCY, occ)
+                ctx.set_option(G.OPT_BLOCKS_PER_SM, bps)
+                try:
+                    agg = ctx.estimate(m, 50_000, 9)
+                finally:
+                    ctx.set_option(G.OPT_OCCUPANCY, -1)
+                    ctx.set_option(G.OPT_BLOCKS_PER_SM, 0)
+                _agg_close(agg, ref_agg, G)
     ctx.load_graph_obj(g)
     ctx.load_query_obj(q)
     assert all(r in (8, 16, 24, 32) for r in ctx.query_info()["refill_min"])
