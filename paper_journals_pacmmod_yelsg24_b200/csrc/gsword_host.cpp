@@ -1161,7 +1161,7 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
         // the query exactly as given plus every option that changes the kernels' schedule
         const int opts[] = {n_qv, ctx->opt_blocks_per_sm, ctx->opt_threads, ctx->opt_chunk, ctx->opt_l2,
                             ctx->opt_coop, ctx->opt_bloom, ctx->opt_eset, ctx->opt_filter, ctx->opt_streaming,
-                            ctx->opt_variant};
+                            ctx->opt_variant, ctx->opt_occ};
         tkey.append(reinterpret_cast<const char*>(opts), sizeof(opts));
         tkey.append(reinterpret_cast<const char*>(q_row_ptr), sizeof(int32_t) * (size_t)(n_qv + 1));
         tkey.append(reinterpret_cast<const char*>(q_col), sizeof(int32_t) * (size_t)q_row_ptr[n_qv]);
