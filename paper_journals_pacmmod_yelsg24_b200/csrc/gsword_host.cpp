@@ -352,7 +352,8 @@ bool plan_is_tree(const Plan& p) {
 
 int launch_config(gsword_ctx* ctx, int method, int mode, LaunchCfg* cfg) {
     size_t smem = 0;
-    const int rows = ctx->query_loaded ? std::max(1, ctx->plan.nq) : GSWORD_MAX_QV;
+    const int rows = gsword::sample_smem_rows(method, ctx->query_loaded ? std::max(1, ctx->plan.nq) : GSWORD_MAX_QV,
+                                              ctx->opt_coop);
     const int occ = gsword::max_blocks_per_sm(method, mode, ctx->opt_threads, rows, &smem);
     if (occ <= 0) return fail(GSWORD_ECUDA, "kernel does not fit on the device (threads=%d)", ctx->opt_threads);
     const int bps = ctx->opt_blocks_per_sm > 0 ? std::min(ctx->opt_blocks_per_sm, occ) : occ;
@@ -1263,7 +1264,8 @@ int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out) {
         }
         if (m == GSWORD_ALLEY && ctx->opt_streaming) mode |= gsword::kModeStream;
         if (ctx->opt_sched != 0) mode |= gsword::kModeSync;
-        const int occ = gsword::max_blocks_per_sm(m, mode, ctx->opt_threads, std::max(1, ctx->plan.nq), nullptr);
+        const int occ = gsword::max_blocks_per_sm(
+            m, mode, ctx->opt_threads, gsword::sample_smem_rows(m, std::max(1, ctx->plan.nq), ctx->opt_coop), nullptr);
         out->occupancy[m] = ctx->opt_blocks_per_sm > 0 ? std::min(ctx->opt_blocks_per_sm, occ) : occ;
     }
     return GSWORD_OK;

@@ -342,11 +342,13 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     __shared__ uint8_t eidx_s[kMaxQV][kMaxQV];
     __shared__ uint8_t uq_s[kMaxQV];
     __shared__ uint32_t pdup_s[kMaxQV];  // variant A5: post-draw DupCheck positions
-    // Alley task-pool results per lane: pool_s[0] = adjacent matched vertices (pool 1),
-    // pool_s[1..4] = refine-mask removals (pool 2, 128 bits)
-    __shared__ uint32_t pool_s[5][256];
-    __shared__ Partial warp_part[32];
-    extern __shared__ uint32_t Ms[];  // Ms[j * blockDim.x + tid] = M[j] of this lane
+    __shared__ Partial warp_part[8];
+    // dynamic shared memory, rows of blockDim.x words (sized on the host by the query and
+    // the coop threshold, so the rest of the SM's L1/shared array stays L1):
+    //   Ms[j * T + tid]          = M[j] of this lane, j < n_q
+    //   pool_s[w * T + tid]      (Alley) w = 0: task-pool results "matched vertex j lies in
+    //                            S_p" (pool 1); w = 1..ceil(coop/32): refine-mask removals
+    extern __shared__ uint32_t Ms[];
 
     const int tid = threadIdx.x;
     const int T = blockDim.x;
@@ -363,6 +365,8 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     __syncthreads();
 
     const int nq = plan_in.nq;
+    uint32_t* const pool_s = Ms + (size_t)nq * (size_t)T;
+    const uint32_t mask_words = (coop_threshold + 31u) >> 5;  // refine-mask rows (<= 4)
     const int sched = SYNC ? sched_arg : 0;
     bool multi_back = false;  // some position has |B(d)| >= 2 (Alley refine kinds 2/3 can occur)
     if (!TREE)
@@ -634,7 +638,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     const bool valid = t < total;
                     test(o, tt - __shfl_sync(kFull, excl, o), valid, ea, eb, tg, lb, soe);
                     if (valid && is_edge<MODE == kModeCount>(g, ea, eb, lb, sectors) == soe)
-                        atomicOr(&pool_s[0][0] + (tg >> 5), 1u << (tg & 31u));
+                        atomicOr(pool_s + (tg >> 5), 1u << (tg & 31u));
                 }
                 __syncwarp();
             };
@@ -645,7 +649,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 const int j = fns_small(omask, k);
                 ea = Ms[op * T + ocol];
                 eb = Ms[j * T + ocol];
-                tg = ((uint32_t)ocol << 5) | (uint32_t)j;  // pool_s[0][ocol], bit j
+                tg = ((uint32_t)ocol << 5) | (uint32_t)j;  // pool_s row 0, lane ocol, bit j
                 soe = true;
             };
             // task of a kind-2 owner: is S_p[i] (label l_d) in N_l(M[j]), i.e. is {M[j], S_p[i]}
@@ -661,13 +665,14 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 const int j = fns_small(omask, nth);
                 ea = Ms[j * T + ocol];
                 eb = (uint32_t)ldg_i32(g.clist + olo + i);
-                tg = ((uint32_t)((1u + (i >> 5)) * 256u + (uint32_t)ocol) << 5) | (i & 31u);
+                tg = ((uint32_t)((1u + (i >> 5)) * (uint32_t)T + (uint32_t)ocol) << 5) | (i & 31u);
                 soe = false;
             };
             int kind = 0;
             uint32_t unk = 0, known = 0, others = 0;
 #pragma unroll
-            for (int w = 0; w < 5; ++w) pool_s[w][tid] = 0u;
+            for (int w = 0; w < 5; ++w)
+                if (METHOD == GSWORD_ALLEY && (uint32_t)w <= mask_words) pool_s[w * T + tid] = 0u;
             if (has && deferred) {
                 // M[j] (same label) with (phi[j], phi[p]) a query edge lies in S_p by the
                 // Alley invariant (every drawn prefix is a partial instance); M[p] never does
@@ -774,7 +779,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
 #endif
             mark(4);
             if (kind == 1) {
-                const uint32_t in_sp = known | pool_s[0][tid];  // matched vertices inside S_p
+                const uint32_t in_sp = known | pool_s[tid];  // matched vertices inside S_p
                 cnt = len_p - __popc(in_sp);
                 if (cnt > 0) {
                     const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
@@ -823,7 +828,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 for (int w = 0; w < 4; ++w) {
                     const uint32_t n_w = (len_p > 32u * w) ? min(len_p - 32u * w, 32u) : 0u;
                     uint32_t m = (n_w == 32u) ? 0xFFFFFFFFu : ((1u << n_w) - 1u);
-                    m &= ~pool_s[1 + w][tid];
+                    if (n_w) m &= ~pool_s[(1 + w) * T + tid];
                     uint32_t mm = dup ? m : 0u;
                     while (mm) {
                         const int i = __ffs(mm) - 1;
@@ -1848,7 +1853,7 @@ const void* select_kernel(int method, int mode) {
 int occ_blocks(int method, int occ_variant) { return kOccBlocks(method, occ_variant); }
 
 int max_blocks_per_sm(int method, int mode, int threads, int ms_rows, size_t* smem_bytes) {
-    const size_t smem = (size_t)ms_rows * (size_t)threads * sizeof(uint32_t);
+    const size_t smem = (size_t)ms_rows * (size_t)threads * sizeof(uint32_t);  // rows: sample_smem_rows
     if (smem_bytes) *smem_bytes = smem;
     int blocks = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, select_kernel(method, mode), threads, smem) !=
@@ -1863,8 +1868,9 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
                           cudaStream_t stream) {
     cudaError_t e = cudaMemsetAsync(d_queue, 0, sizeof(unsigned long long), stream);
     if (e != cudaSuccess) return e;
-    // Ms[j * threads + tid] for j < n_q only: sizing it by the query leaves the rest of the
-    // 256 KB L1/shared array to the L1 cache (spill slots, hot CSR entries)
+    // rows of the dynamic array (sample_smem_rows): sizing it by the query and the coop
+    // threshold leaves the rest of the 256 KB L1/shared array to the L1 cache (spill slots,
+    // hot CSR entries; measured: Alley is L1-capacity sensitive)
     const size_t smem = (size_t)cfg.ms_rows * (size_t)cfg.threads * sizeof(uint32_t);
     const uint32_t thr = (uint32_t)cfg.coop_threshold;
     void* args[] = {(void*)&g,      (void*)&plan,  (void*)&first,   (void*)&count,     (void*)&seed,

@@ -125,7 +125,7 @@ struct LaunchCfg {
     int coop_threshold;
     int sched;  // 0 refill, 1 sample synchronisation, 2 + inheritance (NEXT-3)
     uint32_t refill_min;  // sched 0: refill when at least this many lanes are free (1..32)
-    int ms_rows;          // rows of the per-lane matched-vertex array in shared memory (n_q)
+    int ms_rows;          // rows of the dynamic shared array (sample_smem_rows)
 };
 
 // Applies the GSWORD_OPT_VARIANT bits to a copy of the loaded plan (readings A3, A5).
@@ -196,7 +196,13 @@ cudaError_t launch_build_eset(const int64_t* d_row_ptr, const int32_t* col, int6
                               uint64_t mask, cudaStream_t stream);
 cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* bloom,
                                uint64_t mask, cudaStream_t stream);
-// ms_rows = query vertices (rows of the dynamic shared-memory matched-vertex array)
+// Rows of blockDim.x words of the sampling kernel's dynamic shared memory: n_q rows of
+// matched vertices, plus for Alley the task-pool result row and ceil(coop/32) refine-mask
+// rows.
+inline int sample_smem_rows(int method, int nq, int coop_threshold) {
+    return nq + (method == GSWORD_ALLEY ? 1 + (coop_threshold + 31) / 32 : 0);
+}
+// ms_rows = sample_smem_rows(...)
 int max_blocks_per_sm(int method, int mode, int threads, int ms_rows, size_t* smem_bytes);
 // minimum resident CTAs per SM the sampling kernel is compiled for (launch bounds)
 int occ_blocks(int method, int occ_variant);
