@@ -282,6 +282,15 @@ def run_ours(args):
 
     # algorithmic sectors per launch (counting build, untimed), SURVEY §8(d)
     sectors = {m: ctx.count_sectors(m, first, cnt, args.seed) for m in methods}
+    # sample statistics over the first 1e6 sample ids: depth reached, valid
+    # fraction (per-sample trace records, untimed)
+    depth_stats = {}
+    for m in methods:
+        rec = ctx.trace_samples(m, first, min(cnt, 1_000_000), args.seed)
+        dr = rec["depth_reached"].astype(np.float64)
+        depth_stats[m] = {"samples": int(rec.shape[0]), "mean_depth_reached": float(dr.mean()),
+                          "p99_depth_reached": float(np.percentile(dr, 99)),
+                          "valid_fraction": float(rec["valid"].mean())}
 
     if world > 1:
         dist.barrier()
@@ -405,7 +414,8 @@ def run_ours(args):
                                  "estimate": results[m]["estimate"], "std_err": results[m]["variance"] ** 0.5
                                  if results[m]["variance"] > 0 else 0.0,
                                  "valid_fraction": results[m]["n_valid"] / results[m]["n"],
-                                 "alg_sectors_per_sample": sectors[m] / cnt} for m in methods},
+                                 "alg_sectors_per_sample": sectors[m] / cnt,
+                                 "first_1e6": depth_stats[m]} for m in methods},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "kernel": f"sample_kernel<{name[dom]}>",
                      "peak_kind": peak_kind,
