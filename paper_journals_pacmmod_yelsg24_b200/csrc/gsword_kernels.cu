@@ -870,6 +870,11 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 const int colL = wbase + L;
                 const uint32_t Lsig = __shfl_sync(kFull, msig, L);
                 uint32_t total = 0, my_bal = 0;
+                // lists longer than 32 chunks: lane g also counts the survivors of chunk group
+                // g (G consecutive chunks), so the draw re-tests one group, not the whole prefix
+                const uint32_t G = (((Llen + 31u) >> 5) + 31u) >> 5;  // chunks per group
+                const uint32_t g_lo = (uint32_t)lane * G;
+                uint32_t gcnt = 0;
                 if (OCC == 1 && GSWORD_COOP_WIDE) {
                     // register-rich build: two chunks per round, both tests in one chain
                     for (uint32_t base = 0; base < Llen; base += 64) {
@@ -883,6 +888,8 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                         const unsigned bal0 = __ballot_sync(kFull, k0), bal1 = __ballot_sync(kFull, k1);
                         if ((base >> 5) == (uint32_t)lane) my_bal = bal0;
                         if ((base >> 5) + 1u == (uint32_t)lane) my_bal = bal1;
+                        if ((base >> 5) - g_lo < G) gcnt += __popc(bal0);
+                        if ((base >> 5) + 1u - g_lo < G) gcnt += __popc(bal1);
                         total += __popc(bal0) + __popc(bal1);
                     }
                 } else {
@@ -899,6 +906,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     }
                     const unsigned bal = __ballot_sync(kFull, keep);
                     if ((base >> 5) == (uint32_t)lane) my_bal = bal;
+                    if ((base >> 5) - g_lo < G) gcnt += __popc(bal);
                     total += __popc(bal);
                 }
                 }
@@ -923,8 +931,19 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                         if (lane == c) val = ldg_i32(g.clist + Llo + (uint32_t)c * 32u + fns32(my_bal, k - excl));
                         chosen = __shfl_sync(kFull, val, c);
                     } else {
-                        uint32_t run = 0;
-                        for (uint32_t base = 0; base < Llen; base += 32) {
+                        // the group holding the k-th survivor (warp scan of the group counts),
+                        // then its chunks re-tested in order
+                        uint32_t incl = gcnt;
+#pragma unroll
+                        for (int o = 1; o < 32; o <<= 1) {
+                            const uint32_t y = __shfl_up_sync(kFull, incl, o);
+                            if (lane >= o) incl += y;
+                        }
+                        const unsigned hm = __ballot_sync(kFull, (k >= incl - gcnt) && (k < incl));
+                        const int gs = __ffs(hm) - 1;
+                        uint32_t run = __shfl_sync(kFull, incl - gcnt, gs);
+                        const uint32_t b0 = (uint32_t)gs * G * 32u;
+                        for (uint32_t base = b0; base < Llen; base += 32) {
                             const uint32_t i = base + lane;
                             bool keep = i < Llen;
                             int32_t x = 0;
