@@ -100,27 +100,6 @@ __device__ __forceinline__ bool in_run(const int32_t* __restrict__ col, uint32_t
     return f;
 }
 
-// Up to 4 keys searched in lock step over the same run (independent loads in flight;
-// the first probes coincide and hit L1).  Bit t of the result: key t is present.
-__device__ __forceinline__ uint32_t has4(const int32_t* __restrict__ col, uint32_t lo, uint32_t n, int nk,
-                                         int32_t x0, int32_t x1, int32_t x2, int32_t x3) {
-    if (n == 0) return 0u;
-    uint32_t b0 = lo, b1 = lo, b2 = lo, b3 = lo;
-    while (n > 1) {
-        const uint32_t half = n >> 1;
-        b0 = (ldg_i32(col + b0 + half) <= x0) ? b0 + half : b0;
-        if (nk > 1) b1 = (ldg_i32(col + b1 + half) <= x1) ? b1 + half : b1;
-        if (nk > 2) b2 = (ldg_i32(col + b2 + half) <= x2) ? b2 + half : b2;
-        if (nk > 3) b3 = (ldg_i32(col + b3 + half) <= x3) ? b3 + half : b3;
-        n -= half;
-    }
-    uint32_t r = (ldg_i32(col + b0) == x0) ? 1u : 0u;
-    if (nk > 1 && ldg_i32(col + b1) == x1) r |= 2u;
-    if (nk > 2 && ldg_i32(col + b2) == x2) r |= 4u;
-    if (nk > 3 && ldg_i32(col + b3) == x3) r |= 8u;
-    return r;
-}
-
 // position of the k-th (0-based) set bit of m (k < popc(m))
 __device__ __forceinline__ uint32_t fns32(uint32_t m, uint32_t k) {
     uint32_t pos = 0, c;
@@ -136,12 +115,6 @@ __device__ __forceinline__ uint32_t fns32(uint32_t m, uint32_t k) {
 __device__ __forceinline__ int fns_small(uint32_t m, uint32_t k) {
     while (k--) m &= m - 1;
     return __ffs(m) - 1;
-}
-
-__device__ __forceinline__ uint32_t fns64(uint64_t m, uint32_t k) {
-    const uint32_t lo = (uint32_t)m;
-    const uint32_t c = __popc(lo);
-    return k < c ? fns32(lo, k) : 32u + fns32((uint32_t)(m >> 32), k - c);
 }
 
 // algorithmic sectors of a binary search over a sorted run of `len` 4-byte ids
