@@ -297,7 +297,10 @@ int gsword_estimate_until(gsword_ctx* ctx, gsword_method m, uint64_t seed, doubl
                           uint64_t max_samples, gsword_result* out);
 
 /* Same for the sample-id range [first_sample_id, first_sample_id + n_samples): the
- * multi-GPU split and checkpoint/resume unit (sample ids are global). */
+ * multi-GPU split and checkpoint/resume unit (sample ids are global).
+ * The exclusive end first_sample_id + n_samples must fit in u64 (so the largest usable id
+ * is 2^64 - 2); a wrapping range is EINVAL here and in every other range-taking call
+ * (async, trace, trawl, count_sectors). */
 int gsword_estimate_range(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples,
                           uint64_t seed, gsword_result* out);
 

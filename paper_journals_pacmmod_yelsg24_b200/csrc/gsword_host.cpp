@@ -397,6 +397,7 @@ DeviceGraph device_graph(const gsword_ctx* ctx) {
 
 int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, uint64_t seed, double* d_out4,
         gsword_sample_record* d_records, double* d_sectors) {
+    if (first + count < first) return fail(GSWORD_EINVAL, "sample-id range [first, first + n) overflows u64");
     if (ctx->q_filter) mode |= gsword::kModeCG;
     if (method == GSWORD_ALLEY && ctx->opt_streaming && (mode & 3) != gsword::kModeCount) mode |= gsword::kModeStream;
     if (ctx->opt_sched != 0) mode |= gsword::kModeSync;
@@ -1379,6 +1380,7 @@ int gsword_trace_samples(gsword_ctx* ctx, gsword_method m, uint64_t first, uint6
 namespace {
 int run_trawl(gsword_ctx* ctx, int m, uint64_t first, uint64_t n, uint64_t seed, uint64_t budget,
               gsword_trawl_record* d_rec, double* h4, double* h_timeout) {
+    if (first + n < first) return fail(GSWORD_EINVAL, "trawl: sample-id range [first, first + n) overflows u64");
     const int grid = ctx->num_sms * 8;
     if (grid > ctx->partial_cap) {
         if (ctx->d_partials) cudaFree(ctx->d_partials);

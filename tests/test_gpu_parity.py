@@ -173,6 +173,46 @@ def test_edge_cases(ctx, G):
     _parity(ctx, G, gen.complete_graph(20), gen.clique_query(16), G.WJ, seed=2, first=0, count=2000)
 
 
+def test_degenerate_inputs(ctx, G):
+    """Empty and boundary inputs (SURVEY §8(b) conventions): an edgeless graph, isolated
+    vertices next to a component, n_samples = 0 and 1, a range ending at 2^64 - 1 and
+    one that overflows."""
+    # edgeless graph: every sample dies at depth 1; the single-vertex query is still exact
+    g0 = gen.make_graph(40, [], [], gen.uniform_labels(40, 2, seed=3), 2, name="edgeless")
+    q = gen.query_from_edges(2, [(0, 1)], labels=[0, 1], order=[0, 1])
+    for m in (0, 1):
+        rec = _parity(ctx, G, g0, q, m, seed=4, first=0, count=300)
+        assert not rec["valid"].any()
+        r = ctx.estimate(m, 300, seed=4)
+        assert r["estimate"] == 0.0 and r["n_valid"] == 0 and r["n"] == 300
+    # isolated vertices around a triangle (seed candidates that die at once)
+    n = 64
+    g1 = gen.make_graph(n, [0, 1, 2], [1, 2, 0], None, 1, name="triangle+isolated")
+    for m in (0, 1):
+        _parity(ctx, G, g1, gen.cycle_query(3), m, seed=8, first=17, count=4000)
+    # n_samples = 0 is an error for the aggregates, a no-op for traces
+    ctx.load_graph_obj(g1)
+    ctx.load_query_obj(gen.cycle_query(3))
+    for m in (0, 1):
+        with pytest.raises(G.GswordError) as e:
+            ctx.estimate(m, 0, seed=1)
+        assert e.value.status == -1
+        assert ctx.trace_samples(m, 0, 0, seed=1).shape == (0,)
+    # one sample: variance undefined
+    r = ctx.estimate(1, 1, seed=1)
+    assert r["n"] == 1 and math.isnan(r["variance"])
+    # the last ids of the u64 space (exclusive end 2^64 - 1), and ranges that would wrap
+    top = 2**64 - 1001
+    _parity(ctx, G, g1, gen.cycle_query(3), 0, seed=3, first=top, count=1000, loaded=True)
+    for call in (lambda: ctx.estimate(0, 1001, seed=3, first=top),
+                 lambda: ctx.trace_samples(1, top, 1001, seed=3),
+                 lambda: ctx.trawl(0, 1001, seed=3, first=top),
+                 lambda: ctx.trace_trawl(1, top, 1001, seed=3)):
+        with pytest.raises(G.GswordError) as e:
+            call()
+        assert e.value.status == -1
+
+
 def test_errors(G):
     c = G.Context(0)
     with pytest.raises(G.GswordError) as e:
