@@ -67,8 +67,37 @@ class ClockSampler:
         self.rows = []
         self._stop = threading.Event()
         self._t = None
+        self.source = None
+
+    def _run_nvml(self) -> bool:
+        """NVML (nvidia_ml_py) reads take ~1 ms, so the region gets a sample every ~20 ms."""
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            get_reasons = getattr(pynvml, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+                pynvml.nvmlDeviceGetCurrentClocksThrottleReasons
+            mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            return False
+        # NVML reason bits: sw_power_cap 0x4, hw_slowdown 0x8, sw_thermal 0x20, hw_thermal 0x40
+        bits = (0x8, 0x40, 0x20, 0x4)
+        while not self._stop.is_set():
+            try:
+                sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+                r = int(get_reasons(h))
+                self.rows.append([str(self.index), str(sm), str(mx), "", hex(r)] +
+                                 ["Active" if r & b else "Not Active" for b in bits])
+            except Exception:
+                pass
+            self._stop.wait(0.02)
+        self.source = "nvml"
+        return True
 
     def _run(self):
+        if self._run_nvml():
+            return
+        self.source = "nvidia-smi"
         while not self._stop.is_set():
             try:
                 out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
@@ -101,7 +130,7 @@ class ClockSampler:
                 if len(r) > 5 + i and r[5 + i].lower().startswith("active"):
                     reasons.add(nme)
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(self.rows)}
+                "reasons": sorted(reasons), "samples": len(self.rows), "source": self.source}
 
 
 def measured_peaks():
