@@ -1,0 +1,29 @@
+"""Host logic of bench.py that runs without a GPU: the clock/throttle summary that decides
+whether a bench line is kept (B200_PROFILING.md clocks rule)."""
+import bench
+
+
+def _row(sm, mx, hw=False, hw_th=False, sw_th=False, pcap=False):
+    act = lambda b: "Active" if b else "Not Active"
+    return ["0", str(sm), str(mx), "", "0x0", act(hw), act(hw_th), act(sw_th), act(pcap)]
+
+
+def test_clock_summary_median_max_and_reasons():
+    c = bench.ClockSampler(0)
+    c.rows = [_row(1965, 1965), _row(1800, 1965, pcap=True), _row(1950, 1965), _row(1500, 1965, hw_th=True)]
+    c.source = "nvml"
+    s = c.summary()
+    assert s["sm_mhz"] == (1800 + 1950) / 2
+    assert s["sm_max_mhz"] == 1965
+    assert s["reasons"] == ["hw_thermal_slowdown", "sw_power_cap"]
+    assert s["samples"] == 4 and s["source"] == "nvml"
+
+
+def test_clock_summary_nvidia_smi_rows_and_empty():
+    c = bench.ClockSampler(0)
+    # nvidia-smi csv row: index, sm, max, power, active mask, then the four reason columns
+    c.rows = [["0", "1965", "1965", "650.1", "0x0000000000000000", "Not Active", "Not Active",
+               "Active", "Not Active"]]
+    assert c.summary()["reasons"] == ["sw_thermal_slowdown"]
+    empty = bench.ClockSampler(0).summary()
+    assert empty["samples"] == 0 and empty["sm_mhz"] is None
