@@ -79,6 +79,10 @@ typedef struct {
  *   csize[d] |C_d|, the size of the candidate set drawn from at depth d (0 if unused)
  *   depth_reached: last depth at which a candidate set was formed (nq-1 if complete)
  *   valid    1 iff the sample is a complete instance of q
+ *   sectors  algorithmic 32-byte sectors the sample needs under the model of reading A26
+ *            (DESIGN.md §3): list offsets, drawn/selected vertices, Alley
+ *            driver scans, one sector per membership question; 0 for Alley by warp
+ *            streaming (not modelled)
  *   weight   running fp64 product prod_{d <= depth_reached} csize[d] in depth order (A7);
  *            Y = weight if valid else 0.
  * A WanderJoin vertex drawn and then rejected by Validate is recorded (valid = 0);
@@ -87,7 +91,8 @@ typedef struct {
     uint64_t sample_id;
     uint8_t valid;
     uint8_t depth_reached;
-    uint8_t pad[6];
+    uint8_t pad[2];
+    uint32_t sectors;
     int32_t path[GSWORD_MAX_QV];
     uint32_t csize[GSWORD_MAX_QV];
     double weight;
@@ -205,7 +210,10 @@ int gsword_destroy(gsword_ctx* ctx);
 
 /* Issue all later device work on `cuda_stream` (a cudaStream_t, e.g.
  * torch.cuda.Stream.cuda_stream; NULL = the context's own non-blocking stream; the
- * legacy default stream is cudaStreamLegacy, (void*)0x1).  Borrowed, not destroyed. */
+ * legacy default stream is cudaStreamLegacy, (void*)0x1).  Borrowed, not destroyed.
+ * Ordering: work issued after the switch starts only after all work the context issued
+ * on the previous stream (an event on the old stream, waited on by the new one), so
+ * switching never races the context's reused queue / partial / output buffers. */
 int gsword_set_stream(gsword_ctx* ctx, void* cuda_stream);
 
 /* Set a tunable (gsword_option).  Errors: EINVAL for an unknown option or value. */
@@ -335,11 +343,17 @@ int gsword_finalize(const double* host4, gsword_result* out);
 int gsword_trace_samples(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples,
                          uint64_t seed, gsword_sample_record* host_out);
 
-/* Measurement entry: run [first, first+n) in the counting build of
- * the kernel and return the ALGORITHMIC 32-byte sectors the method must touch,
- * summed over the range (model in DESIGN.md §6).  Synchronous. */
+/* Measurement entry: run [first, first+n) in the counting build of the
+ * kernel (the same refine/sample code as the estimate, plus counters) and return, summed
+ * over the range:
+ *   *sectors_out  the ALGORITHMIC 32-byte sectors of reading A26 (the per-sample `sectors`
+ *                 of gsword_sample_record; equal to the oracle's count, tests pin both)
+ *   *touched_out  (may be NULL) the sectors this implementation's accesses touch: edge-filter
+ *                 words, edge-set buckets (or binary-search probes), list offsets, driver
+ *                 chunks of the cooperative refine and re-tests, drawn elements
+ * Synchronous.  Ignores GSWORD_OPT_STREAMING. */
 int gsword_count_sectors(gsword_ctx* ctx, gsword_method m, uint64_t first_sample_id, uint64_t n_samples,
-                         uint64_t seed, double* sectors_out);
+                         uint64_t seed, double* sectors_out, double* touched_out);
 
 /* Profiling aid: warp-cycles per loop phase summed over all warps, recorded by the last
  * gsword_count_sectors run: [0] refill, [1] draw + GetMinCandidate, [2] WanderJoin step /

@@ -38,7 +38,8 @@ MAX_QV = 16
 
 # per-sample record: restated from the layout contract (152 bytes)
 RECORD_DTYPE = np.dtype([
-    ("sample_id", "<u8"), ("valid", "u1"), ("depth_reached", "u1"), ("pad", "u1", (6,)),
+    ("sample_id", "<u8"), ("valid", "u1"), ("depth_reached", "u1"), ("pad", "u1", (2,)),
+    ("sectors", "<u4"),
     ("path", "<i4", (MAX_QV,)), ("csize", "<u4", (MAX_QV,)), ("weight", "<f8"),
 ])
 assert RECORD_DTYPE.itemsize == 152

@@ -35,7 +35,8 @@ typedef struct {
     uint64_t sample_id;
     uint8_t valid;
     uint8_t depth_reached;
-    uint8_t pad[6];
+    uint8_t pad[2];
+    uint32_t sectors; /* algorithmic 32-byte sectors of the sample (reading A26, below) */
     int32_t path[OR_MAX_QV];
     uint32_t csize[OR_MAX_QV];
     double weight;
@@ -225,20 +226,48 @@ static int64_t stream_select(uint64_t seed, uint64_t sid, int d, const int32_t* 
     return (int64_t)cur_total;
 }
 
+/* ---- algorithmic sectors (SURVEY §8(d) measurement; reading A26 of DESIGN.md §3) -----
+ * The memory the method itself must read, in 32-byte sectors, counted for every position a
+ * sample starts alive (one local-candidate list = one contiguous ascending run of 4-byte ids
+ * whose start/end offsets sit in one 8-byte record; a membership question "x in C(u,u',v)?"
+ * costs ONE sector: one probe of an exact index, the minimum for a random question):
+ *   d = 0      1 sector to read the drawn seed from the stored list C(phi[0]); 0 when
+ *              C(phi[0]) is all of V (M[0] = k needs no memory) or empty.
+ *   d >= 1     |B(d)| sectors for the offsets of the local lists S_j (GetMinCandidate;
+ *              WanderJoin's first-parent variant reads only the parent's: 1).
+ *   WanderJoin +1 for the drawn vertex when |C_d| > 0; then, if it passes DupCheck (registers),
+ *              +1 per IsEdge question in ascending backward position up to the first "no".
+ *   Alley, |B(d)| = 1: if S_p is not empty, +1 per exclusion question "is M[j] in S_p?" for
+ *              every matched j != p with L_q(phi[j]) = L_q(phi[d]), except (label-only lists) when
+ *              (phi[j], phi[p]) is a query edge: then M[j] lies in S_p because the prefix is a
+ *              partial instance; +1 for the selected vertex when |C_d| > 0 (its index follows
+ *              from k and the excluded vertices; the list itself is not scanned).
+ *   Alley, |B(d)| >= 2 and |S_p| > 0: ceil(|S_p| / 8) sectors to scan the driver list S_p; for
+ *              each driver element that is not a matched vertex (registers), +1 per membership
+ *              question in the other lists in ascending backward position up to the first "no";
+ *              the selected vertex is already in registers (0).
+ *   Alley by warp streaming (OR_SELECT_STREAM): not modelled, the record holds 0.
+ * Post-draw DupChecks (variant A5) and the HT update cost nothing. */
+static uint32_t div_up8(int64_t len) { return (uint32_t)((len + 7) / 8); }
+
 /* One position d of a sample (method 0 = WanderJoin, 1 = Alley): forms C_d from the
  * matched prefix M[0..d-1], draws M[d] with r(sid, d), multiplies *W by |C_d| (the running
  * product of Eq. 1 in depth order, reading A7; *W starts as |C_0| at d = 0) and validates.
- * `flags`: OR_* above (0 = the default sampler).  Returns 1 if M[0..d] is still a valid
- * partial instance, 0 if the sample died here. */
-static int step_at(const or_graph* G, const or_query* Q, int method, int flags, uint64_t seed, uint64_t sid,
-                   int d, const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
-                   int32_t* M, double* W, or_record* rec) {
+ * `flags`: OR_* above (0 = the default sampler).  `filter` is the candidate filter (0 =
+ * label only); it only enters the sector count.  Returns 1 if M[0..d] is still a valid
+ * partial instance, 0 if the sample died here.  rec->sectors accumulates the model above. */
+static int step_at(const or_graph* G, const or_query* Q, int method, int flags, int filter, uint64_t seed,
+                   uint64_t sid, int d, const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S,
+                   int32_t* refine, int32_t* M, double* W, or_record* rec) {
+    uint32_t sec_unused = 0;
+    uint32_t* sec = rec ? &rec->sectors : &sec_unused;
     if (d == 0) {
         /* seed from the global candidate set C(phi[0]) */
         *W = (double)C0_len;
         if (C0_len == 0) return 0;
         uint64_t k = uniform_index(draw_r(seed, sid, 0), (uint64_t)C0_len);
         M[0] = C0[k];
+        if (C0_len != G->n) *sec += 1; /* A26: the seed list is read unless it is all of V */
         if (rec) { rec->path[0] = M[0]; rec->csize[0] = (uint32_t)C0_len; }
         return 1;
     }
@@ -256,6 +285,8 @@ static int step_at(const or_graph* G, const or_query* Q, int method, int flags, 
         if (len[b] < len[p]) p = b;
     }
     if (method == 0 && (flags & OR_WJ_PARENT_FIRST)) p = 0; /* variant: first backward position */
+    /* A26: the offsets of every local list GetMinCandidate compares (first-parent: one) */
+    *sec += (method == 0 && (flags & OR_WJ_PARENT_FIRST)) ? 1u : (uint32_t)nb;
     int64_t clen;
     const int32_t* cand = S[p];
     if (method == 0) {
@@ -267,6 +298,7 @@ static int step_at(const or_graph* G, const or_query* Q, int method, int flags, 
         uint64_t k = uniform_index(draw_r(seed, sid, (uint32_t)d), (uint64_t)clen);
         int32_t v = cand[k];
         M[d] = v;
+        *sec += 1; /* A26: the drawn vertex */
         if (rec) { rec->path[d] = v; rec->csize[d] = (uint32_t)clen; }
         /* Validate: DupCheck against all matched vertices, IsEdge for every other
          * matched query neighbour */
@@ -274,6 +306,7 @@ static int step_at(const or_graph* G, const or_query* Q, int method, int flags, 
             if (M[j] == v) return 0;
         for (int b = 0; b < nb; ++b) {
             if (b == p) continue;
+            *sec += 1; /* A26: one IsEdge question */
             if (!contains(S[b], len[b], v)) return 0;
         }
         return 1;
@@ -291,6 +324,29 @@ static int step_at(const or_graph* G, const or_query* Q, int method, int flags, 
             if (alley_keep(x, S, len, nb, p, M, d, !post)) refine[clen++] = x;
         }
         if (clen > 0) v = refine[uniform_index(draw_r(seed, sid, (uint32_t)d), (uint64_t)clen)];
+        /* A26: sectors of this refine + select */
+        if (nb == 1) {
+            if (!post && len[p] > 0) /* no question is needed about an empty S_p */
+                for (int j = 0; j < d; ++j) {
+                    if (j == B[p] || Q->label[Q->order[j]] != Q->label[u]) continue;
+                    if (filter == 0 && Q->adj[Q->order[j]][Q->order[B[p]]]) continue; /* M[j] in S_p */
+                    *sec += 1; /* exclusion question "is M[j] in S_p?" */
+                }
+            if (clen > 0) *sec += 1; /* the selected vertex */
+        } else if (len[p] > 0) {
+            *sec += div_up8(len[p]); /* driver scan */
+            for (int64_t i = 0; i < len[p]; ++i) {
+                int32_t x = cand[i];
+                int matched = 0;
+                for (int j = 0; j < d && !post; ++j) matched |= M[j] == x;
+                if (matched) continue;
+                for (int b = 0; b < nb; ++b) {
+                    if (b == p) continue;
+                    *sec += 1; /* membership question "is x in S_b?" */
+                    if (!contains(S[b], len[b], x)) break;
+                }
+            }
+        }
     }
     *W = *W * (double)clen;
     /* empty refined set: the sample stops */
@@ -306,7 +362,8 @@ static int step_at(const or_graph* G, const or_query* Q, int method, int flags, 
 /* Samples positions 0 .. stop-1 (stop = |V_q| for the plain estimator; the trawling
  * prefix length d otherwise).  Returns Y = W if all `stop` positions were matched, else 0;
  * M and W are left in *Mout / *Wout. */
-static double walk(const or_graph* G, const or_query* Q, int method, int flags, uint64_t seed, uint64_t sid, int stop,
+static double walk(const or_graph* G, const or_query* Q, int method, int flags, int filter, uint64_t seed,
+                   uint64_t sid, int stop,
                    const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
                    or_record* rec, int32_t* Mout, double* Wout) {
     int32_t M[OR_MAX_QV] = {0};
@@ -319,9 +376,10 @@ static double walk(const or_graph* G, const or_query* Q, int method, int flags, 
     }
     for (int d = 0; d < stop && valid; ++d) {
         depth_reached = d;
-        valid = step_at(G, Q, method, flags, seed, sid, d, C0, C0_len, inC, S, refine, M, &W, rec);
+        valid = step_at(G, Q, method, flags, filter, seed, sid, d, C0, C0_len, inC, S, refine, M, &W, rec);
     }
     if (rec) {
+        if (method == 1 && (flags & OR_SELECT_STREAM)) rec->sectors = 0; /* A26: not modelled */
         rec->valid = (uint8_t)valid;
         rec->depth_reached = (uint8_t)depth_reached;
         rec->weight = W;
@@ -331,10 +389,11 @@ static double walk(const or_graph* G, const or_query* Q, int method, int flags, 
     return valid ? W : 0.0;
 }
 
-static double one_sample(const or_graph* G, const or_query* Q, int method, int flags, uint64_t seed, uint64_t sid,
+static double one_sample(const or_graph* G, const or_query* Q, int method, int flags, int filter, uint64_t seed,
+                         uint64_t sid,
                          const int32_t* C0, int64_t C0_len, const uint8_t* inC, int32_t** S, int32_t* refine,
                          or_record* rec) {
-    return walk(G, Q, method, flags, seed, sid, Q->nq, C0, C0_len, inC, S, refine, rec, NULL, NULL);
+    return walk(G, Q, method, flags, filter, seed, sid, Q->nq, C0, C0_len, inC, S, refine, rec, NULL, NULL);
 }
 
 static int load_query(or_query* Q, int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col,
@@ -426,7 +485,7 @@ int or_sample_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, con
     for (int b = 0; b < OR_MAX_QV; ++b) S[b] = buf + (size_t)b * (size_t)(maxdeg + 1);
     int32_t* refine = buf + (size_t)OR_MAX_QV * (size_t)(maxdeg + 1);
     for (uint64_t i = 0; i < count; ++i) {
-        double y = one_sample(&G, &Q, method, flags, seed, first + i, C0, C0_len, inC, S, refine,
+        double y = one_sample(&G, &Q, method, flags, filter, seed, first + i, C0, C0_len, inC, S, refine,
                               rec_out ? &rec_out[i] : NULL);
         if (y_out) y_out[i] = y;
     }
@@ -610,7 +669,7 @@ int or_trawl_range(int64_t n, const int64_t* row_ptr, const int32_t* col, const 
         trawl_state st;
         memset(&st, 0, sizeof(st));
         double W = 0.0;
-        double y = walk(&G, &Q, method, 0, seed, sid, d, C0, C0_len, inC, S, refine, &r, st.M, &W);
+        double y = walk(&G, &Q, method, 0, filter, seed, sid, d, C0, C0_len, inC, S, refine, &r, st.M, &W);
         uint8_t status = 0;
         double t = 0.0;
         if (r.valid) {
@@ -707,7 +766,8 @@ int or_inherit_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, co
             int any = 0;
             for (int l = 0; l < L; ++l) {
                 if (!alive[l]) continue;
-                alive[l] = step_at(&G, &Q, method, flags, seed, first + g0 + (uint64_t)l, d, C0, C0_len, inC, S, refine,
+                alive[l] = step_at(&G, &Q, method, flags, filter, seed, first + g0 + (uint64_t)l, d, C0, C0_len, inC, S,
+                                   refine,
                                    M[l], &W[l], NULL);
                 any |= alive[l];
             }

@@ -192,6 +192,7 @@ struct gsword_ctx {
     cudaStream_t stream = nullptr;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;    // around a whole estimate
     cudaEvent_t evk0 = nullptr, evk1 = nullptr;  // around the last sampling-kernel launch
+    cudaEvent_t ev_switch = nullptr;             // orders a stream switch after the old stream's work
     // graph
     bool graph_loaded = false;
     int32_t* d_col = nullptr;
@@ -671,9 +672,10 @@ int gsword_create(int cuda_device, gsword_ctx** out) {
     if ((e = cudaStreamCreateWithFlags(&ctx->own_stream, cudaStreamNonBlocking)) != cudaSuccess ||
         (e = cudaEventCreate(&ctx->ev0)) != cudaSuccess || (e = cudaEventCreate(&ctx->ev1)) != cudaSuccess ||
         (e = cudaEventCreate(&ctx->evk0)) != cudaSuccess || (e = cudaEventCreate(&ctx->evk1)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&ctx->ev_switch, cudaEventDisableTiming)) != cudaSuccess ||
         (e = cudaMalloc(&ctx->d_queue, sizeof(unsigned long long))) != cudaSuccess ||
         (e = cudaMalloc(&ctx->d_out4, 4 * sizeof(double))) != cudaSuccess ||
-        (e = cudaMalloc(&ctx->d_sectors, sizeof(double))) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_sectors, 2 * sizeof(double))) != cudaSuccess ||
         (e = cudaMalloc(&ctx->d_phase, 8 * sizeof(unsigned long long))) != cudaSuccess) {
         gsword_destroy(ctx);
         return cuda_fail(e, "create");
@@ -697,6 +699,7 @@ int gsword_destroy(gsword_ctx* ctx) {
     if (ctx->ev1) cudaEventDestroy(ctx->ev1);
     if (ctx->evk0) cudaEventDestroy(ctx->evk0);
     if (ctx->evk1) cudaEventDestroy(ctx->evk1);
+    if (ctx->ev_switch) cudaEventDestroy(ctx->ev_switch);
     if (ctx->own_stream) cudaStreamDestroy(ctx->own_stream);
     delete ctx;
     return GSWORD_OK;
@@ -704,7 +707,15 @@ int gsword_destroy(gsword_ctx* ctx) {
 
 int gsword_set_stream(gsword_ctx* ctx, void* cuda_stream) {
     if (!ctx) return fail(GSWORD_EINVAL, "set_stream: NULL context");
-    ctx->stream = cuda_stream ? (cudaStream_t)cuda_stream : ctx->own_stream;
+    cudaStream_t next = cuda_stream ? (cudaStream_t)cuda_stream : ctx->own_stream;
+    if (next != ctx->stream) {
+        // every launch reuses the context's queue, partials and output buffers: work issued on
+        // the new stream must start after everything already issued on the old one
+        CUDA_TRY(cudaSetDevice(ctx->device));
+        CUDA_TRY(cudaEventRecord(ctx->ev_switch, ctx->stream));
+        CUDA_TRY(cudaStreamWaitEvent(next, ctx->ev_switch, 0));
+        ctx->stream = next;
+    }
     return apply_l2_window(ctx);
 }
 
@@ -940,22 +951,27 @@ int gsword_load_graph(gsword_ctx* ctx, int64_t n, const int64_t* row_ptr, const 
     ctx->hot_bytes = hot_bytes;
     ctx->d_bloom = reinterpret_cast<unsigned long long*>(ctx->d_hot);
     ctx->d_seg = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ctx->d_hot) + words * sizeof(unsigned long long));
-    if (nnz > 0) CUDA_TRY(cudaMemcpy(ctx->d_col, col_up, sizeof(int32_t) * (size_t)nnz, cudaMemcpyHostToDevice));
     if ((e = cudaMalloc(&ctx->d_vlabel, sizeof(int32_t) * (size_t)std::max<int64_t>(n, 1))) != cudaSuccess) {
         ctx->free_graph();
         return fail(GSWORD_ENOMEM, "load_graph: cudaMalloc(labels): %s", cudaGetErrorString(e));
     }
+    // every upload is ordered on the context stream (the builds and samplers run there too);
+    // the host staging vectors live until the synchronisation below
+    if (nnz > 0)
+        CUDA_TRY(cudaMemcpyAsync(ctx->d_col, col_up, sizeof(int32_t) * (size_t)nnz, cudaMemcpyHostToDevice, ctx->stream));
     if (labels && n > 0)
-        CUDA_TRY(cudaMemcpy(ctx->d_vlabel, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyHostToDevice));
+        CUDA_TRY(cudaMemcpyAsync(ctx->d_vlabel, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyHostToDevice, ctx->stream));
     else if (n > 0)
-        CUDA_TRY(cudaMemset(ctx->d_vlabel, 0, sizeof(int32_t) * (size_t)n));
-    CUDA_TRY(cudaMemcpy(ctx->d_seg, seg.data(), sizeof(uint32_t) * seg.size(), cudaMemcpyHostToDevice));
+        CUDA_TRY(cudaMemsetAsync(ctx->d_vlabel, 0, sizeof(int32_t) * (size_t)n, ctx->stream));
+    CUDA_TRY(cudaMemcpyAsync(ctx->d_seg, seg.data(), sizeof(uint32_t) * seg.size(), cudaMemcpyHostToDevice, ctx->stream));
     if (L > 1) {
-        if (n > 0) CUDA_TRY(cudaMemcpy(ctx->d_bucket, bucket.data(), sizeof(int32_t) * (size_t)n, cudaMemcpyHostToDevice));
+        if (n > 0)
+            CUDA_TRY(cudaMemcpyAsync(ctx->d_bucket, bucket.data(), sizeof(int32_t) * (size_t)n, cudaMemcpyHostToDevice,
+                                     ctx->stream));
     } else if (n > 0) {
         CUDA_TRY(gsword::launch_build_bucket_identity(ctx->d_bucket, n, ctx->stream));
-        CUDA_TRY(cudaStreamSynchronize(ctx->stream));
     }
+    CUDA_TRY(cudaStreamSynchronize(ctx->stream));
     // Bloom filter (allocated above) and exact edge set, both built on the device
     {
         // exact edge set: 4-key buckets, load factor <= 1/2
@@ -1002,8 +1018,9 @@ int gsword_load_graph_device(gsword_ctx* ctx, int64_t n, const int64_t* d_row_pt
     ctx->free_graph();
     cudaStream_t st = ctx->stream;
     int64_t h_rp[2] = {0, 0};
-    CUDA_TRY(cudaMemcpy(&h_rp[0], d_row_ptr, sizeof(int64_t), cudaMemcpyDeviceToHost));
-    CUDA_TRY(cudaMemcpy(&h_rp[1], d_row_ptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpyAsync(&h_rp[0], d_row_ptr, sizeof(int64_t), cudaMemcpyDeviceToHost, ctx->stream));
+    CUDA_TRY(cudaMemcpyAsync(&h_rp[1], d_row_ptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost, ctx->stream));
+    CUDA_TRY(cudaStreamSynchronize(ctx->stream));
     const int64_t nnz = h_rp[1];
     if (h_rp[0] != 0) return fail(GSWORD_EGRAPH, "load_graph_device: row_ptr[0] != 0");
     if (nnz < 0 || nnz >= ((int64_t)1 << 31) - 1) return fail(GSWORD_ELIMIT, "load_graph_device: 2|E| >= 2^31");
@@ -1431,7 +1448,8 @@ int gsword_trace_trawl(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_
     double h[4], to = 0.0;
     rc = run_trawl(ctx, (int)m, first, n_samples, seed, budget, d_rec, h, &to);
     if (rc == GSWORD_OK) {
-        e = cudaMemcpy(host_out, d_rec, bytes, cudaMemcpyDeviceToHost);
+        e = cudaMemcpyAsync(host_out, d_rec, bytes, cudaMemcpyDeviceToHost, ctx->stream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
         if (e != cudaSuccess) rc = cuda_fail(e, "trace_trawl: copy back");
     }
     cudaFree(d_rec);
@@ -1439,18 +1457,21 @@ int gsword_trace_trawl(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_
 }
 
 int gsword_count_sectors(gsword_ctx* ctx, gsword_method m, uint64_t first, uint64_t n_samples, uint64_t seed,
-                         double* sectors_out) {
+                         double* sectors_out, double* touched_out) {
     int rc = ensure_ready(ctx, (int)m);
     if (rc) return rc;
     if (!sectors_out) return fail(GSWORD_EINVAL, "count_sectors: NULL output");
     if (n_samples == 0) return fail(GSWORD_EINVAL, "count_sectors: n_samples must be >= 1");
     rc = run(ctx, (int)m, gsword::kModeCount, first, n_samples, seed, ctx->d_out4, nullptr, ctx->d_sectors);
     if (rc) return rc;
-    CUDA_TRY(cudaMemcpyAsync(sectors_out, ctx->d_sectors, sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+    double h[2];  // [0] touched by this implementation, [1] algorithmic (reading A26)
+    CUDA_TRY(cudaMemcpyAsync(h, ctx->d_sectors, sizeof(h), cudaMemcpyDeviceToHost, ctx->stream));
     unsigned long long ph[8];
     CUDA_TRY(cudaMemcpyAsync(ph, ctx->d_phase, sizeof(ph), cudaMemcpyDeviceToHost, ctx->stream));
     CUDA_TRY(cudaStreamSynchronize(ctx->stream));
     for (int i = 0; i < 8; ++i) ctx->h_phase[i] = (double)ph[i];
+    *sectors_out = h[1];
+    if (touched_out) *touched_out = h[0];
     return GSWORD_OK;
 }
 

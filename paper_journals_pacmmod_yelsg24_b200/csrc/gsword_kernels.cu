@@ -39,12 +39,6 @@ constexpr unsigned kFull = 0xffffffffu;
 #ifndef GSWORD_SMEM_LANE
 #define GSWORD_SMEM_LANE 1  // sample id and running weight in shared memory
 #endif
-#ifndef GSWORD_COOP_WIDE
-#define GSWORD_COOP_WIDE 0  // 1: occupancy variant 1 runs two coop chunks per round (measured 0-7 % slower: spills)
-#endif
-#ifndef GSWORD_POOL_MERGED
-#define GSWORD_POOL_MERGED 1  // Alley exclusion and membership tests in one task pool
-#endif
 // Alley drivers longer than the coop threshold (<= 64) are refined by the whole warp.
 
 // ---------------------------------------------------------------- Philox4x32-10 (A6)
@@ -214,54 +208,6 @@ __device__ __forceinline__ bool member_all(const DeviceGraph& g, const uint32_t*
     return true;
 }
 
-// Two membership tests at once (x0, x1 each in every N_l(M[j]), j in `mask`): the filter
-// words of both, then the first edge-set buckets of both, are loaded before either is
-// used, so the two tests cost one dependent chain.  k0/k1 enter as "still a candidate".
-__device__ __forceinline__ bool eset_first(const DeviceGraph& g, unsigned long long key, uint64_t bk, bool& done) {
-    const ulonglong2* p = reinterpret_cast<const ulonglong2*>(g.eset + 4 * bk);
-    const ulonglong2 x0 = __ldg(p), x1 = __ldg(p + 1);
-    const bool hit = x0.x == key || x0.y == key || x1.x == key || x1.y == key;
-    done = hit || x0.x == kEmptyKey || x0.y == kEmptyKey || x1.x == kEmptyKey || x1.y == kEmptyKey;
-    return hit;
-}
-
-__device__ __forceinline__ void member_all2(const DeviceGraph& g, const uint32_t* Ms, int stride, int col_of,
-                                            uint32_t mask, int32_t l, int32_t x0, int32_t x1, bool& k0, bool& k1) {
-    double sec = 0.0;
-    if (!g.bloom || !g.eset) {
-        k0 = k0 && member_all<false>(g, Ms, stride, col_of, mask, l, x0, sec);
-        k1 = k1 && member_all<false>(g, Ms, stride, col_of, mask, l, x1, sec);
-        return;
-    }
-    while (mask && (k0 || k1)) {
-        const int j = __ffs(mask) - 1;
-        mask &= mask - 1;
-        const uint32_t a = Ms[j * stride + col_of];
-        const uint64_t h0 = edge_hash(a, (uint32_t)x0), h1 = edge_hash(a, (uint32_t)x1);
-        const unsigned long long w0 = k0 ? __ldg(g.bloom + (h0 & g.bloom_mask)) : 0ull;
-        const unsigned long long w1 = k1 ? __ldg(g.bloom + (h1 & g.bloom_mask)) : 0ull;
-        const uint64_t m0 = bloom_bits(h0), m1 = bloom_bits(h1);
-        k0 = k0 && (w0 & m0) == m0;
-        k1 = k1 && (w1 & m1) == m1;
-        if (!(k0 || k1)) return;
-        bool d0 = !k0, d1 = !k1, e0 = false, e1 = false;
-        uint64_t b0 = h0 & g.eset_mask, b1 = h1 & g.eset_mask;
-        const unsigned long long y0 = edge_key(a, (uint32_t)x0), y1 = edge_key(a, (uint32_t)x1);
-        if (k0) e0 = eset_first(g, y0, b0, d0);
-        if (k1) e1 = eset_first(g, y1, b1, d1);
-        while (!d0) {  // bucket overflow (rare): continue linear probing
-            b0 = (b0 + 1) & g.eset_mask;
-            e0 = eset_first(g, y0, b0, d0);
-        }
-        while (!d1) {
-            b1 = (b1 + 1) & g.eset_mask;
-            e1 = eset_first(g, y1, b1, d1);
-        }
-        k0 = k0 && e0;
-        k1 = k1 && e1;
-    }
-}
-
 // One-word signature of a lane's matched vertices: bit sig_bit(v) is set for every M[j].
 // A clear bit proves x is not matched, so the exact scan of M is skipped (~80 % of the
 // DupChecks of an 8-vertex query).
@@ -279,6 +225,28 @@ __device__ __forceinline__ bool not_matched(const uint32_t* Ms, int stride, int 
 __device__ __forceinline__ bool not_matched_sig(const uint32_t* Ms, int stride, int col_of, uint32_t dup, uint32_t sig,
                                                 int32_t x) {
     return !(sig & sig_bit(x)) || not_matched(Ms, stride, col_of, dup, x);
+}
+
+// Algorithmic sectors (reading A26) of an Alley refine with |B(d)| >= 2 over the driver run
+// clist[lo, lo + len): the driver scan, then for each driver element that is not a matched
+// vertex one membership question per other list in ascending position up to the first "no".
+// Trace / counting builds only (the estimate kernel never calls it).
+__device__ uint32_t model_refine_sectors(const DeviceGraph& g, const uint32_t* Ms, int T, int tid, uint32_t lo,
+                                         uint32_t len, uint32_t others, uint32_t dup, int32_t label) {
+    uint32_t s = (len + 7u) / 8u;
+    double unused = 0.0;
+    for (uint32_t i = 0; i < len; ++i) {
+        const int32_t x = ldg_i32(g.clist + lo + i);
+        if (!not_matched(Ms + tid, T, 0, dup, x)) continue;
+        uint32_t m = others;
+        while (m) {
+            const int j = __ffs(m) - 1;
+            m &= m - 1;
+            s += 1u;
+            if (!is_edge<false>(g, Ms[j * T + tid], (uint32_t)x, label, unused)) break;
+        }
+    }
+    return s;
 }
 
 #ifndef GSWORD_WJ_MIN_BLOCKS
@@ -389,7 +357,11 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
             nsum(s_sq, c_sq, __dmul_rn(y, y));
         }
     };
-    double sectors = 0.0;
+    double sectors = 0.0;  // counting build: sectors the implementation touches
+    // trace / counting builds: algorithmic sectors of reading A26 (this lane's sample, and
+    // the lane's total over its finished samples)
+    uint32_t msec = 0u;
+    double msum = 0.0;
 
     // warp chunk of the queue (warp-uniform)
     uint64_t q_next = 0, q_end = 0;
@@ -468,6 +440,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 d = 0;
                 W = 1.0;
                 msig = 0u;
+                msec = 0u;
                 if (MODE == kModeTrace) {
                     gsword_sample_record* rec = records + (sid - first);
                     rec->sample_id = sid;
@@ -511,6 +484,8 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 lo_p = plan_in.seed_lo;
                 len_p = plan_in.seed_len;
                 if (MODE == kModeCount) sectors += plan_in.seed_identity ? 0.0 : 1.0;
+                // A26: the drawn seed is read from the stored list unless C(phi[0]) is all of V
+                if (MODE != kModeEstimate && len_p != 0u && (int64_t)len_p != g.n) msec += 1u;
             } else if (METHOD == GSWORD_ALLEY && (TREE || ps.nback == 1)) {
                 // one backward neighbour: p is fixed by the plan; the segment load is left
                 // in flight and consumed after the exclusion tests (which need only M)
@@ -518,6 +493,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 local_run<CG>(g, eidx_s[d][p], Ms[p * T + tid], ps.label, &seg_a, &seg_b);
                 deferred = true;
                 if (MODE == kModeCount) sectors += 1.0;
+                if (MODE != kModeEstimate) msec += 1u;  // A26: offsets of S_p
             } else if (TREE) {
                 p = __ffs(ps.back) - 1;
                 uint32_t a, b;
@@ -542,6 +518,9 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     }
                 }
                 if (MODE == kModeCount) sectors += (METHOD == GSWORD_WJ && plan_in.wj_parent_first) ? 1.0 : (double)ps.nback;
+                // A26: the offsets of every list GetMinCandidate compares
+                if (MODE != kModeEstimate)
+                    msec += (METHOD == GSWORD_WJ && plan_in.wj_parent_first) ? 1u : (uint32_t)ps.nback;
             }
         }
 
@@ -559,13 +538,15 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     } else {
                         v = ldg_i32(g.clist + lo_p + k);
                         if (MODE == kModeCount) sectors += 1.0;
-                        // Validate: DupCheck, then IsEdge for the other matched neighbours.
-                        // v in N_l(M[j]) <=> M[j] in N_{L(phi[j])}(v): search the shorter run.
+                        if (MODE != kModeEstimate) msec += 1u;  // A26: the drawn vertex
+                        // Validate: DupCheck, then IsEdge for the other matched neighbours
+                        // (one edge-index question each, ascending position, first "no" ends it)
                         reject = !not_matched_sig(Ms + tid, T, 0, ps.dup, msig, v);
                         uint32_t bm = TREE ? 0u : ps.back & ~(1u << p);
                         while (bm && !reject) {
                             const int j = __ffs(bm) - 1;
                             bm &= bm - 1;
+                            if (MODE != kModeEstimate) msec += 1u;  // A26: one IsEdge question
                             reject = !is_edge<MODE == kModeCount>(g, Ms[j * T + tid], (uint32_t)v, ps.label, sectors);
                         }
                     }
@@ -643,6 +624,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
             };
             int kind = 0;
             uint32_t unk = 0, known = 0, others = 0;
+            uint32_t q_model = 0;  // A26: exclusion questions of a kind-1 step (trace / count)
 #pragma unroll
             for (int w = 0; w < 5; ++w)
                 if (METHOD == GSWORD_ALLEY && (uint32_t)w <= mask_words) pool_s[w * T + tid] = 0u;
@@ -653,6 +635,9 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 const uint32_t qa = qadj_s[p];
                 kind = 1;
                 uint32_t cdup = ps.dup & ~(1u << p);
+                // A26: one question per same-label matched M[j], j != p, except (label-only
+                // lists) those known to lie in S_p
+                if (MODE != kModeEstimate) q_model = (uint32_t)__popc(CG ? cdup : (cdup & ~qa));
                 if (CG) {
                     // under a filter S_p lies inside C(phi[d]): matched vertices outside it
                     // cannot be in S_p
@@ -668,7 +653,6 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 unk = cdup & ~qa;
             }
             __syncwarp();
-#if GSWORD_POOL_MERGED
             // kind 2 is known before the pool for lanes that waited on GetMinCandidate, so the
             // exclusion tests (kind 1) and the membership tests (kind 2) share one pool: one
             // pass of rounds instead of two
@@ -705,16 +689,6 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     if (valid) excl_task(wbase + o, omask, op, k, ea, eb, tg, soe);
                 });
             }
-#else
-            // pool 1: exclusion tests, overlapping the in-flight segment loads
-            pool((kind == 1) ? (uint32_t)__popc(unk) : 0u,
-                 [&](int o, uint32_t k, bool valid, uint32_t& ea, uint32_t& eb, uint32_t& tg, int32_t& lb, bool& soe) {
-                const uint32_t omask = __shfl_sync(kFull, unk, o);
-                const int op = __shfl_sync(kFull, p, o);
-                lb = __shfl_sync(kFull, ps.label, o);
-                if (valid) excl_task(wbase + o, omask, op, k, ea, eb, tg, soe);
-            });
-#endif
             if (deferred) {
                 lo_p = seg_a;
                 len_p = seg_b - seg_a;
@@ -729,28 +703,16 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 } else if (len_p == 0) {
                     kind = 0;
                 } else if (!TREE && !deferred) {
-                    if (len_p > coop_threshold) {
-                        kind = 3;
-                    } else if (!GSWORD_POOL_MERGED) {
-                        kind = 2;
-                        others = ps.back & ~(1u << p);
-                        if (MODE == kModeCount) sectors += (double)scan_sectors(len_p);
-                    }
+                    if (len_p > coop_threshold) kind = 3;
                 }
             }
             mark(3);
-#if !GSWORD_POOL_MERGED
-            // pool 2: membership tests of short refine masks
-            pool((kind == 2) ? len_p * (uint32_t)__popc(others) : 0u,
-                 [&](int o, uint32_t k, bool valid, uint32_t& ea, uint32_t& eb, uint32_t& tg, int32_t& lb, bool& soe) {
-                const uint32_t omask = __shfl_sync(kFull, others, o);
-                const uint32_t olo = __shfl_sync(kFull, lo_p, o);
-                const uint32_t olen = __shfl_sync(kFull, len_p, o);
-                lb = __shfl_sync(kFull, ps.label, o);
-                if (valid) memb_task(wbase + o, omask, olo, olen, k, ea, eb, tg, soe);
-            });
-#endif
             mark(4);
+            if (MODE != kModeEstimate && has && d > 0) {
+                if (kind == 1) msec += q_model + ((len_p > (uint32_t)__popc(known | pool_s[tid])) ? 1u : 0u);
+                if (!TREE && (kind == 2 || kind == 3))
+                    msec += model_refine_sectors(g, Ms, T, tid, lo_p, len_p, ps.back & ~(1u << p), ps.dup, ps.label);
+            }
             if (kind == 1) {
                 const uint32_t in_sp = known | pool_s[tid];  // matched vertices inside S_p
                 cnt = len_p - __popc(in_sp);
@@ -848,24 +810,6 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 const uint32_t G = (((Llen + 31u) >> 5) + 31u) >> 5;  // chunks per group
                 const uint32_t g_lo = (uint32_t)lane * G;
                 uint32_t gcnt = 0;
-                if (OCC == 1 && GSWORD_COOP_WIDE) {
-                    // register-rich build: two chunks per round, both tests in one chain
-                    for (uint32_t base = 0; base < Llen; base += 64) {
-                        const uint32_t i0 = base + lane, i1 = i0 + 32u;
-                        bool k0 = i0 < Llen, k1 = i1 < Llen;
-                        const int32_t x0 = k0 ? ldg_i32(g.clist + Llo + i0) : 0;
-                        const int32_t x1 = k1 ? ldg_i32(g.clist + Llo + i1) : 0;
-                        member_all2(g, Ms, T, colL, others, Lps.label, x0, x1, k0, k1);
-                        k0 = k0 && not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x0);
-                        k1 = k1 && not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x1);
-                        const unsigned bal0 = __ballot_sync(kFull, k0), bal1 = __ballot_sync(kFull, k1);
-                        if ((base >> 5) == (uint32_t)lane) my_bal = bal0;
-                        if ((base >> 5) + 1u == (uint32_t)lane) my_bal = bal1;
-                        if ((base >> 5) - g_lo < G) gcnt += __popc(bal0);
-                        if ((base >> 5) + 1u - g_lo < G) gcnt += __popc(bal1);
-                        total += __popc(bal0) + __popc(bal1);
-                    }
-                } else {
                 // the next chunk's driver elements are loaded while this chunk is tested
                 int32_t xn = ((uint32_t)lane < Llen) ? ldg_i32(g.clist + Llo + lane) : 0;
                 for (uint32_t base = 0; base < Llen; base += 32) {
@@ -881,7 +825,6 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     if ((base >> 5) == (uint32_t)lane) my_bal = bal;
                     if ((base >> 5) - g_lo < G) gcnt += __popc(bal);
                     total += __popc(bal);
-                }
                 }
                 int32_t chosen = -1;
                 if (total > 0) {
@@ -979,8 +922,10 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     gsword_sample_record* rec = records + (sid - first);
                     rec->valid = complete ? 1 : 0;
                     rec->depth_reached = (uint8_t)d;
+                    rec->sectors = msec;
                     rec->weight = W;
                 }
+                if (MODE == kModeCount) msum += (double)msec;
                 has = false;
             } else {
                 d += 1;
@@ -1045,10 +990,11 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
         n_valid += __shfl_xor_sync(kFull, n_valid, o);
         n_done += __shfl_xor_sync(kFull, n_done, o);
         sectors += shfl_xor_d(sectors, o);
+        msum += shfl_xor_d(msum, o);
     }
     const int warp = tid >> 5;
     if (lane == 0) {
-        warp_part[warp] = Partial{sh, sl, qh, ql, n_valid, n_done, sectors, 0.0};
+        warp_part[warp] = Partial{sh, sl, qh, ql, n_valid, n_done, sectors, msum};
     }
     __syncthreads();
     if (tid == 0) {
@@ -1060,6 +1006,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
             acc.valid += o.valid;
             acc.n += o.n;
             acc.sectors += o.sectors;
+            acc.model += o.model;
         }
         partials[blockIdx.x] = acc;
     }
@@ -1569,6 +1516,7 @@ __global__ void __launch_bounds__(128) trawl_kernel(const DeviceGraph g, const P
             acc.valid += o.valid;
             acc.n += o.n;
             acc.sectors += o.sectors;
+            acc.model += o.model;
         }
         partials[blockIdx.x] = acc;
     }
@@ -1578,7 +1526,7 @@ __global__ void __launch_bounds__(128) trawl_kernel(const DeviceGraph g, const P
 __global__ void reduce_kernel(const Partial* __restrict__ partials, int n, double* __restrict__ out4,
                               double* __restrict__ sectors_out) {
     const int lane = threadIdx.x;
-    double sh = 0, sl = 0, qh = 0, ql = 0, sec = 0;
+    double sh = 0, sl = 0, qh = 0, ql = 0, sec = 0, mod = 0;
     unsigned long long valid = 0, cnt = 0;
     for (int i = lane; i < n; i += 32) {
         const Partial p = partials[i];
@@ -1587,6 +1535,7 @@ __global__ void reduce_kernel(const Partial* __restrict__ partials, int n, doubl
         valid += p.valid;
         cnt += p.n;
         sec += p.sectors;
+        mod += p.model;
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
@@ -1597,13 +1546,17 @@ __global__ void reduce_kernel(const Partial* __restrict__ partials, int n, doubl
         valid += __shfl_xor_sync(kFull, valid, o);
         cnt += __shfl_xor_sync(kFull, cnt, o);
         sec += shfl_xor_d(sec, o);
+        mod += shfl_xor_d(mod, o);
     }
     if (lane == 0) {
         out4[0] = __dadd_rn(sh, sl);
         out4[1] = __dadd_rn(qh, ql);
         out4[2] = (double)valid;
         out4[3] = (double)cnt;
-        if (sectors_out) *sectors_out = sec;
+        if (sectors_out) {
+            sectors_out[0] = sec;  // touched sectors (trawl: timeouts)
+            sectors_out[1] = mod;  // algorithmic sectors (A26)
+        }
     }
 }
 
@@ -1842,6 +1795,20 @@ const void* select_kernel(int method, int mode) {
 
 }  // namespace
 
+// Grid of the grid-stride load-time kernels: `per_sm` CTAs on every SM of the current
+// device (multiProcessorCount, queried once per device).
+int sm_grid(int per_sm) {
+    static int cached[64] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 148 * per_sm;
+    if (cached[dev] == 0) {
+        int sms = 0;
+        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) sms = 148;
+        cached[dev] = sms;
+    }
+    return cached[dev] * per_sm;
+}
+
 int occ_blocks(int method, int occ_variant) { return kOccBlocks(method, occ_variant); }
 
 int max_blocks_per_sm(int method, int mode, int threads, int ms_rows, size_t* smem_bytes) {
@@ -1881,43 +1848,43 @@ cudaError_t launch_reduce(const Partial* d_partials, int n_partials, double* d_o
 
 cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* bloom,
                                uint64_t mask, cudaStream_t stream) {
-    bloom_kernel<<<148 * 8, 256, 0, stream>>>(d_row_ptr, col, n, bloom, mask);
+    bloom_kernel<<<sm_grid(8), 256, 0, stream>>>(d_row_ptr, col, n, bloom, mask);
     return cudaGetLastError();
 }
 
 cudaError_t launch_build_eset(const int64_t* d_row_ptr, const int32_t* col, int64_t n, unsigned long long* keys,
                               uint64_t mask, cudaStream_t stream) {
-    eset_kernel<<<148 * 8, 256, 0, stream>>>(d_row_ptr, col, n, keys, mask);
+    eset_kernel<<<sm_grid(8), 256, 0, stream>>>(d_row_ptr, col, n, keys, mask);
     return cudaGetLastError();
 }
 
 cudaError_t launch_filter(const DeviceGraph& g, const QFilter* d_qf, int nq, int filter, uint32_t* cbits,
                           const int32_t* d_vlabel, cudaStream_t stream) {
-    filter_kernel<<<148 * 4, 256, 0, stream>>>(g, d_qf, nq, filter, cbits, d_vlabel);
+    filter_kernel<<<sm_grid(4), 256, 0, stream>>>(g, d_qf, nq, filter, cbits, d_vlabel);
     return cudaGetLastError();
 }
 
 cudaError_t launch_cg_count(const DeviceGraph& g, const uint32_t* cbits, int u, int u2, int32_t label2,
                             uint32_t* counts, cudaStream_t stream) {
-    cg_count_kernel<<<148 * 8, 256, 0, stream>>>(g, cbits, u, u2, label2, counts);
+    cg_count_kernel<<<sm_grid(8), 256, 0, stream>>>(g, cbits, u, u2, label2, counts);
     return cudaGetLastError();
 }
 
 cudaError_t launch_cg_fill(const DeviceGraph& g, const uint32_t* cbits, int u, int u2, int32_t label2,
                            const uint32_t* off, int32_t* out, cudaStream_t stream) {
-    cg_fill_kernel<<<148 * 8, 256, 0, stream>>>(g, cbits, u, u2, label2, off, out);
+    cg_fill_kernel<<<sm_grid(8), 256, 0, stream>>>(g, cbits, u, u2, label2, off, out);
     return cudaGetLastError();
 }
 
 cudaError_t launch_bits_count(const uint32_t* cbits, uint32_t cwords, int u, int64_t n, uint32_t* counts,
                               cudaStream_t stream) {
-    bits_count_kernel<<<148 * 4, 256, 0, stream>>>(cbits, cwords, u, n, counts);
+    bits_count_kernel<<<sm_grid(4), 256, 0, stream>>>(cbits, cwords, u, n, counts);
     return cudaGetLastError();
 }
 
 cudaError_t launch_bits_fill(const uint32_t* cbits, uint32_t cwords, int u, int64_t n, const uint32_t* off,
                              int32_t* out, cudaStream_t stream) {
-    bits_fill_kernel<<<148 * 4, 256, 0, stream>>>(cbits, cwords, u, n, off, out);
+    bits_fill_kernel<<<sm_grid(4), 256, 0, stream>>>(cbits, cwords, u, n, off, out);
     return cudaGetLastError();
 }
 
@@ -2043,35 +2010,35 @@ __global__ void label_fill_kernel(const int32_t* __restrict__ labels, int64_t n,
 
 cudaError_t launch_dev_validate(const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int64_t n,
                                 int32_t n_labels, int* d_bad, cudaStream_t stream) {
-    dev_validate_kernel<<<148 * 8, 256, 0, stream>>>(row_ptr, col, labels, n, n_labels, d_bad);
+    dev_validate_kernel<<<sm_grid(8), 256, 0, stream>>>(row_ptr, col, labels, n, n_labels, d_bad);
     return cudaGetLastError();
 }
 
 cudaError_t launch_dev_seg(const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int64_t n, int32_t L,
                            uint32_t* seg, cudaStream_t stream) {
-    dev_seg_kernel<<<148 * 8, 256, 0, stream>>>(row_ptr, col, labels, n, L, seg);
+    dev_seg_kernel<<<sm_grid(8), 256, 0, stream>>>(row_ptr, col, labels, n, L, seg);
     return cudaGetLastError();
 }
 
 cudaError_t launch_label_hist(const int32_t* labels, int64_t n, unsigned long long* hist, cudaStream_t stream) {
-    label_hist_kernel<<<148 * 4, 256, 0, stream>>>(labels, n, hist);
+    label_hist_kernel<<<sm_grid(4), 256, 0, stream>>>(labels, n, hist);
     return cudaGetLastError();
 }
 
 cudaError_t launch_pair_hist(const int64_t* row_ptr, const int32_t* col, const int32_t* labels, int64_t n, int32_t L,
                              unsigned long long* hist, cudaStream_t stream) {
     const size_t smem = sizeof(unsigned long long) * (size_t)L * (size_t)L;
-    pair_hist_kernel<<<148 * 4, 256, smem, stream>>>(row_ptr, col, labels, n, L, hist);
+    pair_hist_kernel<<<sm_grid(4), 256, smem, stream>>>(row_ptr, col, labels, n, L, hist);
     return cudaGetLastError();
 }
 
 cudaError_t launch_label_bucket(const int32_t* labels, int64_t n, int32_t l, uint32_t* counts,
                                 const unsigned long long* d_base, uint32_t* d_tmp, unsigned long long* d_total,
                                 int32_t* bucket, cudaStream_t stream) {
-    label_count_kernel<<<148 * 4, 256, 0, stream>>>(labels, n, l, counts);
+    label_count_kernel<<<sm_grid(4), 256, 0, stream>>>(labels, n, l, counts);
     cudaError_t e = launch_scan(counts, n + 1, d_base, d_tmp, d_total, stream);
     if (e != cudaSuccess) return e;
-    label_fill_kernel<<<148 * 4, 256, 0, stream>>>(labels, n, l, counts, bucket);
+    label_fill_kernel<<<sm_grid(4), 256, 0, stream>>>(labels, n, l, counts, bucket);
     return cudaGetLastError();
 }
 
@@ -2107,7 +2074,7 @@ cudaError_t launch_gather(const uint32_t* buf, uint64_t words, int steps, int in
 }
 
 cudaError_t launch_build_bucket_identity(int32_t* bucket, int64_t n, cudaStream_t stream) {
-    iota_kernel<<<148 * 4, 256, 0, stream>>>(bucket, n);
+    iota_kernel<<<sm_grid(4), 256, 0, stream>>>(bucket, n);
     return cudaGetLastError();
 }
 

@@ -147,8 +147,8 @@ struct Partial {
     double sq_hi, sq_lo;        // double-double sum of Y*Y
     unsigned long long valid;   // complete instances
     unsigned long long n;       // samples
-    double sectors;             // algorithmic sectors (counting build only)
-    double pad;
+    double sectors;             // counting build: sectors the implementation touches (trawl: timeouts)
+    double model;               // counting build: algorithmic sectors of reading A26
 };
 
 // Kernel entry points (gsword_kernels.cu).  All enqueue on `stream`.

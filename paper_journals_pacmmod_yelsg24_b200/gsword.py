@@ -7,9 +7,8 @@ Names follow the C ABI one to one: gsword_load_graph -> Context.load_graph, etc.
 from __future__ import annotations
 
 import ctypes
-import math
 import os
-from typing import Dict, Optional
+from typing import Dict, Optional, Tuple
 
 import numpy as np
 
@@ -48,7 +47,8 @@ STATUS = {0: "OK", -1: "EINVAL", -2: "ENOGRAPH", -3: "ENOQUERY", -4: "EORDER", -
 
 # gsword_sample_record (152 bytes)
 RECORD_DTYPE = np.dtype([
-    ("sample_id", "<u8"), ("valid", "u1"), ("depth_reached", "u1"), ("pad", "u1", (6,)),
+    ("sample_id", "<u8"), ("valid", "u1"), ("depth_reached", "u1"), ("pad", "u1", (2,)),
+    ("sectors", "<u4"),
     ("path", "<i4", (MAX_QV,)), ("csize", "<u4", (MAX_QV,)), ("weight", "<f8"),
 ])
 assert RECORD_DTYPE.itemsize == 152
@@ -107,7 +107,7 @@ def _load_library() -> ctypes.CDLL:
                                   ctypes.c_int),
         "gsword_finalize": ([P, ctypes.POINTER(_Result)], ctypes.c_int),
         "gsword_trace_samples": ([P, ctypes.c_int, U64, U64, U64, P], ctypes.c_int),
-        "gsword_count_sectors": ([P, ctypes.c_int, U64, U64, U64, P], ctypes.c_int),
+        "gsword_count_sectors": ([P, ctypes.c_int, U64, U64, U64, P, P], ctypes.c_int),
         "gsword_launch_info": ([P, P, P, P], ctypes.c_int),
         "gsword_gather_roofline": ([P, U64, ctypes.c_int, P], ctypes.c_int),
         "gsword_last_kernel_seconds": ([P, P], ctypes.c_int),
@@ -368,15 +368,11 @@ class Context:
                                          _ptr(rec)))
         return rec
 
-    def count_sectors(self, method: int, first: int, n_samples: int, seed: int) -> float:
+    def count_sectors(self, method: int, first: int, n_samples: int, seed: int) -> Tuple[float, float]:
+        """(algorithmic sectors of reading A26, sectors this implementation touches) summed
+        over samples [first, first + n_samples)."""
         out = ctypes.c_double()
+        touched = ctypes.c_double()
         _check(_lib.gsword_count_sectors(self._h, int(method), int(first), int(n_samples), int(seed),
-                                         ctypes.byref(out)))
-        return out.value
-
-
-def variance_tolerance(agg: Dict[str, float], rel: float = 1e-12) -> float:
-    """Absolute tolerance for comparing variances: the subtraction sumsq - sum^2/n can
-    cancel, so the error bound scales with sumsq / (n (n-1))."""
-    n = agg["n"]
-    return rel * abs(agg["sumsq"]) / (n * (n - 1)) + 1e-300 if n >= 2 else math.inf
+                                         ctypes.byref(out), ctypes.byref(touched)))
+        return out.value, touched.value

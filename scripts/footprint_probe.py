@@ -39,7 +39,7 @@ with G.Context(0) as ctx:
                 torch.cuda.synchronize()
                 r = ctx.estimate(meth, N, 42)
                 ts.append(ctx.last_kernel_seconds())
-            sec = ctx.count_sectors(meth, 0, 1_000_000, 42) / 1_000_000
+            sec = ctx.count_sectors(meth, 0, 1_000_000, 42)[0] / 1_000_000
             t = min(ts)
             print(json.dumps({"opts": opts, "scale": s, "n": n, "m": m, "col_mb": 8 * m / 2**20, "method": meth, "kernel_ms": 1e3 * t,
                               "samples_per_s": N / t, "sectors_per_sample": sec, "valid_fraction": r["n_valid"] / N,

@@ -22,7 +22,7 @@ with G.Context(0) as ctx:
     for q in qs:
         ctx.load_query_obj(q)
         for m in (G.WJ, G.ALLEY):
-            sec = ctx.count_sectors(m, 0, int(args.samples), 42)
+            sec = ctx.count_sectors(m, 0, int(args.samples), 42)[0]
             ph = ctx.phase_cycles()
             tot = sum(ph)
             print(f"{q.name:14s} m={m} sectors/sample={sec / args.samples:7.2f} " +

@@ -393,12 +393,14 @@ def random_connected_query(nq: int, extra_edge_p: float, n_labels: int, seed: in
 
 
 def extract_query(g: Graph, k: int, seed: int, dense: bool, max_tries: int = 1000,
-                  require_dense: bool = False) -> Query:
+                  require_dense: bool = False, min_non_tree: int = 0) -> Query:
     """Random-walk query extraction.
 
     dense=True : random walk until k distinct vertices, query = induced subgraph;
                  with require_dense, walks are retried until the query's maximum
                  degree is >= 3 (the paper's dense/sparse split).
+                 min_non_tree retries until |E_q| - (k - 1) >= min_non_tree (cyclic
+                 queries, where Alley's intersections do real work).
     dense=False: self-avoiding walk of k vertices, query = the walk path
                  (max degree 2 < 3, "sparse" per P:L1055).
     Labels are copied from the data vertices, so the count is >= 1.
@@ -451,6 +453,8 @@ def extract_query(g: Graph, k: int, seed: int, dense: bool, max_tries: int = 100
                     degs[b] += 1
                 if degs.max() < 3:
                     continue
+            if len(edges) - (k - 1) < min_non_tree:
+                continue
         else:
             edges = tree_edges
         labels = g.labels[np.asarray(verts)]
@@ -474,9 +478,12 @@ def config_c0() -> Tuple[Graph, List[Query]]:
 
 
 def config_c1() -> Tuple[Graph, List[Query]]:
-    """C1: eu2005-shaped Chung-Lu (|V|=862,664, |E|=16,138,468), unlabelled, 8-vertex queries."""
+    """C1: eu2005-shaped Chung-Lu (|V|=862,664, |E|=16,138,468), unlabelled, 8-vertex queries:
+    sparse (a path), dense (the bench's headline query) and cyclic (>= 3 non-tree edges)."""
     g = chung_lu(862_664, 16_138_468, gamma=2.1, max_over_mean=68_963 / 37.4, seed=2005, name="C1_eu2005")
-    qs = [extract_query(g, 8, seed=20, dense=False), extract_query(g, 8, seed=21, dense=True, require_dense=True)]
+    qs = [extract_query(g, 8, seed=20, dense=False), extract_query(g, 8, seed=21, dense=True, require_dense=True),
+          # cyclic: >= 3 non-tree edges, so several positions intersect two or more lists
+          extract_query(g, 8, seed=22, dense=True, min_non_tree=3)._renamed("cyclic8_s22")]
     return g, qs
 
 
