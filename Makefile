@@ -18,7 +18,7 @@ $(LIB): $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_host.cpp $(CSRC)/internal.h inc
 	$(NVCC) $(NVFLAGS) -shared -o $@ $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_host.cpp 2> build_ptxas.log || (cat build_ptxas.log; false)
 
 $(ORACLE): oracle/oracle.c
-	gcc -O2 -std=c11 -Wall -Wextra -shared -fPIC -o $@ $<
+	gcc -O2 -std=c11 -Wall -Wextra -shared -fPIC -pthread -o $@ $<
 
 clean:
 	rm -f $(LIB) $(ORACLE) build_ptxas.log

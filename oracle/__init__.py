@@ -56,7 +56,7 @@ assert TRAWL_DTYPE.itemsize == 168
 def build(force: bool = False) -> str:
     """Compile oracle.c -> liboracle.so (gcc, plain -O2)."""
     if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-Wextra", "-shared", "-fPIC",
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-Wextra", "-shared", "-fPIC", "-pthread",
                                "-o", _SO, _SRC])
     return _SO
 
@@ -80,6 +80,8 @@ def _load():
             lib.or_sample_range_f.restype = ctypes.c_int
             lib.or_sample_range_v.argtypes = lib.or_sample_range_f.argtypes + [ctypes.c_int]
             lib.or_sample_range_v.restype = ctypes.c_int
+            lib.or_sample_range_mt.argtypes = lib.or_sample_range_v.argtypes + [ctypes.c_int, ctypes.c_uint64]
+            lib.or_sample_range_mt.restype = ctypes.c_int
             lib.or_candidate_sets.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, ctypes.c_int, P]
             lib.or_candidate_sets.restype = ctypes.c_int
             lib.or_trawl_range.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, P, P, P, ctypes.c_int,
@@ -169,23 +171,14 @@ def sample_range(g, q, method: int, seed: int, first: int, count: int, records: 
     y = np.zeros(count, np.float64)
     rec = np.zeros(count, RECORD_DTYPE) if records else None
 
-    def run(a: int, b: int) -> int:
-        yp = ctypes.c_void_p(y.ctypes.data + 8 * a)
-        rp = ctypes.c_void_p(rec.ctypes.data + RECORD_DTYPE.itemsize * a) if records else None
-        return lib.or_sample_range_v(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq,
-                                     _ptr(pr.qrp), _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order),
-                                     int(method), int(seed), int(first + a), int(b - a), yp, rp, int(filter),
-                                     int(select) | int(variant))
-
-    if threads <= 1 or count < 2 * threads:
-        rc = run(0, count) if count else 0
-    else:
-        # dynamic scheduling over chunks of sample ids
-        chunk = max(1, min(65536, count // (threads * 8) or 1))
-        bounds = [(a, min(count, a + chunk)) for a in range(0, count, chunk)]
-        with ThreadPoolExecutor(max_workers=threads) as ex:
-            rcs = list(ex.map(lambda ab: run(*ab), bounds))
-        rc = min(rcs) if rcs else 0
+    # dynamic scheduling over chunks of sample ids on `threads` host threads; the
+    # candidate sets are built once per call and shared by the threads
+    threads = max(1, int(threads))
+    chunk = max(1, min(1024, -(-count // (4 * threads)))) if threads > 1 else max(1, count)
+    rc = lib.or_sample_range_mt(pr.n, _ptr(pr.row_ptr), _ptr(pr.col), _ptr(pr.labels), pr.nq, _ptr(pr.qrp),
+                                _ptr(pr.qcol), _ptr(pr.qlab), _ptr(pr.order), int(method), int(seed), int(first),
+                                int(count), _ptr(y), _ptr(rec) if records else None, int(filter),
+                                int(select) | int(variant), threads, chunk) if count else 0
     if rc != 0:
         raise ValueError(f"oracle rejected input (rc={rc})")
     return y, rec

@@ -24,6 +24,8 @@
  * Every step is written in the paper's order with no blocking, fusion or
  * reordering.  Membership tests use the C library bsearch on ascending lists.
  */
+#include <pthread.h>
+#include <stdatomic.h>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -449,6 +451,11 @@ int or_sample_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, con
                       const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
                       double* y_out, or_record* rec_out, int filter, int flags);
 
+int or_sample_range_mt(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                       int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                       const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
+                       double* y_out, or_record* rec_out, int filter, int flags, int threads, uint64_t chunk);
+
 /* Run samples [first, first + count) with the candidate sets of `filter`. */
 int or_sample_range_f(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
                       int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
@@ -463,36 +470,100 @@ int or_sample_range_v(int64_t n, const int64_t* row_ptr, const int32_t* col, con
                       int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
                       const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
                       double* y_out, or_record* rec_out, int filter, int flags) {
-    or_graph G = {n, row_ptr, col, labels};
+    return or_sample_range_mt(n, row_ptr, col, labels, nq, q_row_ptr, q_col, q_labels, order, method, seed, first,
+                              count, y_out, rec_out, filter, flags, 1, count);
+}
+
+/* Shared, read-only state of one call: the graph, the query, the candidate sets of the
+ * filter and the seed list C(phi[0]) (built once per call), and the dynamic schedule. */
+typedef struct {
+    or_graph G;
     or_query Q;
-    int rc = load_query(&Q, nq, q_row_ptr, q_col, q_labels, order);
+    int method, flags, filter;
+    uint64_t seed, first, count, chunk;
+    const int32_t* C0;
+    int64_t C0_len;
+    const uint8_t* inC;
+    int64_t maxdeg;
+    double* y_out;
+    or_record* rec_out;
+    _Atomic uint64_t next;   /* next unclaimed offset in [0, count) */
+    _Atomic int failed;
+} range_job;
+
+/* One worker: claims chunks of sample ids in order of the shared counter (the dynamic
+ * scheduling of the paper's CPU baselines) and runs each sample plainly. */
+static void* range_worker(void* arg) {
+    range_job* J = (range_job*)arg;
+    int32_t* buf = (int32_t*)malloc(sizeof(int32_t) * (size_t)(J->maxdeg + 1) * (OR_MAX_QV + 1));
+    if (!buf) { J->failed = 1; return NULL; }
+    int32_t* S[OR_MAX_QV];
+    for (int b = 0; b < OR_MAX_QV; ++b) S[b] = buf + (size_t)b * (size_t)(J->maxdeg + 1);
+    int32_t* refine = buf + (size_t)OR_MAX_QV * (size_t)(J->maxdeg + 1);
+    for (;;) {
+        uint64_t a = atomic_fetch_add(&J->next, J->chunk);
+        if (a >= J->count) break;
+        uint64_t b = a + J->chunk < J->count ? a + J->chunk : J->count;
+        for (uint64_t i = a; i < b; ++i) {
+            double y = one_sample(&J->G, &J->Q, J->method, J->flags, J->filter, J->seed, J->first + i, J->C0,
+                                  J->C0_len, J->inC, S, refine, J->rec_out ? &J->rec_out[i] : NULL);
+            if (J->y_out) J->y_out[i] = y;
+        }
+    }
+    free(buf);
+    return NULL;
+}
+
+/* Run samples [first, first + count) on `threads` host threads, chunks of `chunk` ids. */
+int or_sample_range_mt(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* labels,
+                       int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col, const int32_t* q_labels,
+                       const int32_t* order, int method, uint64_t seed, uint64_t first, uint64_t count,
+                       double* y_out, or_record* rec_out, int filter, int flags, int threads, uint64_t chunk) {
+    range_job J;
+    memset(&J, 0, sizeof(J));
+    J.G = (or_graph){n, row_ptr, col, labels};
+    int rc = load_query(&J.Q, nq, q_row_ptr, q_col, q_labels, order);
     if (rc) return rc;
-    int64_t maxdeg = 0;
+    if (threads < 1) threads = 1;
+    if (threads > 256) threads = 256;
+    J.method = method;
+    J.flags = flags;
+    J.filter = filter;
+    J.seed = seed;
+    J.first = first;
+    J.count = count;
+    J.chunk = chunk > 0 ? chunk : 1;
+    J.y_out = y_out;
+    J.rec_out = rec_out;
+    atomic_init(&J.next, 0);
+    atomic_init(&J.failed, 0);
     for (int64_t v = 0; v < n; ++v)
-        if (row_ptr[v + 1] - row_ptr[v] > maxdeg) maxdeg = row_ptr[v + 1] - row_ptr[v];
+        if (row_ptr[v + 1] - row_ptr[v] > J.maxdeg) J.maxdeg = row_ptr[v + 1] - row_ptr[v];
     int32_t* C0 = (int32_t*)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
-    int32_t* buf = (int32_t*)malloc(sizeof(int32_t) * (size_t)(maxdeg + 1) * (OR_MAX_QV + 1));
-    if (!C0 || !buf) { free(C0); free(buf); return -1; }
     uint8_t* inC = (uint8_t*)malloc((size_t)(n > 0 ? n : 1) * (size_t)nq);
-    if (!inC) { free(C0); free(buf); return -1; }
-    candidate_sets(&G, &Q, filter, inC);
+    if (!C0 || !inC) { free(C0); free(inC); return -1; }
+    candidate_sets(&J.G, &J.Q, filter, inC);
     /* global candidate set of phi[0], ascending */
     int64_t C0_len = 0;
-    const uint8_t* in0 = inC + (int64_t)Q.order[0] * n;
+    const uint8_t* in0 = inC + (int64_t)J.Q.order[0] * n;
     for (int64_t v = 0; v < n; ++v)
         if (in0[v]) C0[C0_len++] = (int32_t)v;
-    int32_t* S[OR_MAX_QV];
-    for (int b = 0; b < OR_MAX_QV; ++b) S[b] = buf + (size_t)b * (size_t)(maxdeg + 1);
-    int32_t* refine = buf + (size_t)OR_MAX_QV * (size_t)(maxdeg + 1);
-    for (uint64_t i = 0; i < count; ++i) {
-        double y = one_sample(&G, &Q, method, flags, filter, seed, first + i, C0, C0_len, inC, S, refine,
-                              rec_out ? &rec_out[i] : NULL);
-        if (y_out) y_out[i] = y;
+    J.C0 = C0;
+    J.C0_len = C0_len;
+    J.inC = inC;
+    if (threads == 1) {
+        range_worker(&J);
+    } else {
+        pthread_t tid[256];
+        int started = 0;
+        for (; started < threads; ++started)
+            if (pthread_create(&tid[started], NULL, range_worker, &J) != 0) break;
+        if (started == 0) range_worker(&J);
+        for (int t = 0; t < started; ++t) pthread_join(tid[t], NULL);
     }
     free(inC);
     free(C0);
-    free(buf);
-    return 0;
+    return atomic_load(&J.failed) ? -1 : 0;
 }
 
 /* ---- exact count of embeddings by plain backtracking (reading A1) --------------- */

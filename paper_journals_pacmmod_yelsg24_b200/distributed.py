@@ -50,7 +50,7 @@ def estimate_distributed(ctx: Context, method: int, n_total: int, seed: int, fir
         out4.zero_()
     if cnt > 0:
         ctx.estimate_async(method, f, cnt, seed, out4)
-    if world > 1:
+    if dist.is_initialized():  # the combine runs whenever a group exists (a no-op sum at world 1)
         allreduce_sum4(out4, group)
     return finalize(out4.cpu().numpy())
 
@@ -96,10 +96,14 @@ def combine_host(values4_per_rank) -> Dict[str, float]:
     return finalize(acc)
 
 
-def init_from_env(backend: Optional[str] = None):
+def init_from_env(backend: Optional[str] = None, single_rank_group: bool = False):
     """torchrun plumbing: init the process group from RANK/WORLD_SIZE/MASTER_* and bind
-    LOCAL_RANK's GPU.  Returns (rank, world, local_rank)."""
+    LOCAL_RANK's GPU.  With single_rank_group, a 1-rank group is created at world size 1
+    too (MASTER_ADDR 127.0.0.1 and a free port unless set), so the combine step of the path
+    runs at every N; if that group cannot be created the caller proceeds without one.
+    Returns (rank, world, local_rank)."""
     import os
+    import socket
 
     import torch
     import torch.distributed as dist
@@ -107,14 +111,26 @@ def init_from_env(backend: Optional[str] = None):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1 and not dist.is_initialized():
-        if backend is None:
-            backend = "nccl" if torch.cuda.is_available() else "gloo"
+    if backend is None:
+        backend = "nccl" if torch.cuda.is_available() else "gloo"
+    if backend == "nccl" or torch.cuda.is_available():
+        torch.cuda.set_device(local)
+    if dist.is_initialized():
+        return rank, world, local
+    if world > 1:
         if backend == "nccl":
-            torch.cuda.set_device(local)
             dist.init_process_group(backend, device_id=torch.device("cuda", local))
         else:
             dist.init_process_group(backend)
-    elif torch.cuda.is_available():
-        torch.cuda.set_device(local)
+    elif single_rank_group:
+        if "MASTER_PORT" not in os.environ:
+            with socket.socket() as s:
+                s.bind(("127.0.0.1", 0))
+                os.environ["MASTER_PORT"] = str(s.getsockname()[1])
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        try:
+            kw = {"device_id": torch.device("cuda", local)} if backend == "nccl" else {}
+            dist.init_process_group(backend, rank=0, world_size=1, **kw)
+        except Exception:  # no group: the 4-vector needs no combining at world size 1
+            pass
     return rank, world, local

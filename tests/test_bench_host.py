@@ -26,4 +26,22 @@ def test_clock_summary_nvidia_smi_rows_and_empty():
                "Active", "Not Active"]]
     assert c.summary()["reasons"] == ["sw_thermal_slowdown"]
     empty = bench.ClockSampler(0).summary()
-    assert empty["samples"] == 0 and empty["sm_mhz"] is None
+    assert empty["samples"] == 0 and empty["sm_mhz"] is None and "source" in empty
+
+
+def test_clock_sampler_maps_the_device_by_uuid():
+    class FakeNvml:
+        def __init__(self):
+            self.calls = []
+
+        def nvmlDeviceGetHandleByUUID(self, u):
+            self.calls.append(("uuid", u))
+            return "h-uuid"
+
+        def nvmlDeviceGetHandleByIndex(self, i):
+            self.calls.append(("index", i))
+            return "h-index"
+
+    nv = FakeNvml()
+    c = bench.ClockSampler(3, uuid="GPU-1234", pci_bus_id="0000:1b:00.0")
+    assert c._nvml_handle(nv) == "h-uuid" and nv.calls == [("uuid", "GPU-1234")]

@@ -1,0 +1,126 @@
+"""The multi-GPU layer (north_star (4)) executed on the single-GPU lease.
+
+* Two processes share cuda:0, each runs the sampling + reduction kernels on its
+  rank_range slice of the sample ids (estimate_async), and the kernels' 4-vectors are
+  combined with one gloo all_reduce (NCCL refuses two ranks on one device).  The result
+  must equal a one-process run of the whole range: n and n_valid exactly, sum and sumsq
+  within 1e-12 (BASELINE.json north_star).
+* estimate_distributed under a 1-rank NCCL process group (init_from_env with
+  single_rank_group, as bench.py runs at N = 1): the NCCL all_reduce call site runs on the
+  launch stream and returns the single-range result.
+"""
+import os
+import socket
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+REL = 1e-12
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _slice_worker(rank, world, port, n_total, seed, qi, out_q):
+    import torch
+    import torch.distributed as dist
+
+    import paper_journals_pacmmod_yelsg24_b200 as G
+    from paper_journals_pacmmod_yelsg24_b200.distributed import allreduce_sum4, rank_range
+    from workloads import gen
+
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    g, qs = gen.config_c0()
+    res = []
+    with G.Context(0) as ctx:
+        stream = torch.cuda.Stream(0)
+        ctx.set_stream(stream)
+        ctx.load_graph_obj(g)
+        ctx.load_query_obj(qs[qi])
+        first, cnt = rank_range(n_total, rank, world)
+        for m in (G.WJ, G.ALLEY):
+            out = torch.zeros(4, dtype=torch.float64, device="cuda:0")
+            ctx.estimate_async(m, first, cnt, seed, out)
+            stream.synchronize()
+            t = out.cpu()
+            allreduce_sum4(t)  # the combine of the kernels' partials
+            res.append(t.tolist())
+    out_q.put((rank, res))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def _nccl_worker(n_total, seed, out_q):
+    import torch
+    import torch.distributed as dist
+
+    import paper_journals_pacmmod_yelsg24_b200 as G
+    from paper_journals_pacmmod_yelsg24_b200.distributed import estimate_distributed, init_from_env
+    from workloads import gen
+
+    for k in ("RANK", "WORLD_SIZE", "LOCAL_RANK", "MASTER_PORT"):
+        os.environ.pop(k, None)
+    init_from_env("nccl", single_rank_group=True)
+    backend = dist.get_backend() if dist.is_initialized() else None
+    g, qs = gen.config_c0()
+    res = []
+    with G.Context(0) as ctx:
+        torch.cuda.set_stream(torch.cuda.Stream(0))
+        ctx.load_graph_obj(g)
+        ctx.load_query_obj(qs[3])
+        for m in (G.WJ, G.ALLEY):
+            d = estimate_distributed(ctx, m, n_total, seed)
+            s = ctx.estimate(m, n_total, seed)
+            res.append((d, s))
+    out_q.put((backend, res))
+    if dist.is_initialized():
+        dist.destroy_process_group()
+
+
+def _spawn(target, args, n):
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=target, args=(*(a(r) if callable(a) else a for a in args), q)) for r in range(n)]
+    for p in procs:
+        p.start()
+    out = [q.get(timeout=600) for _ in range(n)]
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    return out
+
+
+def test_two_processes_share_the_gpu_and_combine_kernel_partials():
+    import paper_journals_pacmmod_yelsg24_b200 as G
+    from workloads import gen
+
+    world, n_total, seed, qi = 2, 3_000_001, 23, 2
+    port = _free_port()
+    out = _spawn(_slice_worker, (lambda r: r, world, port, n_total, seed, qi), world)
+    combined = {rank: res for rank, res in out}
+    assert combined[0] == combined[1]  # every rank holds the same combined vector
+    g, qs = gen.config_c0()
+    with G.Context(0) as ctx:
+        ctx.load_graph_obj(g)
+        ctx.load_query_obj(qs[qi])
+        for i, m in enumerate((G.WJ, G.ALLEY)):
+            full = ctx.estimate(m, n_total, seed)
+            s, sq, nv, n = combined[0][i]
+            assert n == n_total == full["n"] and nv == full["n_valid"]
+            assert s == pytest.approx(full["sum"], rel=REL, abs=0.0)
+            assert sq == pytest.approx(full["sumsq"], rel=REL, abs=0.0)
+
+
+def test_estimate_distributed_under_a_one_rank_nccl_group():
+    (backend, res), = _spawn(_nccl_worker, (2_000_000, 31), 1)
+    assert backend == "nccl"
+    for d, s in res:
+        assert d["n"] == s["n"] and d["n_valid"] == s["n_valid"]
+        assert d["sum"] == pytest.approx(s["sum"], rel=REL, abs=0.0)
+        assert d["sumsq"] == pytest.approx(s["sumsq"], rel=REL, abs=0.0)
