@@ -55,7 +55,10 @@ typedef enum {
     GSWORD_EGRAPH = -5,   /* CSR not canonical: unsorted/duplicate/self loop/asymmetric (A10, A11) */
     GSWORD_ELIMIT = -6,   /* nq > GSWORD_MAX_QV, or |V|, 2|E|, n_labels beyond 32-bit indexing */
     GSWORD_ECUDA = -7,    /* CUDA runtime error (including: no device) */
-    GSWORD_ENOMEM = -8    /* device or host allocation failed */
+    GSWORD_ENOMEM = -8,   /* device or host allocation failed */
+    GSWORD_EFAULT = -9    /* the kernels' sample accounting does not match the requested range
+                             (n != n_samples: a corrupted queue counter or partial); the result
+                             is discarded (SURVEY §5 failure detection) */
 } gsword_status;
 
 /* Aggregate of a sample range (Eq. 1; readings A8, A9).
@@ -194,6 +197,11 @@ typedef enum {
                                    /* the autotuned one; 0 default launch bounds, 1   */
                                    /* one CTA/SM less, 2 one more (forced; for A/B    */
                                    /* and sanitizer runs).  Results are unaffected    */
+    GSWORD_OPT_FAULT_QUEUE = 15,   /* fault injection (tests): the next sampling launch */
+                                   /* starts its sample queue at this value instead of */
+                                   /* 0, as a corrupted counter would (ids skipped);   */
+                                   /* one-shot; 0 = off.  Synchronous calls then fail  */
+                                   /* with GSWORD_EFAULT                               */
     GSWORD_OPT_FILTER = 7          /* candidate filter applied by the next            */
                                    /* gsword_load_query: 0 label only, 1 LDF, 2 NLF   */
                                    /* (1-2 build the candidate graph, reading A21)    */
@@ -291,8 +299,9 @@ int gsword_select_order(gsword_ctx* ctx, int strategy, gsword_method m, int32_t 
 
 /* Draw samples 0 .. n_samples-1 with `method` and `seed`, return the HT aggregate
  * (Eq. 1).  Synchronous (waits for the context stream).  Same as
- * gsword_estimate_range(ctx, m, 0, n_samples, seed, out).
- * Errors: ENOGRAPH, ENOQUERY, EINVAL (n_samples == 0, out NULL, bad method), ECUDA. */
+ * gsword_estimate_range(ctx, m, 0, n_samples, seed, out).  The kernels count every sample
+ * id they run; a count different from n_samples is reported as EFAULT.
+ * Errors: ENOGRAPH, ENOQUERY, EINVAL (n_samples == 0, out NULL, bad method), ECUDA, EFAULT. */
 int gsword_estimate(gsword_ctx* ctx, gsword_method m, uint64_t n_samples, uint64_t seed, gsword_result* out);
 
 /* Accuracy-targeted estimate: samples 0, 1, 2, ... in doubling batches (first batch

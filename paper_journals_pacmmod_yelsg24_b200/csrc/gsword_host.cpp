@@ -265,6 +265,7 @@ struct gsword_ctx {
     // (a serving loop re-issuing the same query) reuses them instead of re-running pilots
     int tuned_occ[2] = {0, 0};    // occupancy variant of the estimate kernel (kModeOccShift)
     int opt_occ = -1;             // GSWORD_OPT_OCCUPANCY: -1 autotuned, else forced
+    uint64_t opt_fault_queue = 0;  // GSWORD_OPT_FAULT_QUEUE: one-shot corrupted queue start
     struct Tuned {
         int refill[2], occ[2];
     };
@@ -298,6 +299,15 @@ struct gsword_ctx {
 };
 
 namespace {
+
+// Failure detection: the kernels count every sample id they ran; the total
+// must be the requested range size, else a queue counter or partial was corrupted.
+int check_accounting(const double* h4, uint64_t n_samples, const char* what) {
+    if ((uint64_t)h4[3] != n_samples || h4[2] > h4[3])
+        return fail(GSWORD_EFAULT, "%s: the kernels accounted for %.0f samples (%.0f valid) of %llu requested", what,
+                    h4[3], h4[2], (unsigned long long)n_samples);
+    return GSWORD_OK;
+}
 
 int ensure_ready(gsword_ctx* ctx, int method) {
     if (!ctx) return fail(GSWORD_EINVAL, "NULL context");
@@ -409,6 +419,8 @@ int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, u
     LaunchCfg cfg;
     int rc = launch_config(ctx, method, mode, &cfg);
     if (rc) return rc;
+    cfg.queue_start = ctx->opt_fault_queue;
+    ctx->opt_fault_queue = 0;
     CUDA_TRY(cudaEventRecord(ctx->evk0, ctx->stream));
     const bool counting = (mode & 3) == gsword::kModeCount;
     if (counting) CUDA_TRY(cudaMemsetAsync(ctx->d_phase, 0, 8 * sizeof(unsigned long long), ctx->stream));
@@ -775,6 +787,10 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
             if (value & ~(int64_t)(GSWORD_VARIANT_WJ_PARENT_FIRST | GSWORD_VARIANT_ALLEY_DUPCHECK_POST))
                 return fail(GSWORD_EINVAL, "unknown variant bits 0x%llx", (unsigned long long)value);
             ctx->opt_variant = (int)value;
+            return GSWORD_OK;
+        case GSWORD_OPT_FAULT_QUEUE:
+            if (value < 0) return fail(GSWORD_EINVAL, "fault queue start must be >= 0");
+            ctx->opt_fault_queue = (uint64_t)value;
             return GSWORD_OK;
         case GSWORD_OPT_COOP_THRESHOLD:
             if (value < 0 || value > 128) return fail(GSWORD_EINVAL, "coop threshold must be 0..128");
@@ -1324,6 +1340,8 @@ int gsword_estimate_range(gsword_ctx* ctx, gsword_method m, uint64_t first, uint
     double h[4];
     CUDA_TRY(cudaMemcpyAsync(h, ctx->d_out4, sizeof(h), cudaMemcpyDeviceToHost, ctx->stream));
     CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    rc = check_accounting(h, n_samples, "estimate");
+    if (rc) return rc;
     float ms = 0.f;
     CUDA_TRY(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
     gsword_finalize(h, out);
@@ -1386,9 +1404,12 @@ int gsword_trace_samples(gsword_ctx* ctx, gsword_method m, uint64_t first, uint6
     CUDA_TRY(cudaMemsetAsync(d_rec, 0, bytes, ctx->stream));
     rc = run(ctx, (int)m, gsword::kModeTrace, first, n_samples, seed, ctx->d_out4, d_rec, nullptr);
     if (rc == GSWORD_OK) {
+        double h4[4];
         e = cudaMemcpyAsync(host_out, d_rec, bytes, cudaMemcpyDeviceToHost, ctx->stream);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(h4, ctx->d_out4, sizeof(h4), cudaMemcpyDeviceToHost, ctx->stream);
         if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
         if (e != cudaSuccess) rc = cuda_fail(e, "trace: copy back");
+        else rc = check_accounting(h4, n_samples, "trace");
     }
     cudaFree(d_rec);
     return rc;
@@ -1468,7 +1489,11 @@ int gsword_count_sectors(gsword_ctx* ctx, gsword_method m, uint64_t first, uint6
     CUDA_TRY(cudaMemcpyAsync(h, ctx->d_sectors, sizeof(h), cudaMemcpyDeviceToHost, ctx->stream));
     unsigned long long ph[8];
     CUDA_TRY(cudaMemcpyAsync(ph, ctx->d_phase, sizeof(ph), cudaMemcpyDeviceToHost, ctx->stream));
+    double h4[4];
+    CUDA_TRY(cudaMemcpyAsync(h4, ctx->d_out4, sizeof(h4), cudaMemcpyDeviceToHost, ctx->stream));
     CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    rc = check_accounting(h4, n_samples, "count_sectors");
+    if (rc) return rc;
     for (int i = 0; i < 8; ++i) ctx->h_phase[i] = (double)ph[i];
     *sectors_out = h[1];
     if (touched_out) *touched_out = h[0];

@@ -1560,6 +1560,8 @@ __global__ void reduce_kernel(const Partial* __restrict__ partials, int n, doubl
     }
 }
 
+__global__ void set_u64_kernel(unsigned long long* p, unsigned long long v) { *p = v; }
+
 __global__ void iota_kernel(int32_t* out, int64_t n) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         out[i] = (int32_t)i;
@@ -1827,6 +1829,10 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
                           cudaStream_t stream) {
     cudaError_t e = cudaMemsetAsync(d_queue, 0, sizeof(unsigned long long), stream);
     if (e != cudaSuccess) return e;
+    if (cfg.queue_start) {  // fault injection: a corrupted queue counter
+        set_u64_kernel<<<1, 1, 0, stream>>>(d_queue, cfg.queue_start);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    }
     // rows of the dynamic array (sample_smem_rows): sizing it by the query and the coop
     // threshold leaves the rest of the 256 KB L1/shared array to the L1 cache (spill slots,
     // hot CSR entries; measured: Alley is L1-capacity sensitive)

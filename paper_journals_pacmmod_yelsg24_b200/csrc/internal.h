@@ -126,6 +126,7 @@ struct LaunchCfg {
     int sched;  // 0 refill, 1 sample synchronisation, 2 + inheritance (NEXT-3)
     uint32_t refill_min;  // sched 0: refill when at least this many lanes are free (1..32)
     int ms_rows;          // rows of the dynamic shared array (sample_smem_rows)
+    uint64_t queue_start = 0;  // initial sample-queue value (0; fault injection only)
 };
 
 // Applies the GSWORD_OPT_VARIANT bits to a copy of the loaded plan (readings A3, A5).

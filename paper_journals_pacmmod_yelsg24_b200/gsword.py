@@ -36,6 +36,7 @@ OPT_BLOOM_BITS = 11
 OPT_STREAMING = 12  # Alley by warp streaming (Alg. 3, reading A25)
 OPT_VARIANT = 13  # comparison variants of readings A3/A5 (bit flags below)
 OPT_OCCUPANCY = 14  # estimate-kernel occupancy variant: -1 autotuned, 0/1/2 forced
+OPT_FAULT_QUEUE = 15  # fault injection: the next launch's queue starts here (one-shot)
 VARIANT_WJ_PARENT_FIRST = 2
 VARIANT_ALLEY_DUPCHECK_POST = 4
 SCHED_REFILL, SCHED_SAMPLE_SYNC, SCHED_INHERIT = 0, 1, 2
@@ -43,7 +44,7 @@ FILTER_LABEL, FILTER_LDF, FILTER_NLF = 0, 1, 2
 CUDA_STREAM_LEGACY = 0x1  # cudaStreamLegacy
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOGRAPH", -3: "ENOQUERY", -4: "EORDER", -5: "EGRAPH",
-          -6: "ELIMIT", -7: "ECUDA", -8: "ENOMEM"}
+          -6: "ELIMIT", -7: "ECUDA", -8: "ENOMEM", -9: "EFAULT"}
 
 # gsword_sample_record (152 bytes)
 RECORD_DTYPE = np.dtype([

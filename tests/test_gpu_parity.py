@@ -625,3 +625,31 @@ def test_estimate_until(ctx, G, c0):
     assert full["sum"] == pytest.approx(r["sum"], rel=REL)
     with pytest.raises(G.GswordError):
         ctx.estimate_until(G.ALLEY, 5, rel_se=0.0)
+
+
+def test_fault_injection_queue_corruption_is_caught(ctx, G, c0):
+    """a corrupted sample-queue counter skips sample ids; the n / n_valid
+    accounting of the synchronous calls catches it (GSWORD_EFAULT) and the option is
+    one-shot, so the next call is clean."""
+    import torch
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    ctx.load_query_obj(qs[1])
+    n = 50_000
+    clean = ctx.estimate(G.ALLEY, n, seed=3)
+    for call in (lambda: ctx.estimate(G.ALLEY, n, seed=3),
+                 lambda: ctx.trace_samples(G.WJ, 0, n, 3),
+                 lambda: ctx.count_sectors(G.ALLEY, 0, n, 3)):
+        ctx.set_option(G.OPT_FAULT_QUEUE, 4096)
+        with pytest.raises(G.GswordError) as ei:
+            call()
+        assert ei.value.status == -9 and "accounted for 45904" in str(ei.value)
+    again = ctx.estimate(G.ALLEY, n, seed=3)
+    assert again["n"] == n and again["sum"] == clean["sum"] and again["n_valid"] == clean["n_valid"]
+    # the asynchronous form leaves the check to the caller: n in the 4-vector is short
+    out = torch.zeros(4, dtype=torch.float64, device="cuda:0")
+    ctx.set_stream(torch.cuda.current_stream())
+    ctx.set_option(G.OPT_FAULT_QUEUE, 10 * n)  # beyond the range: nothing runs
+    ctx.estimate_async(G.ALLEY, 0, n, 3, out)
+    assert out.cpu().tolist()[3] == 0.0
+    ctx.set_stream(None)
