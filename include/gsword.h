@@ -135,7 +135,10 @@ typedef struct {
 /* Statistics of the loaded query (gsword_query_info).
  *   candidates[u]  |C(u)| for query vertex u under the filter the query was loaded with
  *   cg_entries     total local-candidate entries of the candidate graph (0 for filter 0)
- *   build_seconds  device time of the candidate-graph build (0 for filter 0) */
+ *   build_seconds  device time of the candidate-graph build (0 for filter 0)
+ *   cg_bytes       device bytes of the candidate graph in the three-CSR format of Fig. 4
+ *                  (P:L770-L776): C(u) bitmaps + rank directories, |C(u)| + 1 offsets per
+ *                  directed query edge, the local lists and the seed list (0 for filter 0) */
 typedef struct {
     int32_t nq;
     int32_t filter;
@@ -146,6 +149,7 @@ typedef struct {
     int32_t occupancy[2];  /* resident CTAs per SM of the estimate kernel in use   */
                            /* per method (after autotune; GSWORD_OPT_BLOCKS_PER_SM */
                            /* may lower it further)                               */
+    uint64_t cg_bytes;
 } gsword_query_stats;
 
 /* Tunables for gsword_set_option (defaults chosen by measurement). */

@@ -218,6 +218,9 @@ struct gsword_ctx {
     int opt_filter = 0;
     int q_filter = 0;                 // filter the loaded query was built with
     uint32_t* d_cbits = nullptr;
+    uint32_t* d_crank = nullptr;   // rank directory of d_cbits (Fig. 4, 2nd CSR)
+    uint2* d_cg_edge = nullptr;    // per directed query edge: {offset base, source u}
+    uint64_t cg_bytes = 0;         // device bytes of the candidate graph
     uint32_t* d_cg_off = nullptr;
     int32_t* d_clist = nullptr;
     int32_t* d_cand0 = nullptr;
@@ -228,10 +231,15 @@ struct gsword_ctx {
 
     void free_query() {
         if (d_cbits) cudaFree(d_cbits);
+        if (d_crank) cudaFree(d_crank);
+        if (d_cg_edge) cudaFree(d_cg_edge);
         if (d_cg_off) cudaFree(d_cg_off);
         if (d_clist) cudaFree(d_clist);
         if (d_cand0) cudaFree(d_cand0);
         d_cbits = nullptr;
+        d_crank = nullptr;
+        d_cg_edge = nullptr;
+        cg_bytes = 0;
         d_cg_off = nullptr;
         d_clist = nullptr;
         d_cand0 = nullptr;
@@ -395,6 +403,8 @@ DeviceGraph device_graph(const gsword_ctx* ctx) {
     g.clist = ctx->q_filter ? ctx->d_clist : ctx->d_col;
     g.cg_off = ctx->q_filter ? ctx->d_cg_off : nullptr;
     g.cbits = ctx->q_filter ? ctx->d_cbits : nullptr;
+    g.crank = ctx->q_filter ? ctx->d_crank : nullptr;
+    g.cg_edge = ctx->q_filter ? ctx->d_cg_edge : nullptr;
     g.cwords = ctx->cwords;
     g.bloom = ctx->opt_bloom ? ctx->d_bloom : nullptr;
     g.bloom_mask = ctx->bloom_words ? ctx->bloom_words - 1 : 0;
@@ -521,9 +531,11 @@ void label_pair_freq(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
     }
 }
 
-// Candidate graph of the query (NEXT-1; Def. 4-5, Fig. 4):
-// C(u) by the filter, then one CSR per directed query edge a -> b with rows
-// C(a, b, v) = N(v) ∩ C(b), and the ascending list of C(phi[0]) for the seed.
+// Candidate graph of the query (NEXT-1; Def. 4-5) in the three-CSR format of
+// Fig. 4 (DeviceGraph in internal.h): C(u) by the filter as a bitmap + rank
+// directory per query vertex, then per directed query edge a -> b the |C(a)| + 1 offsets
+// of the local lists C(a, b, v) = N(v) ∩ C(b) (v in C(a), ascending), chained across the
+// edges into one list array, and the ascending list of C(phi[0]) for the seed.
 int build_candidate_graph(gsword_ctx* ctx, int32_t nq, const int32_t* q_row_ptr, const int32_t* q_col,
                           const int32_t* q_labels, const int32_t* order, Plan* p) {
     cudaStream_t st = ctx->stream;
@@ -553,35 +565,34 @@ int build_candidate_graph(gsword_ctx* ctx, int32_t nq, const int32_t* q_row_ptr,
             qf[u].pcount[k] += 1;
         }
     }
+    // 1st CSR: the directed query edges in (a, b) order (the plan's eidx)
     int eid[GSWORD_MAX_QV][GSWORD_MAX_QV];
     int ne = 0;
     for (int a = 0; a < nq; ++a)
         for (int b = 0; b < nq; ++b) eid[a][b] = adj[a][b] ? ne++ : -1;
     ctx->cwords = (uint32_t)((n + 31) / 32) + 1;
-    const size_t row = (size_t)n + 1;
+    const size_t bits_words = (size_t)nq * ctx->cwords;
     gsword::QFilter* d_qf = nullptr;
     uint32_t* d_tmp = nullptr;
     unsigned long long* d_tot = nullptr;
-    uint32_t* d_cnt0 = nullptr;
-    const size_t tmpw = gsword::scan_tmp_words((int64_t)row);
+    // scratch scans: a rank row (cwords) or an edge's offsets (<= n + 1 entries)
+    const size_t tmpw = gsword::scan_tmp_words(std::max<int64_t>((int64_t)ctx->cwords, n + 1));
     cudaError_t e;
-    if ((e = cudaMalloc(&ctx->d_cbits, sizeof(uint32_t) * (size_t)nq * ctx->cwords)) != cudaSuccess ||
-        (e = cudaMalloc(&ctx->d_cg_off, sizeof(uint32_t) * row * (size_t)std::max(ne, 1))) != cudaSuccess ||
+    if ((e = cudaMalloc(&ctx->d_cbits, sizeof(uint32_t) * bits_words)) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_crank, sizeof(uint32_t) * bits_words)) != cudaSuccess ||
+        (e = cudaMalloc(&ctx->d_cg_edge, sizeof(uint2) * (size_t)std::max(ne, 1))) != cudaSuccess ||
         (e = cudaMalloc(&d_qf, sizeof(qf))) != cudaSuccess ||
         (e = cudaMalloc(&d_tmp, sizeof(uint32_t) * tmpw)) != cudaSuccess ||
-        (e = cudaMalloc(&d_tot, sizeof(unsigned long long) * (size_t)(ne + 2))) != cudaSuccess ||
-        (e = cudaMalloc(&d_cnt0, sizeof(uint32_t) * row)) != cudaSuccess) {
+        (e = cudaMalloc(&d_tot, sizeof(unsigned long long) * (size_t)(ne + nq + 1))) != cudaSuccess) {
         cudaFree(d_qf);
         cudaFree(d_tmp);
         cudaFree(d_tot);
-        cudaFree(d_cnt0);
         return fail(GSWORD_ENOMEM, "load_query: candidate graph allocation: %s", cudaGetErrorString(e));
     }
     auto cleanup = [&]() {
         cudaFree(d_qf);
         cudaFree(d_tmp);
         cudaFree(d_tot);
-        cudaFree(d_cnt0);
         cudaEventDestroy(e0);
         cudaEventDestroy(e1);
     };
@@ -596,28 +607,54 @@ int build_candidate_graph(gsword_ctx* ctx, int32_t nq, const int32_t* q_row_ptr,
     ctx->q_filter = ctx->opt_filter;
     gsword::DeviceGraph g = device_graph(ctx);
     g.cbits = ctx->d_cbits;
+    g.crank = ctx->d_crank;
     g.cwords = ctx->cwords;
     CG_TRY(cudaMemcpyAsync(d_qf, qf, sizeof(qf), cudaMemcpyHostToDevice, st));
-    CG_TRY(cudaMemsetAsync(ctx->d_cbits, 0, sizeof(uint32_t) * (size_t)nq * ctx->cwords, st));
+    CG_TRY(cudaMemsetAsync(ctx->d_cbits, 0, sizeof(uint32_t) * bits_words, st));
     CG_TRY(gsword::launch_filter(g, d_qf, nq, ctx->q_filter, ctx->d_cbits, ctx->d_vlabel, st));
-    // seed list C(phi[0])
-    CG_TRY(gsword::launch_bits_count(ctx->d_cbits, ctx->cwords, order[0], n, d_cnt0, st));
-    CG_TRY(gsword::launch_scan(d_cnt0, (int64_t)row, nullptr, d_tmp, d_tot + ne + 1, st));
-    // per directed edge a -> b: counts, then offsets chained across edges
+    // 2nd CSR: rank directory per query vertex; d_tot[ne + u] = |C(u)|
+    for (int u = 0; u < nq; ++u) {
+        uint32_t* row = ctx->d_crank + (size_t)u * ctx->cwords;
+        CG_TRY(gsword::launch_rank_words(ctx->d_cbits, ctx->cwords, u, ctx->d_crank, st));
+        CG_TRY(gsword::launch_scan(row, (int64_t)ctx->cwords, nullptr, d_tmp, d_tot + ne + u, st));
+    }
+    unsigned long long csz[GSWORD_MAX_QV];
+    CG_TRY(cudaMemcpyAsync(csz, d_tot + ne, sizeof(unsigned long long) * (size_t)nq, cudaMemcpyDeviceToHost, st));
+    CG_TRY(cudaStreamSynchronize(st));
+    // 3rd CSR offsets: edge a -> b gets |C(a)| + 1 entries at base[e]
+    std::vector<uint2> edges((size_t)std::max(ne, 1));
+    uint64_t off_total = 0;
+    for (int a = 0; a < nq; ++a)
+        for (int b = 0; b < nq; ++b)
+            if (eid[a][b] >= 0) {
+                edges[(size_t)eid[a][b]] = make_uint2((uint32_t)off_total, (uint32_t)a);
+                off_total += csz[a] + 1;
+            }
+    if (off_total >= (1ull << 32)) {
+        cleanup();
+        return fail(GSWORD_ELIMIT, "load_query: candidate graph has %llu offsets (>= 2^32)",
+                    (unsigned long long)off_total);
+    }
+    if ((e = cudaMalloc(&ctx->d_cg_off, sizeof(uint32_t) * (size_t)std::max<uint64_t>(off_total, 1))) != cudaSuccess) {
+        cleanup();
+        return fail(GSWORD_ENOMEM, "load_query: candidate graph offsets: %s", cudaGetErrorString(e));
+    }
+    CG_TRY(cudaMemcpyAsync(ctx->d_cg_edge, edges.data(), sizeof(uint2) * edges.size(), cudaMemcpyHostToDevice, st));
+    CG_TRY(cudaMemsetAsync(ctx->d_cg_off, 0, sizeof(uint32_t) * (size_t)std::max<uint64_t>(off_total, 1), st));
     CG_TRY(cudaMemsetAsync(d_tot, 0, sizeof(unsigned long long), st));
     for (int a = 0; a < nq; ++a)
         for (int b = 0; b < nq; ++b) {
             const int ed = eid[a][b];
             if (ed < 0) continue;
-            uint32_t* off = ctx->d_cg_off + (size_t)ed * row;
-            CG_TRY(gsword::launch_cg_count(g, ctx->d_cbits, a, b, q_labels[b], off, st));
-            CG_TRY(gsword::launch_scan(off, (int64_t)row, d_tot + ed, d_tmp, d_tot + ed + 1, st));
+            uint32_t* off = ctx->d_cg_off + edges[(size_t)ed].x;
+            CG_TRY(gsword::launch_cg_count(g, a, b, q_labels[b], off, st));
+            // offsets chained across the edges: absolute positions in the list array
+            CG_TRY(gsword::launch_scan(off, (int64_t)csz[a] + 1, d_tot + ed, d_tmp, d_tot + ed + 1, st));
         }
-    unsigned long long tot[GSWORD_MAX_QV * GSWORD_MAX_QV + 2];
-    CG_TRY(cudaMemcpyAsync(tot, d_tot, sizeof(unsigned long long) * (size_t)(ne + 2), cudaMemcpyDeviceToHost, st));
+    unsigned long long entries = 0;
+    CG_TRY(cudaMemcpyAsync(&entries, d_tot + ne, sizeof(entries), cudaMemcpyDeviceToHost, st));
     CG_TRY(cudaStreamSynchronize(st));
-    const uint64_t entries = tot[ne];
-    const uint64_t n0 = tot[ne + 1];
+    const uint64_t n0 = csz[order[0]];
     if (entries >= (1ull << 32)) {
         cleanup();
         return fail(GSWORD_ELIMIT, "load_query: candidate graph has %llu entries (>= 2^32)",
@@ -629,30 +666,23 @@ int build_candidate_graph(gsword_ctx* ctx, int32_t nq, const int32_t* q_row_ptr,
         return fail(GSWORD_ENOMEM, "load_query: candidate graph (%llu entries): %s", (unsigned long long)entries,
                     cudaGetErrorString(e));
     }
-    CG_TRY(gsword::launch_bits_fill(ctx->d_cbits, ctx->cwords, order[0], n, d_cnt0, ctx->d_cand0, st));
+    CG_TRY(gsword::launch_cand_fill(g, order[0], ctx->d_cand0, st));
     for (int a = 0; a < nq; ++a)
         for (int b = 0; b < nq; ++b) {
             const int ed = eid[a][b];
             if (ed < 0) continue;
-            CG_TRY(gsword::launch_cg_fill(g, ctx->d_cbits, a, b, q_labels[b], ctx->d_cg_off + (size_t)ed * row,
-                                          ctx->d_clist, st));
+            CG_TRY(gsword::launch_cg_fill(g, a, b, q_labels[b], ctx->d_cg_off + edges[(size_t)ed].x, ctx->d_clist, st));
         }
     CG_TRY(cudaEventRecord(e1, st));
-    // candidate counts per query vertex (popcount of the bitmap rows)
-    std::vector<uint32_t> bits((size_t)nq * ctx->cwords);
-    CG_TRY(cudaMemcpyAsync(bits.data(), ctx->d_cbits, sizeof(uint32_t) * bits.size(), cudaMemcpyDeviceToHost, st));
     CG_TRY(cudaStreamSynchronize(st));
     float ms = 0.f;
     CG_TRY(cudaEventElapsedTime(&ms, e0, e1));
 #undef CG_TRY
     cleanup();
-    for (int u = 0; u < nq; ++u) {
-        uint64_t c = 0;
-        for (uint32_t w = 0; w < ctx->cwords; ++w) c += (uint64_t)__builtin_popcount(bits[(size_t)u * ctx->cwords + w]);
-        ctx->cand_count[u] = c;
-    }
+    for (int u = 0; u < nq; ++u) ctx->cand_count[u] = csz[u];
     ctx->cg_entries = entries;
     ctx->cg_seconds = ms * 1e-3;
+    ctx->cg_bytes = sizeof(uint32_t) * (2 * bits_words + off_total + entries + n0) + sizeof(uint2) * (size_t)ne;
     p->seed_lo = 0;
     p->seed_len = (uint32_t)n0;
     p->seed_identity = 0;
@@ -1287,6 +1317,7 @@ int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out) {
     out->filter = ctx->q_filter;
     for (int u = 0; u < ctx->plan.nq; ++u) out->candidates[u] = ctx->cand_count[u];
     out->cg_entries = ctx->cg_entries;
+    out->cg_bytes = ctx->cg_bytes;
     out->build_seconds = ctx->cg_seconds;
     out->refill_min[0] = ctx->tuned_refill[0] ? ctx->tuned_refill[0] : ctx->opt_refill_min;
     out->refill_min[1] = ctx->tuned_refill[1] ? ctx->tuned_refill[1] : ctx->opt_refill_min;

@@ -154,7 +154,12 @@ template <bool CG>
 __device__ __forceinline__ void local_run(const DeviceGraph& g, int e, uint32_t v, int32_t l, uint32_t* a,
                                           uint32_t* b) {
     if (CG) {
-        const uint32_t* off = g.cg_off + (size_t)e * (size_t)(g.n + 1) + v;
+        // Fig. 4: query edge e (1st CSR) -> position of v in C(u) (2nd CSR, rank directory)
+        // -> offsets of C(u, u', v) (3rd CSR); v lies in C(u) (it was matched to u)
+        const uint2 ed = __ldg(g.cg_edge + e);
+        const size_t w = (size_t)ed.y * g.cwords + (v >> 5);
+        const uint32_t bits = ldg_u32(g.cbits + w), pre = ldg_u32(g.crank + w);
+        const uint32_t* off = g.cg_off + (size_t)ed.x + pre + __popc(bits & ((1u << (v & 31u)) - 1u));
         *a = ldg_u32(off);
         *b = ldg_u32(off + 1);
     } else {
@@ -1642,44 +1647,47 @@ __device__ __forceinline__ bool bit_of(const uint32_t* cbits, uint32_t cwords, i
     return (cbits[(size_t)u * cwords + (v >> 5)] >> (v & 31u)) & 1u;
 }
 
-// counts[v] = |N_{label2}(v) ∩ C(u2)| if v in C(u) else 0;  counts[n] = 0
-__global__ void cg_count_kernel(const DeviceGraph g, const uint32_t* __restrict__ cbits, int u, int u2,
-                                int32_t label2, uint32_t* __restrict__ counts) {
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= g.n; v += (int64_t)gridDim.x * blockDim.x) {
-        uint32_t c = 0;
-        if (v < g.n && bit_of(cbits, g.cwords, u, (uint32_t)v)) {
-            uint32_t a, b;
-            segment(g, (uint32_t)v, label2, &a, &b);
-            for (uint32_t i = a; i < b; ++i) c += bit_of(cbits, g.cwords, u2, (uint32_t)g.col[i]) ? 1u : 0u;
-        }
-        counts[v] = c;
+// position of v in the ascending list C(u) (v in C(u)): the rank directory of the bitmap
+__device__ __forceinline__ uint32_t cand_rank(const DeviceGraph& g, int u, uint32_t v) {
+    const size_t w = (size_t)u * g.cwords + (v >> 5);
+    return g.crank[w] + __popc(g.cbits[w] & ((1u << (v & 31u)) - 1u));
+}
+
+// crank[u][w] = popc(cbits[u][w]); the exclusive scan of the row follows
+__global__ void rank_words_kernel(const uint32_t* __restrict__ cbits, uint32_t cwords, int u,
+                                  uint32_t* __restrict__ crank) {
+    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < cwords; w += (int64_t)gridDim.x * blockDim.x)
+        crank[(size_t)u * cwords + w] = __popc(cbits[(size_t)u * cwords + w]);
+}
+
+// counts[rank_u(v)] = |N_{label2}(v) ∩ C(u2)| for v in C(u) (Fig. 4, 3rd CSR sizes)
+__global__ void cg_count_kernel(const DeviceGraph g, int u, int u2, int32_t label2, uint32_t* __restrict__ counts) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < g.n; v += (int64_t)gridDim.x * blockDim.x) {
+        if (!bit_of(g.cbits, g.cwords, u, (uint32_t)v)) continue;
+        uint32_t c = 0, a, b;
+        segment(g, (uint32_t)v, label2, &a, &b);
+        for (uint32_t i = a; i < b; ++i) c += bit_of(g.cbits, g.cwords, u2, (uint32_t)g.col[i]) ? 1u : 0u;
+        counts[cand_rank(g, u, (uint32_t)v)] = c;
     }
 }
 
-__global__ void cg_fill_kernel(const DeviceGraph g, const uint32_t* __restrict__ cbits, int u, int u2,
-                               int32_t label2, const uint32_t* __restrict__ off, int32_t* __restrict__ out) {
+__global__ void cg_fill_kernel(const DeviceGraph g, int u, int u2, int32_t label2, const uint32_t* __restrict__ off,
+                               int32_t* __restrict__ out) {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < g.n; v += (int64_t)gridDim.x * blockDim.x) {
-        if (!bit_of(cbits, g.cwords, u, (uint32_t)v)) continue;
-        uint32_t pos = off[v];
+        if (!bit_of(g.cbits, g.cwords, u, (uint32_t)v)) continue;
+        uint32_t pos = off[cand_rank(g, u, (uint32_t)v)];
         uint32_t a, b;
         segment(g, (uint32_t)v, label2, &a, &b);
         for (uint32_t i = a; i < b; ++i) {
             const int32_t w = g.col[i];
-            if (bit_of(cbits, g.cwords, u2, (uint32_t)w)) out[pos++] = w;
+            if (bit_of(g.cbits, g.cwords, u2, (uint32_t)w)) out[pos++] = w;
         }
     }
 }
 
-__global__ void bits_count_kernel(const uint32_t* __restrict__ cbits, uint32_t cwords, int u, int64_t n,
-                                  uint32_t* __restrict__ counts) {
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= n; v += (int64_t)gridDim.x * blockDim.x)
-        counts[v] = (v < n && bit_of(cbits, cwords, u, (uint32_t)v)) ? 1u : 0u;
-}
-
-__global__ void bits_fill_kernel(const uint32_t* __restrict__ cbits, uint32_t cwords, int u, int64_t n,
-                                 const uint32_t* __restrict__ off, int32_t* __restrict__ out) {
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-        if (bit_of(cbits, cwords, u, (uint32_t)v)) out[off[v]] = (int32_t)v;
+__global__ void cand_fill_kernel(const DeviceGraph g, int u, int32_t* __restrict__ out) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < g.n; v += (int64_t)gridDim.x * blockDim.x)
+        if (bit_of(g.cbits, g.cwords, u, (uint32_t)v)) out[cand_rank(g, u, (uint32_t)v)] = (int32_t)v;
 }
 
 // ---- exclusive scan (three phases): 2048 elements per block
@@ -1870,27 +1878,25 @@ cudaError_t launch_filter(const DeviceGraph& g, const QFilter* d_qf, int nq, int
     return cudaGetLastError();
 }
 
-cudaError_t launch_cg_count(const DeviceGraph& g, const uint32_t* cbits, int u, int u2, int32_t label2,
-                            uint32_t* counts, cudaStream_t stream) {
-    cg_count_kernel<<<sm_grid(8), 256, 0, stream>>>(g, cbits, u, u2, label2, counts);
+cudaError_t launch_rank_words(const uint32_t* cbits, uint32_t cwords, int u, uint32_t* crank, cudaStream_t stream) {
+    rank_words_kernel<<<sm_grid(2), 256, 0, stream>>>(cbits, cwords, u, crank);
     return cudaGetLastError();
 }
 
-cudaError_t launch_cg_fill(const DeviceGraph& g, const uint32_t* cbits, int u, int u2, int32_t label2,
-                           const uint32_t* off, int32_t* out, cudaStream_t stream) {
-    cg_fill_kernel<<<sm_grid(8), 256, 0, stream>>>(g, cbits, u, u2, label2, off, out);
+cudaError_t launch_cg_count(const DeviceGraph& g, int u, int u2, int32_t label2, uint32_t* counts,
+                            cudaStream_t stream) {
+    cg_count_kernel<<<sm_grid(8), 256, 0, stream>>>(g, u, u2, label2, counts);
     return cudaGetLastError();
 }
 
-cudaError_t launch_bits_count(const uint32_t* cbits, uint32_t cwords, int u, int64_t n, uint32_t* counts,
-                              cudaStream_t stream) {
-    bits_count_kernel<<<sm_grid(4), 256, 0, stream>>>(cbits, cwords, u, n, counts);
+cudaError_t launch_cg_fill(const DeviceGraph& g, int u, int u2, int32_t label2, const uint32_t* off, int32_t* out,
+                           cudaStream_t stream) {
+    cg_fill_kernel<<<sm_grid(8), 256, 0, stream>>>(g, u, u2, label2, off, out);
     return cudaGetLastError();
 }
 
-cudaError_t launch_bits_fill(const uint32_t* cbits, uint32_t cwords, int u, int64_t n, const uint32_t* off,
-                             int32_t* out, cudaStream_t stream) {
-    bits_fill_kernel<<<sm_grid(4), 256, 0, stream>>>(cbits, cwords, u, n, off, out);
+cudaError_t launch_cand_fill(const DeviceGraph& g, int u, int32_t* out, cudaStream_t stream) {
+    cand_fill_kernel<<<sm_grid(4), 256, 0, stream>>>(g, u, out);
     return cudaGetLastError();
 }
 

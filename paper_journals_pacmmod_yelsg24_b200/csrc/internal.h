@@ -54,12 +54,20 @@ struct QFilter {
 //   bloom: blocked Bloom filter over the undirected edge set (one 64-bit word per
 //   test, 3 bits, ~16 bits per edge): "no" is exact, "maybe" falls back to the
 //   binary search.  NULL = disabled.
-//   clist/cg_off/cbits: the lists the sampler draws from.  Filter 0 (label only):
-//   clist = col, runs located through seg.  Filters 1-2 (LDF/NLF, NEXT-1): the
-//   candidate graph (Def. 5, Fig. 4) -- one CSR per directed query edge
-//   e = (u -> u'): clist[cg_off[e*(n+1) + v] .. cg_off[e*(n+1) + v + 1]) =
-//   C(u, u', v) = N(v) ∩ C(u') ascending (empty when v is not in C(u)); cbits row u =
-//   membership bitmap of C(u).
+//   clist/cg_off/cbits/crank/cg_edge: the lists the sampler draws from.  Filter 0
+//   (label only): clist = col, runs located through seg.  Filters 1-2 (LDF/NLF,
+//   NEXT-1): the candidate graph in the three-CSR format of Fig. 4 (Def. 5, P:L526,
+//   P:L770-L776):
+//     1st CSR  the query edges: e = (u -> u') indexes cg_edge[e] = {base, u};
+//     2nd CSR  C(u) in ascending id, held as the membership bitmap cbits row u with a
+//              rank directory crank row u (exclusive popcount prefix per 32-bit word):
+//              the position of v in C(u) is crank[u][v/32] + popc(cbits[u][v/32] below
+//              v) -- two independent loads instead of the paper's search;
+//     3rd CSR  per edge e, |C(u)| + 1 offsets at cg_off[base ...]: the local candidate
+//              list C(u, u', v) = N(v) ∩ C(u') of the i-th v of C(u) is
+//              clist[cg_off[base + i] .. cg_off[base + i + 1]), ascending.
+//   Memory O(nq |V| / 8 + sum_e |C(u_e)| + entries), not O(|E_q| |V|); a lookup is only
+//   made for v in C(u) (every matched vertex lies in its query vertex's candidate set).
 struct DeviceGraph {
     const int32_t* col;
     const uint32_t* seg;
@@ -67,6 +75,8 @@ struct DeviceGraph {
     const int32_t* clist;
     const uint32_t* cg_off;
     const uint32_t* cbits;
+    const uint32_t* crank;     // rank directory of cbits (same shape)
+    const uint2* cg_edge;      // per directed query edge: {offset base in cg_off, source u}
     uint32_t cwords;           // words per cbits row
     const unsigned long long* bloom;
     uint64_t bloom_mask;  // words - 1 (words is a power of two)
@@ -179,14 +189,15 @@ cudaError_t launch_trawl(int method, bool trace, bool cg, const DeviceGraph& g, 
 // candidate graph build (NEXT-1)
 cudaError_t launch_filter(const DeviceGraph& g, const QFilter* d_qf, int nq, int filter, uint32_t* cbits,
                           const int32_t* d_vlabel, cudaStream_t stream);
-cudaError_t launch_cg_count(const DeviceGraph& g, const uint32_t* cbits, int u, int u2, int32_t label2,
-                            uint32_t* counts, cudaStream_t stream);
-cudaError_t launch_cg_fill(const DeviceGraph& g, const uint32_t* cbits, int u, int u2, int32_t label2,
-                           const uint32_t* off, int32_t* out, cudaStream_t stream);
-cudaError_t launch_bits_count(const uint32_t* cbits, uint32_t cwords, int u, int64_t n, uint32_t* counts,
-                              cudaStream_t stream);
-cudaError_t launch_bits_fill(const uint32_t* cbits, uint32_t cwords, int u, int64_t n, const uint32_t* off,
-                             int32_t* out, cudaStream_t stream);
+// rank directory row u: crank[u][w] = popc(cbits[u][w]) (scanned afterwards)
+cudaError_t launch_rank_words(const uint32_t* cbits, uint32_t cwords, int u, uint32_t* crank, cudaStream_t stream);
+// counts[rank_u(v)] = |N_label2(v) ∩ C(u2)| for every v in C(u)  (g.cbits / g.crank set)
+cudaError_t launch_cg_count(const DeviceGraph& g, int u, int u2, int32_t label2, uint32_t* counts,
+                            cudaStream_t stream);
+cudaError_t launch_cg_fill(const DeviceGraph& g, int u, int u2, int32_t label2, const uint32_t* off, int32_t* out,
+                           cudaStream_t stream);
+// out[rank_u(v)] = v for every v in C(u): the ascending list C(u)
+cudaError_t launch_cand_fill(const DeviceGraph& g, int u, int32_t* out, cudaStream_t stream);
 // exclusive scan of n u32 in place, offset by *d_base (64-bit, may be NULL = 0); the
 // 64-bit grand total goes to *d_total.  d_tmp holds scan_tmp_words(n) words.
 size_t scan_tmp_words(int64_t n);

@@ -78,7 +78,7 @@ class _Result(ctypes.Structure):
 class _QueryStats(ctypes.Structure):
     _fields_ = [("nq", ctypes.c_int32), ("filter", ctypes.c_int32), ("candidates", ctypes.c_uint64 * MAX_QV),
                 ("cg_entries", ctypes.c_uint64), ("build_seconds", ctypes.c_double),
-                ("refill_min", ctypes.c_int32 * 2), ("occupancy", ctypes.c_int32 * 2)]
+                ("refill_min", ctypes.c_int32 * 2), ("occupancy", ctypes.c_int32 * 2), ("cg_bytes", ctypes.c_uint64)]
 
 
 class _PlanInfo(ctypes.Structure):
@@ -315,7 +315,7 @@ class Context:
         st = _QueryStats()
         _check(_lib.gsword_query_info(self._h, ctypes.byref(st)))
         return {"nq": st.nq, "filter": st.filter, "candidates": list(st.candidates)[:st.nq],
-                "cg_entries": int(st.cg_entries), "build_seconds": st.build_seconds,
+                "cg_entries": int(st.cg_entries), "build_seconds": st.build_seconds, "cg_bytes": int(st.cg_bytes),
                 "refill_min": list(st.refill_min), "occupancy": list(st.occupancy)}
 
     # convenience for workloads.gen.Graph / Query objects
