@@ -12,10 +12,10 @@ NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-O3,-pthread -Xptx
 all: $(LIB) $(ORACLE)
 
 variant:
-	$(NVCC) $(NVFLAGS) -shared -o $(OUT) $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_frontier.cu $(CSRC)/gsword_host.cpp 2> $(OUT).ptxas.log || (cat $(OUT).ptxas.log; false)
+	$(NVCC) $(NVFLAGS) -shared -o $(OUT) $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_host.cpp 2> $(OUT).ptxas.log || (cat $(OUT).ptxas.log; false)
 
-$(LIB): $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_frontier.cu $(CSRC)/gsword_host.cpp $(CSRC)/internal.h $(CSRC)/device_util.cuh include/gsword.h
-	$(NVCC) $(NVFLAGS) -shared -o $@ $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_frontier.cu $(CSRC)/gsword_host.cpp 2> build_ptxas.log || (cat build_ptxas.log; false)
+$(LIB): $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_host.cpp $(CSRC)/internal.h $(CSRC)/device_util.cuh include/gsword.h
+	$(NVCC) $(NVFLAGS) -shared -o $@ $(CSRC)/gsword_kernels.cu $(CSRC)/gsword_host.cpp 2> build_ptxas.log || (cat build_ptxas.log; false)
 
 $(ORACLE): oracle/oracle.c
 	gcc -O2 -std=c11 -Wall -Wextra -shared -fPIC -pthread -o $@ $<

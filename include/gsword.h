@@ -150,8 +150,6 @@ typedef struct {
                            /* per method (after autotune; GSWORD_OPT_BLOCKS_PER_SM */
                            /* may lower it further)                               */
     uint64_t cg_bytes;
-    int32_t path[2];       /* sampler path of estimates per method: 0 persistent refill   */
-                           /* kernel, 1 level-synchronous frontier (GSWORD_OPT_PATH)     */
 } gsword_query_stats;
 
 /* Tunables for gsword_set_option (defaults chosen by measurement). */
@@ -203,18 +201,6 @@ typedef enum {
                                    /* the autotuned one; 0 default launch bounds, 1   */
                                    /* one CTA/SM less, 2 one more (forced; for A/B    */
                                    /* and sanitizer runs).  Results are unaffected    */
-    GSWORD_OPT_PATH = 16,          /* Alley sampler: -1 (default) autotuned at query   */
-                                   /* load, 0 the persistent refill kernel, 1 the      */
-                                   /* level-synchronous frontier kernels (one launch   */
-                                   /* per position over a compacted frontier of live   */
-                                   /* samples; default rules only: variant 0, refill   */
-                                   /* schedule, no streaming, >= 2 query vertices).    */
-                                   /* Results are unaffected; count_sectors always     */
-                                   /* uses the persistent kernel                       */
-    GSWORD_OPT_FRONTIER_BATCH = 17, /* samples per batch of the frontier path (power   */
-                                   /* of two, 2^10 .. 2^24, default 2^22): its buffers  */
-                                   /* take ~2 x batch x (12 + 4 nq) bytes (traces: +4 nq */
-                                   /* + 4); results are unaffected                     */
     GSWORD_OPT_FAULT_QUEUE = 15,   /* fault injection (tests): the next sampling launch */
                                    /* starts its sample queue at this value instead of */
                                    /* 0, as a corrupted counter would (ids skipped);   */

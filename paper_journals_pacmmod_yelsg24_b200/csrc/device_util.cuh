@@ -1,6 +1,6 @@
-// device_util.cuh — device helpers shared by the sampling kernels (gsword_kernels.cu:
-// the persistent refill kernels, streaming, trawling) and the level-synchronous frontier
-// kernels (gsword_frontier.cu).  Not part of the public ABI; every function is inline.
+// device_util.cuh — device helpers of the sampling kernels (gsword_kernels.cu: the
+// persistent refill kernels, warp streaming, trawling): Philox, edge index, list runs,
+// compensated sums.  Not part of the public ABI; every function is inline.
 #pragma once
 
 #include <cstdint>
@@ -169,27 +169,6 @@ __device__ __forceinline__ bool is_edge(const DeviceGraph& g, uint32_t a, uint32
     uint32_t lo, hi;
     segment(g, a, lb, &lo, &hi);
     if (COUNT) sec += 1.0 + (double)bs_sectors(hi - lo);
-    return in_run(g.col, lo, hi, (int32_t)b);
-}
-
-// The exact part of is_edge once the filter word of hash h said "maybe" (or there is no
-// filter): the edge-set buckets, or a binary search of b in N_lb(a).
-__device__ __forceinline__ bool is_edge_after_filter(const DeviceGraph& g, uint32_t a, uint32_t b, uint64_t h,
-                                                     int32_t lb, double& sec) {
-    (void)sec;
-    if (g.eset) {
-        const unsigned long long key = edge_key(a, b);
-        uint64_t bk = h & g.eset_mask;
-        while (true) {
-            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(g.eset + 4 * bk);
-            const ulonglong2 x0 = __ldg(p), x1 = __ldg(p + 1);
-            if (x0.x == key || x0.y == key || x1.x == key || x1.y == key) return true;
-            if (x0.x == kEmptyKey || x0.y == kEmptyKey || x1.x == kEmptyKey || x1.y == kEmptyKey) return false;
-            bk = (bk + 1) & g.eset_mask;
-        }
-    }
-    uint32_t lo, hi;
-    segment(g, a, lb, &lo, &hi);
     return in_run(g.col, lo, hi, (int32_t)b);
 }
 

@@ -274,21 +274,8 @@ struct gsword_ctx {
     int tuned_occ[2] = {0, 0};    // occupancy variant of the estimate kernel (kModeOccShift)
     int opt_occ = -1;             // GSWORD_OPT_OCCUPANCY: -1 autotuned, else forced
     uint64_t opt_fault_queue = 0;  // GSWORD_OPT_FAULT_QUEUE: one-shot corrupted queue start
-    int opt_path = -1;             // GSWORD_OPT_PATH: -1 autotuned, 0 persistent, 1 frontier
-    uint32_t opt_fr_batch = 1u << 22;  // GSWORD_OPT_FRONTIER_BATCH: samples per frontier batch
-    int tuned_path[2] = {0, 0};    // autotuned sampler path per method (1 = frontier)
-    // level-synchronous frontier (gsword_frontier.cu): two SoA buffers of capacity fr_cap
-    // with fr_rows rows of M (and of csize when fr_trace)
-    void* d_frontier = nullptr;
-    size_t frontier_bytes = 0;
-    gsword::FrontierBufs fr_a{}, fr_b{};
-    uint32_t fr_cap = 0;
-    int fr_rows = 0;
-    bool fr_trace = false;
-    uint32_t* d_fr_counts = nullptr;
-    int fr_grid[2][2] = {{0, 0}, {0, 0}};  // [cg][trace]
     struct Tuned {
-        int refill[2], occ[2], path[2];
+        int refill[2], occ[2];
     };
     std::map<std::string, Tuned> tune_cache;
     int opt_eset = 1;
@@ -429,94 +416,9 @@ DeviceGraph device_graph(const gsword_ctx* ctx) {
     return g;
 }
 
-// The level-synchronous frontier sampler applies to Alley with the default sampler rules
-// (no comparison variant, refill schedule, count-then-index) and at least two positions.
-bool frontier_eligible(const gsword_ctx* ctx, int method, int mode) {
-    return method == GSWORD_ALLEY && ((mode & 3) == gsword::kModeEstimate || (mode & 3) == gsword::kModeTrace) &&
-           ctx->opt_sched == 0 && !ctx->opt_streaming && ctx->opt_variant == 0 && ctx->plan.nq >= 2 &&
-           ctx->opt_fault_queue == 0;
-}
-
-bool use_frontier(const gsword_ctx* ctx, int method, int mode) {
-    if (!frontier_eligible(ctx, method, mode)) return false;
-    if (ctx->opt_path >= 0) return ctx->opt_path == 1;
-    return ctx->opt_autotune && ctx->tuned_path[method & 1] == 1 && (mode & 3) == gsword::kModeEstimate;
-}
-
-// Frontier buffers for the loaded query: two SoA frontiers of capacity cap (a power of two
-// up to 2^22 samples), nq rows of M (and of csize + sector counts for traces).
-int ensure_frontier(gsword_ctx* ctx, uint64_t count, bool trace) {
-    uint32_t cap = std::min<uint32_t>(1u << 16, ctx->opt_fr_batch);
-    while (cap < count && cap < ctx->opt_fr_batch) cap <<= 1;
-    const int rows = ctx->plan.nq;
-    if (ctx->d_frontier && ctx->fr_cap >= cap && ctx->fr_rows >= rows && (ctx->fr_trace || !trace)) return GSWORD_OK;
-    cap = std::max(cap, ctx->fr_cap);
-    const int r2 = std::max(rows, ctx->fr_rows);
-    const bool tr = trace || ctx->fr_trace;
-    // per buffer: W f64 + slot u32 + M r2 x i32 (+ cs r2 x u32 + msec u32)
-    const size_t per = (size_t)cap * (4 + 8 + 4 * (size_t)r2 + (tr ? 4 * (size_t)r2 + 4 : 0));
-    if (ctx->d_frontier) cudaFree(ctx->d_frontier);
-    ctx->d_frontier = nullptr;
-    cudaError_t e = cudaMalloc(&ctx->d_frontier, 2 * per);
-    if (e != cudaSuccess) {
-        ctx->fr_cap = 0;
-        return fail(GSWORD_ENOMEM, "frontier: cudaMalloc(%zu): %s", 2 * per, cudaGetErrorString(e));
-    }
-    if (!ctx->d_fr_counts) CUDA_TRY(cudaMalloc(&ctx->d_fr_counts, sizeof(uint32_t) * GSWORD_MAX_QV));
-    ctx->frontier_bytes = 2 * per;
-    char* base = reinterpret_cast<char*>(ctx->d_frontier);
-    for (int k = 0; k < 2; ++k) {
-        gsword::FrontierBufs& f = k ? ctx->fr_b : ctx->fr_a;
-        char* q = base + (size_t)k * per;
-        f.W = reinterpret_cast<double*>(q);
-        q += (size_t)cap * 8;
-        f.slot = reinterpret_cast<uint32_t*>(q);
-        q += (size_t)cap * 4;
-        f.M = reinterpret_cast<int32_t*>(q);
-        q += (size_t)cap * 4 * (size_t)r2;
-        f.cs = tr ? reinterpret_cast<uint32_t*>(q) : nullptr;
-        if (tr) q += (size_t)cap * 4 * (size_t)r2;
-        f.msec = tr ? reinterpret_cast<uint32_t*>(q) : nullptr;
-    }
-    ctx->fr_cap = cap;
-    ctx->fr_rows = r2;
-    ctx->fr_trace = tr;
-    return GSWORD_OK;
-}
-
-int run_frontier(gsword_ctx* ctx, int mode, uint64_t first, uint64_t count, uint64_t seed, double* d_out4,
-                 gsword_sample_record* d_records) {
-    const bool trace = (mode & 3) == gsword::kModeTrace;
-    const bool cg = ctx->q_filter != 0;
-    int rc = ensure_frontier(ctx, count, trace);
-    if (rc) return rc;
-    int& grid = ctx->fr_grid[cg][trace];
-    if (grid == 0) grid = gsword::frontier_grid(cg, trace, ctx->num_sms);
-    if (grid <= 0) return fail(GSWORD_ECUDA, "frontier kernels do not fit on the device");
-    if (grid > ctx->partial_cap) {
-        if (ctx->d_partials) cudaFree(ctx->d_partials);
-        ctx->d_partials = nullptr;
-        CUDA_TRY(cudaMalloc(&ctx->d_partials, sizeof(Partial) * (size_t)grid));
-        ctx->partial_cap = grid;
-    }
-    ctx->last_grid = grid;
-    ctx->last_threads = 256;
-    CUDA_TRY(cudaEventRecord(ctx->evk0, ctx->stream));
-    cudaError_t e = gsword::launch_frontier(device_graph(ctx), ctx->plan, cg, trace, ctx->fr_a, ctx->fr_b, ctx->fr_cap,
-                                            std::min(ctx->fr_cap, ctx->opt_fr_batch), ctx->d_fr_counts, first, count,
-                                            seed, (uint32_t)ctx->opt_coop, grid, ctx->d_partials, d_records,
-                                            ctx->stream);
-    if (e != cudaSuccess) return cuda_fail(e, "launch frontier kernels");
-    CUDA_TRY(cudaEventRecord(ctx->evk1, ctx->stream));
-    e = gsword::launch_reduce(ctx->d_partials, grid, d_out4, nullptr, ctx->stream);
-    if (e != cudaSuccess) return cuda_fail(e, "launch reduce kernel");
-    return GSWORD_OK;
-}
-
 int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, uint64_t seed, double* d_out4,
         gsword_sample_record* d_records, double* d_sectors) {
     if (first + count < first) return fail(GSWORD_EINVAL, "sample-id range [first, first + n) overflows u64");
-    if (use_frontier(ctx, method, mode)) return run_frontier(ctx, mode, first, count, seed, d_out4, d_records);
     if (ctx->q_filter) mode |= gsword::kModeCG;
     if (method == GSWORD_ALLEY && ctx->opt_streaming && (mode & 3) != gsword::kModeCount) mode |= gsword::kModeStream;
     if (ctx->opt_sched != 0) mode |= gsword::kModeSync;
@@ -835,8 +737,6 @@ int gsword_destroy(gsword_ctx* ctx) {
     if (ctx->d_out4) cudaFree(ctx->d_out4);
     if (ctx->d_sectors) cudaFree(ctx->d_sectors);
     if (ctx->d_phase) cudaFree(ctx->d_phase);
-    if (ctx->d_frontier) cudaFree(ctx->d_frontier);
-    if (ctx->d_fr_counts) cudaFree(ctx->d_fr_counts);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
     if (ctx->ev1) cudaEventDestroy(ctx->ev1);
     if (ctx->evk0) cudaEventDestroy(ctx->evk0);
@@ -917,15 +817,6 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
             if (value & ~(int64_t)(GSWORD_VARIANT_WJ_PARENT_FIRST | GSWORD_VARIANT_ALLEY_DUPCHECK_POST))
                 return fail(GSWORD_EINVAL, "unknown variant bits 0x%llx", (unsigned long long)value);
             ctx->opt_variant = (int)value;
-            return GSWORD_OK;
-        case GSWORD_OPT_PATH:
-            if (value < -1 || value > 1) return fail(GSWORD_EINVAL, "sampler path must be -1 (auto), 0 or 1");
-            ctx->opt_path = (int)value;
-            return GSWORD_OK;
-        case GSWORD_OPT_FRONTIER_BATCH:
-            if (value < 1024 || value > (1 << 24) || (value & (value - 1)))
-                return fail(GSWORD_EINVAL, "frontier batch must be a power of two in [2^10, 2^24]");
-            ctx->opt_fr_batch = (uint32_t)value;
             return GSWORD_OK;
         case GSWORD_OPT_FAULT_QUEUE:
             if (value < 0) return fail(GSWORD_EINVAL, "fault queue start must be >= 0");
@@ -1330,13 +1221,12 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
     ctx->query_loaded = true;
     ctx->tuned_refill[0] = ctx->tuned_refill[1] = 0;
     ctx->tuned_occ[0] = ctx->tuned_occ[1] = 0;
-    ctx->tuned_path[0] = ctx->tuned_path[1] = 0;
     std::string tkey;
     if (ctx->opt_autotune && ctx->opt_sched == 0) {
         // the query exactly as given plus every option that changes the kernels' schedule
         const int opts[] = {n_qv, ctx->opt_blocks_per_sm, ctx->opt_threads, ctx->opt_chunk, ctx->opt_l2,
                             ctx->opt_coop, ctx->opt_bloom, ctx->opt_eset, ctx->opt_filter, ctx->opt_streaming,
-                            ctx->opt_variant, ctx->opt_occ, ctx->opt_path};
+                            ctx->opt_variant, ctx->opt_occ};
         tkey.append(reinterpret_cast<const char*>(opts), sizeof(opts));
         tkey.append(reinterpret_cast<const char*>(q_row_ptr), sizeof(int32_t) * (size_t)(n_qv + 1));
         tkey.append(reinterpret_cast<const char*>(q_col), sizeof(int32_t) * (size_t)q_row_ptr[n_qv]);
@@ -1347,7 +1237,6 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
             for (int m = 0; m < 2; ++m) {
                 ctx->tuned_refill[m] = it->second.refill[m];
                 ctx->tuned_occ[m] = it->second.occ[m];
-                ctx->tuned_path[m] = it->second.path[m];
             }
         }
     }
@@ -1408,26 +1297,14 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
                     ctx->tuned_occ[m] = 1 + c;
                 }
         }
-        // Phase 3 (Alley): the level-synchronous frontier kernels against the best persistent
-        // configuration, on the same id range (the frontier must win by 1.5 % too)
-        if (ctx->opt_path < 0 && frontier_eligible(ctx, GSWORD_ALLEY, gsword::kModeEstimate) && rc2 == GSWORD_OK &&
-            e == cudaSuccess) {
-            float t3[2][4] = {};
-            time_phase(1, [&](int m, int) { ctx->tuned_path[m] = 1; }, t3);
-            ctx->tuned_path[GSWORD_WJ] = 0;
-            ctx->tuned_path[GSWORD_ALLEY] = (t3[GSWORD_ALLEY][0] < 0.985f * best[GSWORD_ALLEY]) ? 1 : 0;
-        }
         for (cudaEvent_t x : evs) cudaEventDestroy(x);
         if (rc2 != GSWORD_OK || e != cudaSuccess) {
             ctx->tuned_refill[0] = ctx->tuned_refill[1] = 0;
             ctx->tuned_occ[0] = ctx->tuned_occ[1] = 0;
-            ctx->tuned_path[0] = ctx->tuned_path[1] = 0;
             return rc2 != GSWORD_OK ? rc2 : cuda_fail(e, "autotune");
         }
         if (ctx->tune_cache.size() >= 4096) ctx->tune_cache.clear();
-        ctx->tune_cache[tkey] = {{ctx->tuned_refill[0], ctx->tuned_refill[1]},
-                                 {ctx->tuned_occ[0], ctx->tuned_occ[1]},
-                                 {ctx->tuned_path[0], ctx->tuned_path[1]}};
+        ctx->tune_cache[tkey] = {{ctx->tuned_refill[0], ctx->tuned_refill[1]}, {ctx->tuned_occ[0], ctx->tuned_occ[1]}};
     }
     return GSWORD_OK;
 }
@@ -1444,7 +1321,6 @@ int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out) {
     out->build_seconds = ctx->cg_seconds;
     out->refill_min[0] = ctx->tuned_refill[0] ? ctx->tuned_refill[0] : ctx->opt_refill_min;
     out->refill_min[1] = ctx->tuned_refill[1] ? ctx->tuned_refill[1] : ctx->opt_refill_min;
-    for (int m = 0; m < 2; ++m) out->path[m] = use_frontier(ctx, m, gsword::kModeEstimate) ? 1 : 0;
     for (int m = 0; m < 2; ++m) {
         int mode = gsword::kModeEstimate | (ctx->q_filter ? gsword::kModeCG : 0);
         if (ctx->opt_sched == 0 && !(m == GSWORD_ALLEY && ctx->opt_streaming)) {

@@ -162,26 +162,6 @@ struct Partial {
     double model;               // counting build: algorithmic sectors of reading A26
 };
 
-// Level-synchronous frontier of the Alley sampler (gsword_frontier.cu): structure of
-// arrays with capacity `cap` (M and cs hold nq rows of cap entries).
-struct FrontierBufs {
-    uint32_t* slot;   // sample offset within the batch
-    double* W;        // running weight
-    int32_t* M;       // M[j * cap + i]: matched vertex of position j
-    uint32_t* cs;     // traces: csize[j * cap + i]
-    uint32_t* msec;   // traces: A26 sectors so far
-};
-// CTAs per launch of the frontier kernels (every level uses the same grid); 0 = no fit
-int frontier_grid(bool cg, bool trace, int num_sms);
-// Runs samples [first, first + count) of the loaded plan (Alley, default variant, nq >= 2)
-// level by level in batches of `cap`, accumulating into d_partials[grid] (zeroed here);
-// d_counts: kMaxQV u32 of scratch; d_records (traces) indexed by sample id - first.
-// cap = row stride of the buffers, batch (<= cap) = samples per batch.
-cudaError_t launch_frontier(const DeviceGraph& g, const Plan& plan, bool cg, bool trace, const FrontierBufs& a,
-                            const FrontierBufs& b, uint32_t cap, uint32_t batch, uint32_t* d_counts, uint64_t first,
-                            uint64_t count, uint64_t seed, uint32_t coop_threshold, int grid, Partial* d_partials,
-                            gsword_sample_record* d_records, cudaStream_t stream);
-
 // Kernel entry points (gsword_kernels.cu).  All enqueue on `stream`.
 cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan& plan, const LaunchCfg& cfg,
                           uint64_t first, uint64_t count, uint64_t seed, unsigned long long* d_queue,

@@ -37,8 +37,6 @@ OPT_STREAMING = 12  # Alley by warp streaming (Alg. 3, reading A25)
 OPT_VARIANT = 13  # comparison variants of readings A3/A5 (bit flags below)
 OPT_OCCUPANCY = 14  # estimate-kernel occupancy variant: -1 autotuned, 0/1/2 forced
 OPT_FAULT_QUEUE = 15  # fault injection: the next launch's queue starts here (one-shot)
-OPT_PATH = 16  # Alley sampler path: -1 autotuned, 0 persistent refill kernel, 1 frontier kernels
-OPT_FRONTIER_BATCH = 17  # samples per frontier batch (power of two, 2^10..2^24)
 VARIANT_WJ_PARENT_FIRST = 2
 VARIANT_ALLEY_DUPCHECK_POST = 4
 SCHED_REFILL, SCHED_SAMPLE_SYNC, SCHED_INHERIT = 0, 1, 2
@@ -80,8 +78,7 @@ class _Result(ctypes.Structure):
 class _QueryStats(ctypes.Structure):
     _fields_ = [("nq", ctypes.c_int32), ("filter", ctypes.c_int32), ("candidates", ctypes.c_uint64 * MAX_QV),
                 ("cg_entries", ctypes.c_uint64), ("build_seconds", ctypes.c_double),
-                ("refill_min", ctypes.c_int32 * 2), ("occupancy", ctypes.c_int32 * 2), ("cg_bytes", ctypes.c_uint64),
-                ("path", ctypes.c_int32 * 2)]
+                ("refill_min", ctypes.c_int32 * 2), ("occupancy", ctypes.c_int32 * 2), ("cg_bytes", ctypes.c_uint64)]
 
 
 class _PlanInfo(ctypes.Structure):
@@ -319,7 +316,7 @@ class Context:
         _check(_lib.gsword_query_info(self._h, ctypes.byref(st)))
         return {"nq": st.nq, "filter": st.filter, "candidates": list(st.candidates)[:st.nq],
                 "cg_entries": int(st.cg_entries), "build_seconds": st.build_seconds, "cg_bytes": int(st.cg_bytes),
-                "refill_min": list(st.refill_min), "occupancy": list(st.occupancy), "path": list(st.path)}
+                "refill_min": list(st.refill_min), "occupancy": list(st.occupancy)}
 
     # convenience for workloads.gen.Graph / Query objects
     def load_graph_obj(self, g) -> None:

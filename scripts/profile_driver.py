@@ -23,6 +23,7 @@ ap.add_argument("--coop", type=int, default=-1)
 ap.add_argument("--threads", type=int, default=0)
 ap.add_argument("--chunk", type=int, default=0)
 ap.add_argument("--bps", type=int, default=0)
+ap.add_argument("--methods", default="0,1")
 args = ap.parse_args()
 
 g, qs = gen.CONFIGS[args.config]()
@@ -39,11 +40,12 @@ with G.Context(0) as ctx:
         ctx.set_option(G.OPT_BLOCKS_PER_SM, args.bps)
     ctx.load_graph_obj(g)
     ctx.load_query_obj(q)
-    for m in (G.WJ, G.ALLEY):
+    methods = [int(x) for x in args.methods.split(",")]
+    for m in methods:
         ctx.estimate(m, 1_000_000, 42)
     torch.cuda.synchronize()
     torch.cuda.profiler.start()
-    res = {m: ctx.estimate(m, int(args.samples), 42) for m in (G.WJ, G.ALLEY)}
+    res = {m: ctx.estimate(m, int(args.samples), 42) for m in methods}
     torch.cuda.profiler.stop()
     for m, r in res.items():
         print(f"method={m} samples={int(args.samples)} seconds={r['seconds']:.4f} "
