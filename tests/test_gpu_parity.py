@@ -83,7 +83,7 @@ def test_c0_estimate_near_exact(ctx, G, c0):
         ctx.load_query_obj(q)
         for m in (G.WJ, G.ALLEY):
             r = ctx.estimate(m, 1_000_000, seed=7)
-            assert abs(r["estimate"] - truth) <= 5 * math.sqrt(max(r["variance"], 0.0)) + 1e-9
+            assert abs(r["estimate"] - truth) <= 3 * math.sqrt(max(r["variance"], 0.0)) + 1e-9
 
 
 # ------------------------------------------------------------------ fuzz: tiny random inputs
@@ -492,7 +492,7 @@ def test_trawl_parity(ctx, G, c0, method):
         _trawl_parity(ctx, G, g, q, method, 5, 0, 20_000, 2**62)
         truth = oracle.count_embeddings(g, q)
         r = ctx.trawl(method, 1_000_000, 8)
-        assert abs(r["estimate"] - truth) <= 5 * math.sqrt(max(r["variance"], 0.0)) + 1e-9
+        assert abs(r["estimate"] - truth) <= 3 * math.sqrt(max(r["variance"], 0.0)) + 1e-9
 
 
 def test_trawl_parity_c2_and_filter(ctx, G):

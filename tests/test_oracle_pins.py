@@ -225,18 +225,30 @@ def test_sampler_z_scores_tiny(method):
         if var1 == 0:
             assert est == truth
     zs = np.array(zs)
-    assert np.all(np.abs(zs) < 5)
-    assert abs(zs.mean()) < 5 / math.sqrt(30)
+    # BASELINE.json north_star: the estimate lands within 3 sigma (sigma from the exact variance
+    # of one sample, tree walk) for every seed; the seeds are fixed, so this is deterministic.
+    # The spread must also look normal: ~68 % within 1 sigma, ~95 % within 2, mean ~0.
+    assert np.all(np.abs(zs) < 3)
+    assert 0.45 <= float(np.mean(np.abs(zs) < 1)) <= 0.9
+    assert float(np.mean(np.abs(zs) < 2)) >= 0.85
+    assert abs(zs.mean()) < 3 / math.sqrt(30)
 
 
 @pytest.mark.parametrize("method", [oracle.WJ, oracle.ALLEY])
-def test_sampler_c0_within_4_sigma(c0, method):
+def test_sampler_c0_within_3_sigma(c0, method):
+    # every C0 query (BASELINE configs[0]) x 3 seeds at 1e5 samples, against the exact count
     g, qs = c0
-    for q in qs[:6]:
+    zs = []
+    for q in qs:
         truth = oracle.count_embeddings(g, q)
-        agg = oracle.estimate(g, q, method, seed=1, n_samples=100_000, threads=4)
-        sigma = math.sqrt(agg["variance"]) if agg["variance"] > 0 else 0.0
-        assert abs(agg["estimate"] - truth) <= 4 * sigma + 1e-9, (q.name, truth, agg)
+        for seed in (1, 2, 3):
+            agg = oracle.estimate(g, q, method, seed=seed, n_samples=100_000, threads=4)
+            sigma = math.sqrt(agg["variance"]) if agg["variance"] > 0 else 0.0
+            assert abs(agg["estimate"] - truth) <= 3 * sigma + 1e-9, (q.name, seed, truth, agg)
+            if sigma > 0:
+                zs.append((agg["estimate"] - truth) / sigma)
+    zs = np.array(zs)
+    assert float(np.mean(np.abs(zs) < 2)) >= 0.85
 
 
 def test_split_range_identity(c0):

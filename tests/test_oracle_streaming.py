@@ -138,13 +138,13 @@ def test_stream_does_not_change_wanderjoin(c0):
         assert a.tobytes() == b.tobytes()
 
 
-def test_stream_c0_within_4_sigma(c0):
+def test_stream_c0_within_3_sigma(c0):
     g, qs = c0
     for q in qs[:4]:
         truth = oracle.count_embeddings(g, q)
         agg = oracle.estimate(g, q, oracle.ALLEY, seed=2, n_samples=100_000, threads=4, select=S)
         sigma = math.sqrt(agg["variance"]) if agg["variance"] > 0 else 0.0
-        assert abs(agg["estimate"] - truth) <= 4 * sigma + 1e-9, (q.name, truth, agg)
+        assert abs(agg["estimate"] - truth) <= 3 * sigma + 1e-9, (q.name, truth, agg)
 
 
 def test_inheritance_with_streaming_unbiased():
