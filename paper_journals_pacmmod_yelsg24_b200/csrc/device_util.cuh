@@ -172,6 +172,37 @@ __device__ __forceinline__ bool is_edge(const DeviceGraph& g, uint32_t a, uint32
     return in_run(g.col, lo, hi, (int32_t)b);
 }
 
+// The two halves of is_edge: the filter test alone ("maybe", never a false "no"; true when
+// there is no filter), and the exact test alone (edge-set buckets, or a binary search).
+template <bool COUNT>
+__device__ __forceinline__ bool bloom_maybe(const DeviceGraph& g, uint32_t a, uint32_t b, double& sec) {
+    if (!g.bloom) return true;
+    if (COUNT) sec += 1.0;
+    const uint64_t h = edge_hash(a, b);
+    const uint64_t m = bloom_bits(h);
+    return (__ldg(g.bloom + (h & g.bloom_mask)) & m) == m;
+}
+
+template <bool COUNT>
+__device__ __forceinline__ bool is_edge_exact(const DeviceGraph& g, uint32_t a, uint32_t b, int32_t lb, double& sec) {
+    if (g.eset) {
+        const unsigned long long key = edge_key(a, b);
+        uint64_t bk = edge_hash(a, b) & g.eset_mask;
+        while (true) {
+            if (COUNT) sec += 1.0;
+            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(g.eset + 4 * bk);
+            const ulonglong2 x0 = __ldg(p), x1 = __ldg(p + 1);
+            if (x0.x == key || x0.y == key || x1.x == key || x1.y == key) return true;
+            if (x0.x == kEmptyKey || x0.y == kEmptyKey || x1.x == kEmptyKey || x1.y == kEmptyKey) return false;
+            bk = (bk + 1) & g.eset_mask;
+        }
+    }
+    uint32_t lo, hi;
+    segment(g, a, lb, &lo, &hi);
+    if (COUNT) sec += 1.0 + (double)bs_sectors(hi - lo);
+    return in_run(g.col, lo, hi, (int32_t)b);
+}
+
 // Is x in every N_l(M[j]) for j in `mask`?  M column `col_of` in shared memory.
 template <bool COUNT>
 __device__ __forceinline__ bool member_all(const DeviceGraph& g, const uint32_t* Ms, int stride, int col_of,

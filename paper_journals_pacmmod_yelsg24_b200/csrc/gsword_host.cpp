@@ -362,6 +362,11 @@ int occ_variant(const gsword_ctx* ctx, int method) {
     return ctx->opt_autotune ? ctx->tuned_occ[method & 1] : 0;
 }
 
+// refill threshold in use for `method` (autotuned or GSWORD_OPT_REFILL_MIN)
+int refill_min_of(const gsword_ctx* ctx, int method) {
+    return (ctx->opt_autotune && ctx->tuned_refill[method & 1] > 0) ? ctx->tuned_refill[method & 1] : ctx->opt_refill_min;
+}
+
 // every position d >= 1 has exactly one backward neighbour (spanning-tree order)
 bool plan_is_tree(const Plan& p) {
     for (int d = 1; d < p.nq; ++d)
@@ -382,8 +387,7 @@ int launch_config(gsword_ctx* ctx, int method, int mode, LaunchCfg* cfg) {
     cfg->coop_threshold = ctx->opt_coop;
     cfg->sched = ctx->opt_sched;
     cfg->ms_rows = rows;
-    cfg->refill_min = (uint32_t)((ctx->opt_autotune && ctx->tuned_refill[method & 1] > 0) ? ctx->tuned_refill[method & 1]
-                                                                                       : ctx->opt_refill_min);
+    cfg->refill_min = (uint32_t)refill_min_of(ctx, method);
     if (cfg->grid > ctx->partial_cap) {
         if (ctx->d_partials) cudaFree(ctx->d_partials);
         ctx->d_partials = nullptr;
@@ -425,6 +429,7 @@ int run(gsword_ctx* ctx, int method, int mode, uint64_t first, uint64_t count, u
     if ((mode & (3 | gsword::kModeSync | gsword::kModeStream)) == gsword::kModeEstimate) {
         mode |= occ_variant(ctx, method) << gsword::kModeOccShift;
         if (plan_is_tree(ctx->plan)) mode |= gsword::kModeTree;
+        if (method == GSWORD_ALLEY && refill_min_of(ctx, method) == 32) mode |= gsword::kModeLock;
     }
     LaunchCfg cfg;
     int rc = launch_config(ctx, method, mode, &cfg);
@@ -1326,6 +1331,7 @@ int gsword_query_info(gsword_ctx* ctx, gsword_query_stats* out) {
         if (ctx->opt_sched == 0 && !(m == GSWORD_ALLEY && ctx->opt_streaming)) {
             mode |= occ_variant(ctx, m) << gsword::kModeOccShift;
             if (plan_is_tree(ctx->plan)) mode |= gsword::kModeTree;
+            if (m == GSWORD_ALLEY && refill_min_of(ctx, m) == 32) mode |= gsword::kModeLock;
         }
         if (m == GSWORD_ALLEY && ctx->opt_streaming) mode |= gsword::kModeStream;
         if (ctx->opt_sched != 0) mode |= gsword::kModeSync;

@@ -61,7 +61,10 @@ __host__ __device__ constexpr int kOccBlocks(int method, int occ) {
 // TREE: every position d >= 1 has exactly one backward neighbour (a spanning-tree query
 // order, e.g. paths and stars): WanderJoin has no IsEdge validation and Alley only the
 // single-list refine, so the multi-list code is compiled out (estimate kernels only).
-template <int METHOD, int MODE, bool CG, bool SYNC, int OCC = 0, bool TREE = false>
+// LOCK: refill threshold 32 (a warp takes new samples only when all 32 lanes are free), so
+// every live lane of a warp is at the same depth: Alley's exclusion tests are the same set for
+// every lane and each lane runs its own, two in flight, without the task pool (estimate only).
+template <int METHOD, int MODE, bool CG, bool SYNC, int OCC = 0, bool TREE = false, bool LOCK = false>
 __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     sample_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
                                                      const uint64_t count, const uint64_t seed, const int chunk,
@@ -444,6 +447,26 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 }
                 known = cdup & qa;
                 unk = cdup & ~qa;
+                if (LOCK) {
+                    // depth-synchronous warp: this lane's own exclusion tests, two in flight
+                    // (the filter words of both, then the buckets of the "maybe"s), while the
+                    // segment load of S_p is still in flight
+                    const uint32_t a = Ms[p * T + tid];
+                    uint32_t m = unk;
+                    double unused = 0.0;
+                    while (m) {
+                        const int j0 = __ffs(m) - 1;
+                        m &= m - 1;
+                        const int j1 = m ? __ffs(m) - 1 : -1;
+                        if (m) m &= m - 1;
+                        const uint32_t x0 = Ms[j0 * T + tid], x1 = j1 >= 0 ? Ms[j1 * T + tid] : 0u;
+                        const bool f0 = bloom_maybe<false>(g, a, x0, unused);
+                        const bool f1 = j1 >= 0 && bloom_maybe<false>(g, a, x1, unused);
+                        if (f0 && is_edge_exact<false>(g, a, x0, ps.label, unused)) known |= 1u << j0;
+                        if (f1 && is_edge_exact<false>(g, a, x1, ps.label, unused)) known |= 1u << j1;
+                    }
+                    unk = 0u;
+                }
             }
             __syncwarp();
             // kind 2 is known before the pool for lanes that waited on GetMinCandidate, so the
@@ -507,7 +530,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                     msec += model_refine_sectors(g, Ms, T, tid, lo_p, len_p, ps.back & ~(1u << p), ps.dup, ps.label);
             }
             if (kind == 1) {
-                const uint32_t in_sp = known | pool_s[tid];  // matched vertices inside S_p
+                const uint32_t in_sp = LOCK ? known : (known | pool_s[tid]);  // matched vertices inside S_p
                 cnt = len_p - __popc(in_sp);
                 if (cnt > 0) {
                     const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
@@ -1550,17 +1573,20 @@ __global__ void scan_add_kernel(uint32_t* __restrict__ data, int64_t n, const ui
     if (i0 + 1 < n) data[i0 + 1] += add;
 }
 
-template <int METHOD, bool CG, bool TREE>
+template <int METHOD, bool CG, bool TREE, bool LOCK>
 const void* estimate_ptr(int occ) {
-    if (occ == 1) return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 1, TREE>);
-    if (occ == 2) return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 2, TREE>);
-    return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 0, TREE>);
+    if (occ == 1) return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 1, TREE, LOCK>);
+    if (occ == 2) return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 2, TREE, LOCK>);
+    return reinterpret_cast<const void*>(&sample_kernel<METHOD, kModeEstimate, CG, false, 0, TREE, LOCK>);
 }
 
 template <int METHOD, int MODE, bool CG>
-const void* kernel_ptr(bool sync, int occ = 0, bool tree = false) {
-    if (MODE == kModeEstimate && !sync)
-        return tree ? estimate_ptr<METHOD, CG, true>(occ) : estimate_ptr<METHOD, CG, false>(occ);
+const void* kernel_ptr(bool sync, int occ = 0, bool tree = false, bool lock = false) {
+    if (MODE == kModeEstimate && !sync) {
+        if (METHOD == GSWORD_ALLEY && lock)
+            return tree ? estimate_ptr<METHOD, CG, true, true>(occ) : estimate_ptr<METHOD, CG, false, true>(occ);
+        return tree ? estimate_ptr<METHOD, CG, true, false>(occ) : estimate_ptr<METHOD, CG, false, false>(occ);
+    }
     return sync ? reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE, CG, true>)
                 : reinterpret_cast<const void*>(&sample_kernel<METHOD, MODE, CG, false>);
 }
@@ -1574,6 +1600,7 @@ const void* select_kernel_cg(int method, int mode) {
     const bool sync = (mode & kModeSync) != 0;
     const int occ = (mode >> kModeOccShift) & 3;
     const bool tree = (mode & kModeTree) != 0;
+    const bool lock = (mode & kModeLock) != 0;
     mode &= 3;
     if (method == GSWORD_WJ) {
         if (mode == kModeTrace) return kernel_ptr<GSWORD_WJ, kModeTrace, CG>(sync);
@@ -1582,7 +1609,7 @@ const void* select_kernel_cg(int method, int mode) {
     }
     if (mode == kModeTrace) return kernel_ptr<GSWORD_ALLEY, kModeTrace, CG>(sync);
     if (mode == kModeCount) return kernel_ptr<GSWORD_ALLEY, kModeCount, CG>(sync);
-    return kernel_ptr<GSWORD_ALLEY, kModeEstimate, CG>(sync, occ, tree);
+    return kernel_ptr<GSWORD_ALLEY, kModeEstimate, CG>(sync, occ, tree, lock);
 }
 
 // mode: kMode* | kModeCG when the query was loaded with a candidate filter

@@ -217,7 +217,8 @@ enum Mode {
     kModeSync = 16,   // flag: a scheduling mode other than refill (GSWORD_OPT_SCHEDULE != 0)
     kModeOccShift = 5,  // bits 5-6: occupancy variant of the estimate kernel (0 default, 1 one
                         // CTA/SM less, 2 one more; refill schedule only), see occ_blocks()
-    kModeTree = 128     // flag: every position has one backward neighbour (estimate kernels)
+    kModeTree = 128,    // flag: every position has one backward neighbour (estimate kernels)
+    kModeLock = 256     // flag: Alley estimate with refill threshold 32 (depth-synchronous warps)
 };
 
 }  // namespace gsword

@@ -653,3 +653,38 @@ def test_fault_injection_queue_corruption_is_caught(ctx, G, c0):
     ctx.estimate_async(G.ALLEY, 0, n, 3, out)
     assert out.cpu().tolist()[3] == 0.0
     ctx.set_stream(None)
+
+
+@pytest.mark.parametrize("occ", [0, 1, 2])
+def test_refill32_depth_synchronous_kernel(ctx, G, c0, occ):
+    """Refill threshold 32 selects the depth-synchronous Alley estimate kernel (each lane runs
+    its own exclusion tests, no task pool; LOCK in gsword_kernels.cu): aggregates equal the
+    oracle's on C0, small random graphs, the three C1 queries and C2, for every occupancy
+    variant and the spanning-tree specialisation (paths)."""
+    ctx.set_option(G.OPT_AUTOTUNE, 0)
+    ctx.set_option(G.OPT_REFILL_MIN, 32)
+    ctx.set_option(G.OPT_OCCUPANCY, occ)
+    try:
+        cases = []
+        g, qs = c0
+        cases += [(g, q, 100_000) for q in qs]
+        for s in range(4):
+            gs = gen.random_small_graph(30, 0.4, 2, seed=900 + s)
+            cases.append((gs, gen.random_connected_query(6, 0.5, 2, 910 + s), 30_000))
+        g1, q1 = gen.config_c1()
+        cases += [(g1, q, 100_000) for q in q1]
+        g2, q2 = gen.config_c2()
+        cases += [(g2, q, 100_000) for q in q2]
+        loaded = None
+        for gg, q, n in cases:
+            if loaded is not gg:
+                ctx.load_graph_obj(gg)
+                loaded = gg
+            ctx.load_query_obj(q)
+            agg = ctx.estimate(G.ALLEY, n, seed=13, first=5)
+            y, _ = oracle.sample_range(gg, q, G.ALLEY, 13, 5, n, records=False, threads=8)
+            _agg_close(agg, oracle.aggregate(y), G)
+    finally:
+        ctx.set_option(G.OPT_AUTOTUNE, 1)
+        ctx.set_option(G.OPT_REFILL_MIN, 16)
+        ctx.set_option(G.OPT_OCCUPANCY, -1)
