@@ -1,5 +1,7 @@
 """Small estimate / trace runs for compute-sanitizer (memcheck, racecheck, synccheck,
-initcheck): both methods, every refine path (coop thresholds 0 and 64), trace mode."""
+initcheck): both methods, every refine path (coop thresholds 0 and 64), every occupancy
+variant, refill thresholds 16 and 32 (the depth-synchronous Alley kernel), trace and counting
+builds, and a query loaded with the NLF candidate graph (Fig. 4 layout build + sampling)."""
 import os
 import sys
 
@@ -22,8 +24,17 @@ with G.Context(0) as ctx:
             for m in (G.WJ, G.ALLEY):
                 for occ in (0, 1, 2):  # every occupancy variant of the estimate kernel
                     ctx.set_option(G.OPT_OCCUPANCY, occ)
-                    r = ctx.estimate(m, 20_000, 1)
+                    for rmin in (16, 32):  # 32: the depth-synchronous (LOCK) Alley kernel
+                        ctx.set_option(G.OPT_REFILL_MIN, rmin)
+                        r = ctx.estimate(m, 20_000, 1)
+                    ctx.set_option(G.OPT_REFILL_MIN, 16)
                 ctx.set_option(G.OPT_OCCUPANCY, -1)
                 rec = ctx.trace_samples(m, 0, 2000, 1)
                 s = ctx.count_sectors(m, 0, 2000, 1)
                 print(qq.name, m, coop, r["n_valid"], int(rec["valid"].sum()), s)
+    ctx.set_option(G.OPT_FILTER, 2)  # the candidate graph (three-CSR layout) build and its samplers
+    ctx.load_query_obj(q)
+    for m in (G.WJ, G.ALLEY):
+        r = ctx.estimate(m, 20_000, 1)
+        rec = ctx.trace_samples(m, 0, 2000, 1)
+        print("nlf", q.name, m, r["n_valid"], int(rec["valid"].sum()), ctx.query_info()["cg_bytes"])
