@@ -524,12 +524,14 @@ def run_ours(args):
     achieved = alg_bytes / dom_s / 1e9
     peak, peak_kind = measured_peaks()
     traffic = None
+    ncu_counters = None
     try:
         with open(args.traffic_file) as f:
             tf = json.load(f)
         if tf.get("workload") == WORKLOAD and name[dom] in tf.get("dram_bytes_per_sample", {}):
             # ncu --set full capture (cold cache, serialised) scaled to this launch's samples
             traffic = float(tf["dram_bytes_per_sample"][name[dom]]) * cnt
+            ncu_counters = dict(tf.get("counters", {}), source=tf.get("source"))
     except Exception:
         traffic = None
     # K5 random-gather rates of this device, measured now
@@ -545,6 +547,7 @@ def run_ours(args):
         "dram_frac": traffic / dom_s / 1e9 / peak if traffic else None,
         "gather_sectors_per_s": gather, "alg_sectors_per_s": sec_rate,
         "gather_frac": sec_rate / gather["l2_resident_64MB"], "gather_frac_hbm": sec_rate / gather["hbm_2GB"],
+        "ncu_counters": ncu_counters,
         "model": "reading A26 (DESIGN.md §3): offsets + drawn/selected vertices + Alley driver scans at "
                  "|B(d)|>=2 + one sector per membership question; counted by the kernel's counting build "
                  "over this launch, equal to the oracle's count (tests/test_gpu_sectors.py)",

@@ -51,7 +51,31 @@ for r in raw[2:]:
     traffic[k] = tb / samples
 out['_capture'] = {'report': rep, 'samples_per_launch': samples, 'workload': WORKLOAD}
 json.dump(out, open(out_path, 'w'), indent=1)
+
+
+def num(k, key):
+    v = out.get(k, {}).get(key)
+    return float(v.split()[0].replace(',', '')) if v else None
+
+
+# the counters the north star asks the design to be backed by, per sampling kernel
+counters = {}
+for k in ('wj', 'alley'):
+    if k not in out:
+        continue
+    counters[k] = {
+        "achieved_occupancy_pct": num(k, 'Achieved Occupancy'),
+        "active_threads_per_warp_instruction": num(k, 'smsp__thread_inst_executed_per_inst_executed.ratio'),
+        "warp_execution_efficiency": (num(k, 'smsp__thread_inst_executed_per_inst_executed.ratio') or 0) / 32.0,
+        "issue_slots_busy_pct": num(k, 'Issue Slots Busy'),
+        "eligible_warps_per_scheduler": num(k, 'Eligible Warps Per Scheduler'),
+        "l2_hit_rate_pct": num(k, 'lts__t_sector_hit_rate.pct'),
+        "l1_global_load_sectors_per_sample": (num(k, 'l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum') or 0) / samples,
+        "l2_sectors_per_sample": (num(k, 'lts__t_sectors.sum') or 0) / samples,
+        "dram_sectors_per_sample": traffic.get(k, 0.0) / 32.0,
+    }
 json.dump({"workload": WORKLOAD, "captured_samples_per_launch": samples, "dram_bytes_per_sample": traffic,
+           "counters": counters,
            "source": out_path + " (ncu --set full; dram__bytes_read.sum + dram__bytes_write.sum)"},
           open("profiles/traffic_latest.json", "w"), indent=1)
 print(json.dumps(out, indent=1))
