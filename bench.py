@@ -72,6 +72,10 @@ def parse():
     ap.add_argument("--quick", action="store_true", help="small config for smoke-testing the script")
     ap.add_argument("--no-qerror", action="store_true", help="skip the (untimed) C0 q-error leg")
     ap.add_argument("--no-cyclic", action="store_true", help="skip the cyclic-query leg")
+    # test aids for the N > 1 path on a one-GPU box (not bench numbers): every rank on cuda:0,
+    # gloo instead of NCCL (NCCL refuses two ranks on one device)
+    ap.add_argument("--dist-backend", choices=["nccl", "gloo"], default="nccl", help=argparse.SUPPRESS)
+    ap.add_argument("--same-device", action="store_true", help=argparse.SUPPRESS)
     return ap.parse_args()
 
 
@@ -317,7 +321,9 @@ def run_ours(args):
 
     # one process per GPU; a process group (NCCL) exists at every N, so the combine step
     # runs inside every timed step, a 1-rank all_reduce at N = 1
-    rank, world, local = init_from_env("nccl", single_rank_group=True)
+    if args.same_device:
+        os.environ["LOCAL_RANK"] = "0"
+    rank, world, local = init_from_env(args.dist_backend, single_rank_group=True)
     combine = dist.is_initialized()
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)

@@ -124,3 +124,36 @@ def test_estimate_distributed_under_a_one_rank_nccl_group():
         assert d["n"] == s["n"] and d["n_valid"] == s["n_valid"]
         assert d["sum"] == pytest.approx(s["sum"], rel=REL, abs=0.0)
         assert d["sumsq"] == pytest.approx(s["sumsq"], rel=REL, abs=0.0)
+
+
+def _bench_line(args, nproc):
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    common = ["bench.py", "--quick", "--steps", "2", "--warmup", "1", "--no-qerror", "--no-cpu-baseline",
+              "--no-cyclic"] + args
+    if nproc == 1:
+        cmd = [sys.executable] + common
+    else:
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
+               "--master-addr", "127.0.0.1", "--master-port", str(_free_port())] + common + ["--gpus", str(nproc)]
+    out = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=900)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, out.stdout[-2000:]
+    return json.loads(lines[0])
+
+
+def test_bench_two_ranks_on_one_gpu_matches_one_rank():
+    """bench.py's N > 1 path (graph broadcast over the process group, device-side graph load,
+    rank_range split, the all_reduce inside the timed step and inside e2e, max-over-ranks
+    timing) run as 2 ranks sharing cuda:0 over gloo: the combined estimates equal a one-rank
+    run over the same 4e6 sample ids."""
+    two = _bench_line(["--samples", "2e6", "--dist-backend", "gloo", "--same-device"], 2)
+    one = _bench_line(["--samples", "4e6"], 1)
+    assert two["n_gpus"] == 2 and one["n_gpus"] == 1 and two["value"] > 0 and two["e2e"]["value"] > 0
+    for m in ("wj", "alley"):
+        a, b = two["per_method"][m], one["per_method"][m]
+        assert a["valid_fraction"] == b["valid_fraction"]
+        assert a["estimate"] == pytest.approx(b["estimate"], rel=REL, abs=0.0)
