@@ -284,11 +284,38 @@ def run_reference(args):
 
 
 # ---------------------------------------------------------------- q-error
-def qerror_leg(G, ctx, args, samples: int = 100_000_000):
-    """q-error against the exact count where one exists: BASELINE configs[0] (C0), exact
-    counts from tests/golden/c0_exact_counts.txt (written by the oracle's enumerator).
+def star_count(g, s: int) -> int:
+    """Embeddings of the star K_{1,s} in an unlabelled graph: sum_v deg(v)^(falling s)
+    (the closed form pinned against brute force in tests/test_oracle_pins.py)."""
+    import numpy as np
+    deg = np.diff(g.row_ptr).astype(np.int64)
+    tot = 0
+    for dv in deg[deg >= s].tolist():
+        f = 1
+        for i in range(s):
+            f *= dv - i
+        tot += f
+    return tot
+
+
+def qerror_leg(G, ctx, args, g1=None, samples: int = 100_000_000):
+    """q-error against the exact count where one exists: the C1 graph (the bench's, still
+    loaded) with stars K_{1,3} and K_{1,4} (closed form), then BASELINE configs[0] (C0) with
+    exact counts from tests/golden/c0_exact_counts.txt (written by the oracle's enumerator).
     Untimed; runs after the timed region on the same context."""
     from workloads import gen
+    c1 = None
+    if g1 is not None:
+        c1 = {}
+        for s in (3, 4):
+            q = gen.star_query(s)
+            truth = star_count(g1, s)
+            ctx.load_query_obj(q)
+            for m, key in ((G.WJ, "wj"), (G.ALLEY, "alley")):
+                r = ctx.estimate(m, samples, args.seed)
+                c1[f"star{s}_{key}"] = {"exact": truth, "estimate": r["estimate"],
+                                        "qerror": G.qerror(truth, r["estimate"]),
+                                        "rel_std_err": (r["variance"] ** 0.5) / r["estimate"] if r["estimate"] else None}
     path = os.path.join(ROOT, "tests", "golden", "c0_exact_counts.txt")
     exact = {}
     for line in open(path):
@@ -306,7 +333,8 @@ def qerror_leg(G, ctx, args, samples: int = 100_000_000):
             errs.append(G.qerror(exact[q.name], r["estimate"]))
         out[key] = {"median": statistics.median(errs), "max": max(errs)}
     return {"config": "C0 (BASELINE configs[0]): 11 four-vertex queries", "samples_per_query": samples,
-            "exact_from": "tests/golden/c0_exact_counts.txt (oracle enumerator)", **out}
+            "exact_from": "tests/golden/c0_exact_counts.txt (oracle enumerator)", **out,
+            "c1_stars": c1, "c1_exact_from": "closed form sum_v deg(v)^(falling s) (SURVEY P5)"}
 
 
 # ---------------------------------------------------------------- our arm
@@ -574,7 +602,7 @@ def run_ours(args):
                                       "sample": f"{per1} + {per1} samples, {dt1:.1f} s"}}
 
     info = ctx.launch_info()
-    qerr = qerror_leg(G, ctx, args) if not (args.quick or args.no_qerror) else None
+    qerr = qerror_leg(G, ctx, args, g1=g) if not (args.quick or args.no_qerror) else None
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": 1e3 * max_time / args.steps, "higher_is_better": True,

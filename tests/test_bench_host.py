@@ -45,3 +45,14 @@ def test_clock_sampler_maps_the_device_by_uuid():
     nv = FakeNvml()
     c = bench.ClockSampler(3, uuid="GPU-1234", pci_bus_id="0000:1b:00.0")
     assert c._nvml_handle(nv) == "h-uuid" and nv.calls == [("uuid", "GPU-1234")]
+
+
+def test_star_count_closed_form():
+    # K_{1,s} embeddings = sum_v deg(v)^(falling s): K_6 (deg 5), ring C_7 (deg 2), star K_{1,4}
+    from workloads import gen
+    assert bench.star_count(gen.complete_graph(6), 3) == 6 * 5 * 4 * 3
+    assert bench.star_count(gen.ring_graph(7), 2) == 7 * 2 * 1
+    assert bench.star_count(gen.ring_graph(7), 3) == 0
+    g = gen.query_from_edges(5, [(0, i) for i in range(1, 5)])
+    star = gen.make_graph(5, [0, 0, 0, 0], [1, 2, 3, 4], None, 1)
+    assert bench.star_count(star, 4) == 4 * 3 * 2 * 1 and g.nq == 5
