@@ -720,3 +720,60 @@ def test_wanderjoin_alley_cross_check(ctx, G, c0):
             rel = lambda r: math.sqrt(max(r["variance"], 0.0)) / r["estimate"]
             assert rel(al) <= rel(wj), q.name
     assert agreed >= 8
+
+
+def test_stream_switch_orders_reused_buffers(ctx, G, c0):
+    """gsword_set_stream: work issued on a new stream starts after the context's
+    work on the old one (every launch reuses the queue, partials and output buffers).  A long
+    Alley estimate on stream A, a switch to stream B and a WanderJoin estimate there must give
+    the sequential results."""
+    import torch
+    g, qs = c0
+    ctx.load_graph_obj(g)
+    ctx.load_query_obj(qs[6])
+    ref_al = ctx.estimate(G.ALLEY, 30_000_000, seed=21)
+    ref_wj = ctx.estimate(G.WJ, 3_000_000, seed=22)
+    sa, sb = torch.cuda.Stream(), torch.cuda.Stream()
+    oa = torch.zeros(4, dtype=torch.float64, device="cuda:0")
+    ob = torch.zeros(4, dtype=torch.float64, device="cuda:0")
+    try:
+        ctx.set_stream(sa)
+        ctx.estimate_async(G.ALLEY, 0, 30_000_000, 21, oa)
+        ctx.set_stream(sb)
+        ctx.estimate_async(G.WJ, 0, 3_000_000, 22, ob)
+        sa.synchronize()
+        sb.synchronize()
+    finally:
+        ctx.set_stream(None)
+    for out, ref in ((oa, ref_al), (ob, ref_wj)):
+        r = G.finalize(out.cpu().numpy())
+        assert r["n"] == ref["n"] and r["n_valid"] == ref["n_valid"]
+        assert r["sum"] == pytest.approx(ref["sum"], rel=REL, abs=0.0)
+
+
+def test_two_contexts_run_concurrently(G, c0):
+    """Two contexts on one device (e.g. two serving workers) on their own streams, launched
+    back to back without host synchronisation: both results equal the sequential ones."""
+    import torch
+    g, qs = c0
+    with G.Context(0) as c1, G.Context(0) as c2:
+        for c in (c1, c2):
+            c.load_graph_obj(g)
+        c1.load_query_obj(qs[0])
+        c2.load_query_obj(qs[7])
+        ref1 = c1.estimate(G.ALLEY, 20_000_000, seed=5)
+        ref2 = c2.estimate(G.WJ, 20_000_000, seed=6)
+        s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+        o1 = torch.zeros(4, dtype=torch.float64, device="cuda:0")
+        o2 = torch.zeros(4, dtype=torch.float64, device="cuda:0")
+        c1.set_stream(s1)
+        c2.set_stream(s2)
+        c1.estimate_async(G.ALLEY, 0, 20_000_000, 5, o1)
+        c2.estimate_async(G.WJ, 0, 20_000_000, 6, o2)
+        torch.cuda.synchronize()
+        for out, ref in ((o1, ref1), (o2, ref2)):
+            r = G.finalize(out.cpu().numpy())
+            assert r["n"] == ref["n"] and r["n_valid"] == ref["n_valid"]
+            assert r["sum"] == pytest.approx(ref["sum"], rel=REL, abs=0.0)
+        c1.set_stream(None)
+        c2.set_stream(None)
