@@ -698,7 +698,7 @@ int build_candidate_graph(gsword_ctx* ctx, int32_t nq, const int32_t* q_row_ptr,
 
 extern "C" {
 
-int gsword_version(void) { return 100; }
+int gsword_version(void) { return 200; }  // 2.00: A26 sectors in records, count_sectors(model, touched), EFAULT, cg_bytes
 
 const char* gsword_last_error(void) { return g_last_error.c_str(); }
 
