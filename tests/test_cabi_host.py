@@ -30,7 +30,7 @@ def test_library_exports_every_declared_symbol():
 
 
 def test_version():
-    assert G.version() == 100
+    assert G.version() == 200
 
 
 def test_check_graph_accepts_canonical(c0):
