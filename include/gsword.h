@@ -176,7 +176,7 @@ typedef enum {
                                    /* synchronisation; default 16); no effect on    */
                                    /* results                                         */
     GSWORD_OPT_AUTOTUNE = 10,      /* 1 (default): gsword_load_query times pilots of   */
-                                   /* refill thresholds 8/16/24/32 per method and     */
+                                   /* refill thresholds 8/16/24/28/32 per method and  */
                                    /* keeps the fastest, then times the estimate      */
                                    /* kernel compiled for one CTA/SM less and one     */
                                    /* more (register budget vs occupancy) at that     */

@@ -1247,14 +1247,14 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
     }
     if (ctx->opt_autotune && ctx->opt_sched == 0 && ctx->tuned_refill[0] == 0) {
         // schedule autotune (no effect on any result).  Phase 1: refill thresholds
-        // 16/8/24/32 (samples of long-lived walks favour depth-synchronous warps, short-lived
+        // 16/8/24/32/28 (samples of long-lived walks favour depth-synchronous warps, short-lived
         // ones frequent refills).  Phase 2, at the chosen threshold: the
         // estimate kernel compiled for one CTA/SM less (more registers, fewer spills) and one
         // more.  Every candidate is timed over the same id range of `big` samples, preceded
         // by a warm-up over a range of its own (short or repeated pilots favour whichever
         // candidate profits from the tail or from a warm L2); each phase queues its runs back
         // to back on the context stream, timed by events, with one host synchronisation.
-        static const int cand[4] = {16, 8, 24, 32};
+        static const int cand[5] = {16, 8, 24, 32, 28};  // 28: C1 dense Alley (profiles/r02_refill_sweep.jsonl)
         const uint64_t big = 8000000, warm = 1000000, range0 = 1ull << 40;
         int rc2 = GSWORD_OK;
         cudaError_t e = cudaSuccess;
@@ -1264,8 +1264,8 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
             if (e == cudaSuccess) evs.push_back(*out);
         };
         // times[m][c] for candidate c of method m; sets tuned_* before each run
-        auto time_phase = [&](int ncand, auto&& apply, float (*times)[4]) {
-            cudaEvent_t ev[2][4][2];
+        auto time_phase = [&](int ncand, auto&& apply, float (*times)[5]) {
+            cudaEvent_t ev[2][5][2];
             for (int m = 0; m < 2 && rc2 == GSWORD_OK && e == cudaSuccess; ++m)
                 for (int c = 0; c < ncand && rc2 == GSWORD_OK && e == cudaSuccess; ++c) {
                     apply(m, c);
@@ -1283,12 +1283,12 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
                 for (int c = 0; c < ncand && e == cudaSuccess; ++c)
                     e = cudaEventElapsedTime(&times[m][c], ev[m][c][0], ev[m][c][1]);
         };
-        float t1[2][4] = {}, t2[2][4] = {};
-        time_phase(4, [&](int m, int c) { ctx->tuned_refill[m] = cand[c]; }, t1);
+        float t1[2][5] = {}, t2[2][5] = {};
+        time_phase(5, [&](int m, int c) { ctx->tuned_refill[m] = cand[c]; }, t1);
         float best[2] = {0.f, 0.f};
         for (int m = 0; m < 2; ++m) {
             int bc = 0;
-            for (int c = 1; c < 4; ++c)
+            for (int c = 1; c < 5; ++c)
                 if (t1[m][c] < t1[m][bc]) bc = c;
             ctx->tuned_refill[m] = cand[bc];
             best[m] = t1[m][bc];
@@ -1297,7 +1297,7 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
         for (int m = 0; m < 2; ++m) {
             ctx->tuned_occ[m] = 0;
             for (int c = 0; c < 2 && ctx->opt_occ < 0; ++c)
-                if (t2[m][c] < 0.985f * best[m]) {  // a variant must win by 1.5 % (pilot noise)
+                if (t2[m][c] < 0.99f * best[m]) {  // a variant must win by 1 % (pilot noise)
                     best[m] = t2[m][c];
                     ctx->tuned_occ[m] = 1 + c;
                 }

@@ -584,7 +584,7 @@ def test_autotune_does_not_change_results(ctx, G, c0):
     ctx.set_option(G.OPT_AUTOTUNE, 1)
     ctx.load_query_obj(q)
     info = ctx.query_info()
-    assert all(r in (8, 16, 24, 32) for r in info["refill_min"])
+    assert all(r in (8, 16, 24, 28, 32) for r in info["refill_min"])
     assert info["occupancy"][0] in (5, 6, 7) and info["occupancy"][1] in (4, 5, 6)
     for m in (0, 1):
         assert ctx.trace_samples(m, 0, 30_000, 4).tobytes() == ref[m].tobytes()
