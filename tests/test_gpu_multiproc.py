@@ -126,14 +126,14 @@ def test_estimate_distributed_under_a_one_rank_nccl_group():
         assert d["sumsq"] == pytest.approx(s["sumsq"], rel=REL, abs=0.0)
 
 
-def _bench_line(args, nproc):
+def _bench_line(args, nproc, torchrun=False):
     import json
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     common = ["bench.py", "--quick", "--steps", "2", "--warmup", "1", "--no-qerror", "--no-cpu-baseline",
               "--no-cyclic"] + args
-    if nproc == 1:
+    if nproc == 1 and not torchrun:
         cmd = [sys.executable] + common
     else:
         cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
@@ -157,3 +157,16 @@ def test_bench_two_ranks_on_one_gpu_matches_one_rank():
         a, b = two["per_method"][m], one["per_method"][m]
         assert a["valid_fraction"] == b["valid_fraction"]
         assert a["estimate"] == pytest.approx(b["estimate"], rel=REL, abs=0.0)
+
+
+def test_bench_under_torchrun_with_one_rank():
+    """The driver's N = 1 launch form (torch.distributed.run, one rank): bench.py joins the
+    launcher's store with a 1-rank NCCL group, runs the all_reduce in the step, and prints
+    one line equal to the plain run's estimates; the reference arm prints its line too."""
+    tr = _bench_line(["--samples", "2e6"], 1, torchrun=True)
+    plain = _bench_line(["--samples", "2e6"], 1)
+    assert tr["n_gpus"] == 1 and "NCCL" in tr["config"]["combine"]
+    for m in ("wj", "alley"):
+        assert tr["per_method"][m]["estimate"] == pytest.approx(plain["per_method"][m]["estimate"], rel=REL, abs=0.0)
+    ref = _bench_line(["--impl", "reference", "--cpu-samples", "2000"], 1, torchrun=True)
+    assert ref["impl"] == "reference" and ref["value"] > 0
