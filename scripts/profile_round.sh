@@ -11,7 +11,7 @@ cd "$(dirname "$0")/.."
 TAG=${1:-latest}
 mkdir -p gpurun_out profiles
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
-    --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline \
+    --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-qerror --no-cyclic \
     > gpurun_out/${TAG}_launches_bench.log 2>&1
 # profile_driver brackets the two bench-size launches with cudaProfilerStart/Stop
 timeout 900 ncu --set full --import-source on --clock-control none --profile-from-start off -k regex:sample_kernel -c 2 \
