@@ -42,6 +42,97 @@ using namespace dev;
 #endif
 // Alley drivers longer than the coop threshold (<= 64) are refined by the whole warp.
 
+// Warp-cooperative Alley refine + sample of one lane's long driver run clist[Llo, Llo+Llen)
+// (Fig. 19 AL; reading A5): 32 coalesced elements per round, each lane tests its
+// element against the other lists (`others`, the matched vertices of column colL) and the
+// matched same-label vertices, `ballot` -> the chunk's survivor mask, held in lane c for chunk c
+// (lists <= 1024) -> warp prefix sum of popcounts -> find-nth of the k-th survivor; longer lists
+// keep per-lane group counts (G chunks per group) and re-test only the group holding the k-th.
+// Deterministic replacement of the paper's reservoir warp streaming.  Every lane calls it;
+// total (|C_d|) and chosen (the drawn vertex, -1 if none) are returned to every lane.
+template <bool COUNT>
+__device__ __forceinline__ void coop_refine(const DeviceGraph& g, const uint32_t* Ms, int T, int lane, int colL,
+                                            uint32_t Llo, uint32_t Llen, uint32_t others, const PlanStep& Lps,
+                                            uint32_t Lsig, uint32_t Lr_lo, uint32_t Lr_hi, double& sectors,
+                                            uint32_t& total_out, int32_t& chosen_out) {
+    uint32_t total = 0, my_bal = 0;
+    // lists longer than 32 chunks: lane g also counts the survivors of chunk group
+    // g (G consecutive chunks), so the draw re-tests one group, not the whole prefix
+    const uint32_t G = (((Llen + 31u) >> 5) + 31u) >> 5;  // chunks per group
+    const uint32_t g_lo = (uint32_t)lane * G;
+    uint32_t gcnt = 0;
+    // the next chunk's driver elements are loaded while this chunk is tested
+    int32_t xn = ((uint32_t)lane < Llen) ? ldg_i32(g.clist + Llo + lane) : 0;
+    for (uint32_t base = 0; base < Llen; base += 32) {
+        const uint32_t i = base + lane;
+        bool keep = i < Llen;
+        const int32_t x = xn;
+        if (i + 32u < Llen) xn = ldg_i32(g.clist + Llo + i + 32u);
+        if (keep) {
+            keep = member_all<COUNT>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
+                   not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x);
+        }
+        const unsigned bal = __ballot_sync(kFull, keep);
+        if ((base >> 5) == (uint32_t)lane) my_bal = bal;
+        if ((base >> 5) - g_lo < G) gcnt += __popc(bal);
+        total += __popc(bal);
+    }
+    int32_t chosen = -1;
+    if (total > 0) {
+        const uint64_t Lr = ((uint64_t)Lr_hi << 32) | Lr_lo;
+        const uint32_t k = (uint32_t)__umul64hi(Lr, (uint64_t)total);
+        if (Llen <= 32u * 32u) {
+            // lane c holds the ballot of chunk c: warp scan of popcounts
+            const uint32_t pc = __popc(my_bal);
+            uint32_t incl = pc;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, incl, o);
+                if (lane >= o) incl += y;
+            }
+            const uint32_t excl = incl - pc;
+            const bool here = (k >= excl) && (k < incl);
+            const unsigned hm = __ballot_sync(kFull, here);
+            const int c = __ffs(hm) - 1;
+            int32_t val = 0;
+            if (lane == c) val = ldg_i32(g.clist + Llo + (uint32_t)c * 32u + fns32(my_bal, k - excl));
+            chosen = __shfl_sync(kFull, val, c);
+        } else {
+            // the group holding the k-th survivor (warp scan of the group counts),
+            // then its chunks re-tested in order
+            uint32_t incl = gcnt;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, incl, o);
+                if (lane >= o) incl += y;
+            }
+            const unsigned hm = __ballot_sync(kFull, (k >= incl - gcnt) && (k < incl));
+            const int gs = __ffs(hm) - 1;
+            uint32_t run = __shfl_sync(kFull, incl - gcnt, gs);
+            const uint32_t b0 = (uint32_t)gs * G * 32u;
+            for (uint32_t base = b0; base < Llen; base += 32) {
+                const uint32_t i = base + lane;
+                bool keep = i < Llen;
+                int32_t x = 0;
+                if (keep) {
+                    x = ldg_i32(g.clist + Llo + i);
+                    keep = member_all<COUNT>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
+                           not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x);
+                }
+                const unsigned bal = __ballot_sync(kFull, keep);
+                const uint32_t c = __popc(bal);
+                if (run + c > k) {
+                    chosen = __shfl_sync(kFull, x, (int)fns32(bal, k - run));
+                    break;
+                }
+                run += c;
+            }
+        }
+    }
+    total_out = total;
+    chosen_out = chosen;
+}
+
 #ifndef GSWORD_WJ_MIN_BLOCKS
 #define GSWORD_WJ_MIN_BLOCKS 6  // 42 registers: 48 warps per SM (measured best)
 #endif
@@ -620,80 +711,10 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 const uint32_t others = Lps.back & ~(1u << Lp);
                 const int colL = wbase + L;
                 const uint32_t Lsig = __shfl_sync(kFull, msig, L);
-                uint32_t total = 0, my_bal = 0;
-                // lists longer than 32 chunks: lane g also counts the survivors of chunk group
-                // g (G consecutive chunks), so the draw re-tests one group, not the whole prefix
-                const uint32_t G = (((Llen + 31u) >> 5) + 31u) >> 5;  // chunks per group
-                const uint32_t g_lo = (uint32_t)lane * G;
-                uint32_t gcnt = 0;
-                // the next chunk's driver elements are loaded while this chunk is tested
-                int32_t xn = ((uint32_t)lane < Llen) ? ldg_i32(g.clist + Llo + lane) : 0;
-                for (uint32_t base = 0; base < Llen; base += 32) {
-                    const uint32_t i = base + lane;
-                    bool keep = i < Llen;
-                    const int32_t x = xn;
-                    if (i + 32u < Llen) xn = ldg_i32(g.clist + Llo + i + 32u);
-                    if (keep) {
-                        keep = member_all<MODE == kModeCount>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
-                               not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x);
-                    }
-                    const unsigned bal = __ballot_sync(kFull, keep);
-                    if ((base >> 5) == (uint32_t)lane) my_bal = bal;
-                    if ((base >> 5) - g_lo < G) gcnt += __popc(bal);
-                    total += __popc(bal);
-                }
-                int32_t chosen = -1;
-                if (total > 0) {
-                    const uint64_t Lr = ((uint64_t)Lr_hi << 32) | Lr_lo;
-                    const uint32_t k = (uint32_t)__umul64hi(Lr, (uint64_t)total);
-                    if (Llen <= 32u * 32u) {
-                        // lane c holds the ballot of chunk c: warp scan of popcounts
-                        const uint32_t pc = __popc(my_bal);
-                        uint32_t incl = pc;
-#pragma unroll
-                        for (int o = 1; o < 32; o <<= 1) {
-                            const uint32_t y = __shfl_up_sync(kFull, incl, o);
-                            if (lane >= o) incl += y;
-                        }
-                        const uint32_t excl = incl - pc;
-                        const bool here = (k >= excl) && (k < incl);
-                        const unsigned hm = __ballot_sync(kFull, here);
-                        const int c = __ffs(hm) - 1;
-                        int32_t val = 0;
-                        if (lane == c) val = ldg_i32(g.clist + Llo + (uint32_t)c * 32u + fns32(my_bal, k - excl));
-                        chosen = __shfl_sync(kFull, val, c);
-                    } else {
-                        // the group holding the k-th survivor (warp scan of the group counts),
-                        // then its chunks re-tested in order
-                        uint32_t incl = gcnt;
-#pragma unroll
-                        for (int o = 1; o < 32; o <<= 1) {
-                            const uint32_t y = __shfl_up_sync(kFull, incl, o);
-                            if (lane >= o) incl += y;
-                        }
-                        const unsigned hm = __ballot_sync(kFull, (k >= incl - gcnt) && (k < incl));
-                        const int gs = __ffs(hm) - 1;
-                        uint32_t run = __shfl_sync(kFull, incl - gcnt, gs);
-                        const uint32_t b0 = (uint32_t)gs * G * 32u;
-                        for (uint32_t base = b0; base < Llen; base += 32) {
-                            const uint32_t i = base + lane;
-                            bool keep = i < Llen;
-                            int32_t x = 0;
-                            if (keep) {
-                                x = ldg_i32(g.clist + Llo + i);
-                                keep = member_all<MODE == kModeCount>(g, Ms, T, colL, others, Lps.label, x, sectors) &&
-                                       not_matched_sig(Ms, T, colL, Lps.dup, Lsig, x);
-                            }
-                            const unsigned bal = __ballot_sync(kFull, keep);
-                            const uint32_t c = __popc(bal);
-                            if (run + c > k) {
-                                chosen = __shfl_sync(kFull, x, (int)fns32(bal, k - run));
-                                break;
-                            }
-                            run += c;
-                        }
-                    }
-                }
+                uint32_t total;
+                int32_t chosen;
+                coop_refine<MODE == kModeCount>(g, Ms, T, lane, colL, Llo, Llen, others, Lps, Lsig, Lr_lo, Lr_hi, sectors,
+                                                total, chosen);
                 if (lane == L) {
                     cnt = total;
                     v = chosen;
