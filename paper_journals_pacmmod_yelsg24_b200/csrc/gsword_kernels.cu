@@ -133,6 +133,122 @@ __device__ __forceinline__ void coop_refine(const DeviceGraph& g, const uint32_t
     chosen_out = chosen;
 }
 
+// A10: the CTA's partial in a fixed order.  Each lane's Neumaier pair becomes a double-double,
+// a warp butterfly adds the lanes, lane 0 of every warp stores the warp's partial in
+// warp_part[warp], and thread 0 adds the warps in warp order into partials[blockIdx.x].
+// Every thread of the CTA calls it (it synchronises the CTA).
+__device__ __forceinline__ void write_cta_partial(Partial* warp_part, Partial* __restrict__ partials, double s_sum,
+                                                  double c_sum, double s_sq, double c_sq, unsigned long long valid,
+                                                  unsigned long long n, double sectors, double model) {
+    const int tid = threadIdx.x, lane = tid & 31;
+    double sh = __dadd_rn(s_sum, c_sum), sl = __dsub_rn(c_sum, __dsub_rn(sh, s_sum));
+    double qh = __dadd_rn(s_sq, c_sq), ql = __dsub_rn(c_sq, __dsub_rn(qh, s_sq));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const double bh = shfl_xor_d(sh, o), bl = shfl_xor_d(sl, o);
+        const double ch = shfl_xor_d(qh, o), cl = shfl_xor_d(ql, o);
+        dd_add(sh, sl, bh, bl);
+        dd_add(qh, ql, ch, cl);
+        valid += __shfl_xor_sync(kFull, valid, o);
+        n += __shfl_xor_sync(kFull, n, o);
+        sectors += shfl_xor_d(sectors, o);
+        model += shfl_xor_d(model, o);
+    }
+    if (lane == 0) warp_part[tid >> 5] = Partial{sh, sl, qh, ql, valid, n, sectors, model};
+    __syncthreads();
+    if (tid == 0) {
+        Partial acc = warp_part[0];
+        for (int w = 1; w < (int)(blockDim.x >> 5); ++w) {
+            const Partial& o = warp_part[w];
+            dd_add(acc.sum_hi, acc.sum_lo, o.sum_hi, o.sum_lo);
+            dd_add(acc.sq_hi, acc.sq_lo, o.sq_hi, o.sq_lo);
+            acc.valid += o.valid;
+            acc.n += o.n;
+            acc.sectors += o.sectors;
+            acc.model += o.model;
+        }
+        partials[blockIdx.x] = acc;
+    }
+}
+
+// Alley single-list select (|B(d)| = 1): the k-th (0-based) element of the ascending run
+// clist[lo, ...) that is not one of the matched vertices in the position mask X (all of which
+// lie in the run): the smallest idx with idx = k + #{x in X : x <= run[idx]}.  With at most two
+// excluded vertices idx lies in [k, k + |X|]: that window is loaded at once and the fixed point
+// found in registers (one memory round trip instead of up to |X| + 1 dependent ones).
+// Ms_lane = this lane's column of the matched vertices (row stride T).
+__device__ __forceinline__ int32_t select_excluding(const DeviceGraph& g, const uint32_t* Ms_lane, int T, uint32_t lo,
+                                                    uint32_t k, uint32_t X) {
+    const int nx = __popc(X);
+#if GSWORD_SELECT_WINDOW
+    if (nx <= 2) {
+        const int32_t* wb = g.clist + lo + k;
+        const int32_t w0 = ldg_i32(wb);
+        const int32_t w1 = nx >= 1 ? ldg_i32(wb + 1) : 0;
+        const int32_t w2 = nx >= 2 ? ldg_i32(wb + 2) : 0;
+        const int32_t x0 = nx >= 1 ? (int32_t)Ms_lane[(__ffs(X) - 1) * T] : INT32_MAX;
+        const int32_t x1 = nx >= 2 ? (int32_t)Ms_lane[(31 - __clz(X)) * T] : INT32_MAX;
+        uint32_t i = 0;
+#pragma unroll
+        for (int it = 0; it < 2; ++it) {
+            const int32_t wi = i == 0 ? w0 : (i == 1 ? w1 : w2);
+            i = (uint32_t)(x0 <= wi) + (uint32_t)(x1 <= wi);
+        }
+        return i == 0 ? w0 : (i == 1 ? w1 : w2);
+    }
+#endif
+    int32_t v = 0;
+    for (uint32_t idx = k;;) {
+        v = ldg_i32(g.clist + lo + idx);
+        uint32_t c = 0, xm = X;
+        while (xm) {
+            const int j = __ffs(xm) - 1;
+            xm &= xm - 1;
+            c += ((int32_t)Ms_lane[j * T] <= v) ? 1u : 0u;
+        }
+        if (idx == k + c) break;
+        idx = k + c;
+    }
+    return v;
+}
+
+// Alley short-driver refine (|B(d)| >= 2, |S_p| <= the cooperative threshold, <= 128): the
+// refine mask over clist[lo, lo + len) is "not removed by a pooled membership test" (pool rows
+// 1..4 of this lane, bit set = removed) and "not a matched same-label vertex" (injectivity, dup
+// mask, signature sig); returns |C_d| and writes the k-th survivor (k = mulhi64(r, |C_d|)) to *v.
+__device__ __forceinline__ uint32_t refine_mask_select(const DeviceGraph& g, const uint32_t* Ms_lane,
+                                                       const uint32_t* pool_lane, int T, uint32_t lo, uint32_t len,
+                                                       uint32_t dup, uint32_t sig, uint64_t r, int32_t* v) {
+    uint32_t keep[4];
+    uint32_t cnt = 0;
+#pragma unroll
+    for (int w = 0; w < 4; ++w) {
+        const uint32_t n_w = (len > 32u * w) ? min(len - 32u * w, 32u) : 0u;
+        uint32_t m = (n_w == 32u) ? 0xFFFFFFFFu : ((1u << n_w) - 1u);
+        if (n_w) m &= ~pool_lane[(1 + w) * T];
+        uint32_t mm = dup ? m : 0u;
+        while (mm) {
+            const int i = __ffs(mm) - 1;
+            mm &= mm - 1;
+            if (!not_matched_sig(Ms_lane, T, 0, dup, sig, ldg_i32(g.clist + lo + 32u * w + i))) m &= ~(1u << i);
+        }
+        keep[w] = m;
+        cnt += __popc(m);
+    }
+    if (cnt > 0) {
+        uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
+        uint32_t pos = 0;
+#pragma unroll
+        for (int w = 0; w < 4; ++w) {
+            const uint32_t c = __popc(keep[w]);
+            if (k < c && pos == 0u) pos = 32u * w + fns32(keep[w], k) + 1u;  // +1: found marker
+            if (pos == 0u) k -= c;
+        }
+        *v = ldg_i32(g.clist + lo + pos - 1u);
+    }
+    return cnt;
+}
+
 #ifndef GSWORD_WJ_MIN_BLOCKS
 #define GSWORD_WJ_MIN_BLOCKS 6  // 42 registers: 48 warps per SM (measured best)
 #endif
@@ -624,74 +740,11 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 const uint32_t in_sp = LOCK ? known : (known | pool_s[tid]);  // matched vertices inside S_p
                 cnt = len_p - __popc(in_sp);
                 if (cnt > 0) {
-                    const uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
-                    // smallest idx with idx = k + #{x in X : x <= S_p[idx]}: the k-th survivor
-                    const int nx = __popc(in_sp);
-#if GSWORD_SELECT_WINDOW
-                    if (nx <= 2) {
-                        // idx lies in [k, k + nx] (inside S_p since cnt = len_p - nx > k): load
-                        // that window at once and find the fixed point in registers (one
-                        // memory round trip instead of up to nx + 1 dependent ones)
-                        const int32_t* wb = g.clist + lo_p + k;
-                        const int32_t w0 = ldg_i32(wb);
-                        const int32_t w1 = nx >= 1 ? ldg_i32(wb + 1) : 0;
-                        const int32_t w2 = nx >= 2 ? ldg_i32(wb + 2) : 0;
-                        const int32_t x0 = nx >= 1 ? (int32_t)Ms[(__ffs(in_sp) - 1) * T + tid] : INT32_MAX;
-                        const int32_t x1 = nx >= 2 ? (int32_t)Ms[(31 - __clz(in_sp)) * T + tid] : INT32_MAX;
-                        uint32_t i = 0;
-#pragma unroll
-                        for (int it = 0; it < 2; ++it) {
-                            const int32_t wi = i == 0 ? w0 : (i == 1 ? w1 : w2);
-                            i = (uint32_t)(x0 <= wi) + (uint32_t)(x1 <= wi);
-                        }
-                        v = i == 0 ? w0 : (i == 1 ? w1 : w2);
-                    } else
-#endif
-                    for (uint32_t idx = k;;) {
-                        v = ldg_i32(g.clist + lo_p + idx);
-                        uint32_t c = 0, xm = in_sp;
-                        while (xm) {
-                            const int j = __ffs(xm) - 1;
-                            xm &= xm - 1;
-                            c += ((int32_t)Ms[j * T + tid] <= v) ? 1u : 0u;
-                        }
-                        if (idx == k + c) break;
-                        idx = k + c;
-                    }
+                    v = select_excluding(g, Ms + tid, T, lo_p, (uint32_t)__umul64hi(r, (uint64_t)cnt), in_sp);
                     if (MODE == kModeCount) sectors += 1.0;
                 }
             } else if (!TREE && kind == 2) {
-                // refine mask over S_p (<= 128 elements, 4 words): not removed by a membership
-                // test and not a matched same-label vertex (injectivity)
-                const uint32_t dup = ps.dup & ~(1u << p);
-                uint32_t keep[4];
-                cnt = 0;
-#pragma unroll
-                for (int w = 0; w < 4; ++w) {
-                    const uint32_t n_w = (len_p > 32u * w) ? min(len_p - 32u * w, 32u) : 0u;
-                    uint32_t m = (n_w == 32u) ? 0xFFFFFFFFu : ((1u << n_w) - 1u);
-                    if (n_w) m &= ~pool_s[(1 + w) * T + tid];
-                    uint32_t mm = dup ? m : 0u;
-                    while (mm) {
-                        const int i = __ffs(mm) - 1;
-                        mm &= mm - 1;
-                        if (!not_matched_sig(Ms + tid, T, 0, dup, msig, ldg_i32(g.clist + lo_p + 32u * w + i)))
-                            m &= ~(1u << i);
-                    }
-                    keep[w] = m;
-                    cnt += __popc(m);
-                }
-                if (cnt > 0) {
-                    uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
-                    uint32_t pos = 0;
-#pragma unroll
-                    for (int w = 0; w < 4; ++w) {
-                        const uint32_t c = __popc(keep[w]);
-                        if (k < c && pos == 0u) pos = 32u * w + fns32(keep[w], k) + 1u;  // +1: found marker
-                        if (pos == 0u) k -= c;
-                    }
-                    v = ldg_i32(g.clist + lo_p + pos - 1u);
-                }
+                cnt = refine_mask_select(g, Ms + tid, pool_s + tid, T, lo_p, len_p, ps.dup & ~(1u << p), msig, r, &v);
             }
             const bool coop = !TREE && (kind == 3);
             mark(5);
@@ -816,37 +869,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
         n_done = (lane == 0) ? wq_s[tid >> 5][2] : 0ull;
     }
     // ---------------- A10: warp -> CTA partial, fixed order ----------------
-    double sh = __dadd_rn(s_sum, c_sum), sl = __dsub_rn(c_sum, __dsub_rn(sh, s_sum));
-    double qh = __dadd_rn(s_sq, c_sq), ql = __dsub_rn(c_sq, __dsub_rn(qh, s_sq));
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        const double bh = shfl_xor_d(sh, o), bl = shfl_xor_d(sl, o);
-        const double ch = shfl_xor_d(qh, o), cl = shfl_xor_d(ql, o);
-        dd_add(sh, sl, bh, bl);
-        dd_add(qh, ql, ch, cl);
-        n_valid += __shfl_xor_sync(kFull, n_valid, o);
-        n_done += __shfl_xor_sync(kFull, n_done, o);
-        sectors += shfl_xor_d(sectors, o);
-        msum += shfl_xor_d(msum, o);
-    }
-    const int warp = tid >> 5;
-    if (lane == 0) {
-        warp_part[warp] = Partial{sh, sl, qh, ql, n_valid, n_done, sectors, msum};
-    }
-    __syncthreads();
-    if (tid == 0) {
-        Partial acc = warp_part[0];
-        for (int w = 1; w < (T >> 5); ++w) {
-            const Partial& o = warp_part[w];
-            dd_add(acc.sum_hi, acc.sum_lo, o.sum_hi, o.sum_lo);
-            dd_add(acc.sq_hi, acc.sq_lo, o.sq_hi, o.sq_lo);
-            acc.valid += o.valid;
-            acc.n += o.n;
-            acc.sectors += o.sectors;
-            acc.model += o.model;
-        }
-        partials[blockIdx.x] = acc;
-    }
+    write_cta_partial(warp_part, partials, s_sum, c_sum, s_sq, c_sq, n_valid, n_done, sectors, msum);
 }
 
 // ---------------------------------------------------------------- warp streaming (NEXT-3)
@@ -1108,31 +1131,7 @@ __global__ void __launch_bounds__(256) stream_kernel(const DeviceGraph g, const 
     }
 
     // ---------------- A10: warp -> CTA partial, fixed order ----------------
-    double sh = __dadd_rn(s_sum, c_sum), sl = __dsub_rn(c_sum, __dsub_rn(sh, s_sum));
-    double qh = __dadd_rn(s_sq, c_sq), ql = __dsub_rn(c_sq, __dsub_rn(qh, s_sq));
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        const double bh = shfl_xor_d(sh, o), bl = shfl_xor_d(sl, o);
-        const double ch = shfl_xor_d(qh, o), cl = shfl_xor_d(ql, o);
-        dd_add(sh, sl, bh, bl);
-        dd_add(qh, ql, ch, cl);
-        n_valid += __shfl_xor_sync(kFull, n_valid, o);
-        n_done += __shfl_xor_sync(kFull, n_done, o);
-    }
-    const int warp = tid >> 5;
-    if (lane == 0) warp_part[warp] = Partial{sh, sl, qh, ql, n_valid, n_done, 0.0, 0.0};
-    __syncthreads();
-    if (tid == 0) {
-        Partial acc = warp_part[0];
-        for (int w = 1; w < (T >> 5); ++w) {
-            const Partial& o = warp_part[w];
-            dd_add(acc.sum_hi, acc.sum_lo, o.sum_hi, o.sum_lo);
-            dd_add(acc.sq_hi, acc.sq_lo, o.sq_hi, o.sq_lo);
-            acc.valid += o.valid;
-            acc.n += o.n;
-        }
-        partials[blockIdx.x] = acc;
-    }
+    write_cta_partial(warp_part, partials, s_sum, c_sum, s_sq, c_sq, n_valid, n_done, 0.0, 0.0);
 }
 
 // ---------------------------------------------------------------- trawling (NEXT-2)
@@ -1330,33 +1329,7 @@ __global__ void __launch_bounds__(128) trawl_kernel(const DeviceGraph g, const P
         }
     }
     // block partial (fixed order); timeouts ride in the `sectors` slot
-    double sh = __dadd_rn(s_sum, c_sum), sl = __dsub_rn(c_sum, __dsub_rn(sh, s_sum));
-    double qh = __dadd_rn(s_sq, c_sq), ql = __dsub_rn(c_sq, __dsub_rn(qh, s_sq));
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        const double bh = shfl_xor_d(sh, o), bl = shfl_xor_d(sl, o);
-        const double ch = shfl_xor_d(qh, o), cl = shfl_xor_d(ql, o);
-        dd_add(sh, sl, bh, bl);
-        dd_add(qh, ql, ch, cl);
-        n_nonzero += __shfl_xor_sync(kFull, n_nonzero, o);
-        n_done += __shfl_xor_sync(kFull, n_done, o);
-        n_timeout += shfl_xor_d(n_timeout, o);
-    }
-    if (lane == 0) warp_part[tid >> 5] = Partial{sh, sl, qh, ql, n_nonzero, n_done, n_timeout, 0.0};
-    __syncthreads();
-    if (tid == 0) {
-        Partial acc = warp_part[0];
-        for (int w = 1; w < (int)(blockDim.x >> 5); ++w) {
-            const Partial& o = warp_part[w];
-            dd_add(acc.sum_hi, acc.sum_lo, o.sum_hi, o.sum_lo);
-            dd_add(acc.sq_hi, acc.sq_lo, o.sq_hi, o.sq_lo);
-            acc.valid += o.valid;
-            acc.n += o.n;
-            acc.sectors += o.sectors;
-            acc.model += o.model;
-        }
-        partials[blockIdx.x] = acc;
-    }
+    write_cta_partial(warp_part, partials, s_sum, c_sum, s_sq, c_sq, n_nonzero, n_done, n_timeout, 0.0);
 }
 
 // Grid reduction in CTA order (one warp; lane-strided then a fixed butterfly).

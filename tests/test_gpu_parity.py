@@ -611,7 +611,7 @@ def test_autotune_does_not_change_results(ctx, G, c0):
                 _agg_close(agg, ref_agg, G)
     ctx.load_graph_obj(g)
     ctx.load_query_obj(q)
-    assert all(r in (8, 16, 24, 32) for r in ctx.query_info()["refill_min"])
+    assert all(r in (8, 16, 24, 28, 32) for r in ctx.query_info()["refill_min"])
 
 
 def test_estimate_until(ctx, G, c0):
