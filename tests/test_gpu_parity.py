@@ -777,3 +777,35 @@ def test_two_contexts_run_concurrently(G, c0):
             assert r["sum"] == pytest.approx(ref["sum"], rel=REL, abs=0.0)
         c1.set_stream(None)
         c2.set_stream(None)
+
+
+def test_estimate_instance_per_sample(ctx, G, c0, c1):
+    """The timed estimate instance (the autotuned OCC / TREE / LOCK specialisation that
+    bench.py launches, not the trace build) checked sample by sample: a one-id range makes its
+    aggregate the sample's own weight, which must equal the oracle's bit for bit (a single
+    value passes the compensated sums and the double-double reduction unchanged); 64-id windows
+    (two warps' worth of lanes sharing the task pool and the refill queue) must match the
+    oracle's window sums at 1e-12 with n_valid exact.  C0 and the C1 bench queries, the
+    cyclic one included."""
+    for (g, qs), qidx in ((c0, range(len(c0[1]))), (c1, range(len(c1[1])))):
+        ctx.load_graph_obj(g)
+        for qi in qidx:
+            q = qs[qi]
+            ctx.load_query_obj(q)
+            for m in (0, 1):
+                y, ref = oracle.sample_range(g, q, m, 42, 0, 6400, records=True, threads=8)
+                y = np.asarray(y, dtype=np.float64)
+                valid = np.nonzero(ref["valid"])[0]
+                invalid = np.nonzero(ref["valid"] == 0)[0]
+                ids = list(valid[:40]) + list(invalid[:8]) + [6399]
+                for i in ids:
+                    r = ctx.estimate(m, 1, 42, first=int(i))
+                    assert r["n"] == 1 and r["n_valid"] == int(ref["valid"][i])
+                    w = float(y[i])
+                    assert r["sum"] == w, (g.name, q.name, m, int(i), r["sum"], w)
+                for first in range(0, 6400, 640):
+                    r = ctx.estimate(m, 64, 42, first=first)
+                    w = y[first:first + 64]
+                    assert r["n"] == 64 and r["n_valid"] == int((ref["valid"][first:first + 64] != 0).sum())
+                    assert r["sum"] == pytest.approx(float(np.sum(w)), rel=REL, abs=0.0)
+                    assert r["sumsq"] == pytest.approx(float(np.sum(w * w)), rel=REL, abs=0.0)
