@@ -206,6 +206,13 @@ typedef enum {
                                    /* 0, as a corrupted counter would (ids skipped);   */
                                    /* one-shot; 0 = off.  Synchronous calls then fail  */
                                    /* with GSWORD_EFAULT                               */
+    GSWORD_OPT_TRAWL_WARP = 16,    /* gsword_trawl_range enumeration: 1 (default) the  */
+                                   /* warp-cooperative kernel (32 candidates tested   */
+                                   /* per round, last-position survivors counted by   */
+                                   /* popcount), 0 one lane per sample depth first.   */
+                                   /* Same counts and timeouts (the node total of a   */
+                                   /* sample's tree decides the timeout); traces     */
+                                   /* always use the per-lane kernel                  */
     GSWORD_OPT_FILTER = 7          /* candidate filter applied by the next            */
                                    /* gsword_load_query: 0 label only, 1 LDF, 2 NLF   */
                                    /* (1-2 build the candidate graph, reading A21)    */

@@ -274,6 +274,7 @@ struct gsword_ctx {
     int tuned_occ[2] = {0, 0};    // occupancy variant of the estimate kernel (kModeOccShift)
     int opt_occ = -1;             // GSWORD_OPT_OCCUPANCY: -1 autotuned, else forced
     uint64_t opt_fault_queue = 0;  // GSWORD_OPT_FAULT_QUEUE: one-shot corrupted queue start
+    int opt_trawl_warp = 1;        // GSWORD_OPT_TRAWL_WARP: warp-cooperative trawling enumeration
     struct Tuned {
         int refill[2], occ[2];
     };
@@ -826,6 +827,9 @@ int gsword_set_option(gsword_ctx* ctx, int option, int64_t value) {
         case GSWORD_OPT_FAULT_QUEUE:
             if (value < 0) return fail(GSWORD_EINVAL, "fault queue start must be >= 0");
             ctx->opt_fault_queue = (uint64_t)value;
+            return GSWORD_OK;
+        case GSWORD_OPT_TRAWL_WARP:
+            ctx->opt_trawl_warp = value ? 1 : 0;
             return GSWORD_OK;
         case GSWORD_OPT_COOP_THRESHOLD:
             if (value < 0 || value > 128) return fail(GSWORD_EINVAL, "coop threshold must be 0..128");
@@ -1464,7 +1468,7 @@ int run_trawl(gsword_ctx* ctx, int m, uint64_t first, uint64_t n, uint64_t seed,
         ctx->partial_cap = grid;
     }
     CUDA_TRY(cudaEventRecord(ctx->evk0, ctx->stream));
-    CUDA_TRY(gsword::launch_trawl(m, d_rec != nullptr, ctx->q_filter != 0, device_graph(ctx), ctx->plan, grid, first,
+    CUDA_TRY(gsword::launch_trawl(m, d_rec != nullptr, ctx->opt_trawl_warp != 0, ctx->q_filter != 0, device_graph(ctx), ctx->plan, grid, first,
                                   n, seed, budget, ctx->d_queue, ctx->d_partials, d_rec, ctx->stream));
     CUDA_TRY(cudaEventRecord(ctx->evk1, ctx->stream));
     CUDA_TRY(gsword::launch_reduce(ctx->d_partials, grid, ctx->d_out4, ctx->d_sectors, ctx->stream));

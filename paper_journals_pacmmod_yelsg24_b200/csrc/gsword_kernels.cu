@@ -305,7 +305,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
         uq_s[tid] = plan_in.uq[tid];
         pdup_s[tid] = plan_in.pdup[tid];
     }
-    if (tid < kMaxQV * kMaxQV) eidx_s[tid / kMaxQV][tid % kMaxQV] = plan_in.eidx[tid / kMaxQV][tid % kMaxQV];
+    for (int i = tid; i < kMaxQV * kMaxQV; i += blockDim.x) eidx_s[i / kMaxQV][i % kMaxQV] = plan_in.eidx[i / kMaxQV][i % kMaxQV];
     __syncthreads();
 
     const int nq = plan_in.nq;
@@ -915,7 +915,7 @@ __global__ void __launch_bounds__(256) stream_kernel(const DeviceGraph g, const 
         plan_s[tid] = plan_in.step[tid];
         pdup_s[tid] = plan_in.pdup[tid];
     }
-    if (tid < kMaxQV * kMaxQV) eidx_s[tid / kMaxQV][tid % kMaxQV] = plan_in.eidx[tid / kMaxQV][tid % kMaxQV];
+    for (int i = tid; i < kMaxQV * kMaxQV; i += blockDim.x) eidx_s[i / kMaxQV][i % kMaxQV] = plan_in.eidx[i / kMaxQV][i % kMaxQV];
     __syncthreads();
     const int nq = plan_in.nq;
 
@@ -1187,6 +1187,80 @@ __device__ __forceinline__ bool extends(const DeviceGraph& g, const PlanStep& ps
     return true;
 }
 
+// The sampled prefix of a trawling sample: positions 0 .. dd-1 with the method's rules and the
+// same draws as the plain sampler; M[0..dd-1] and W = prod |C_d| out, false when it dies.
+template <int METHOD, bool TRACE, bool CG>
+__device__ __forceinline__ bool trawl_prefix(const DeviceGraph& g, const Plan& plan_in, const PlanStep* plan_s,
+                                             const uint8_t (*eidx_s)[kMaxQV], uint64_t seed, uint64_t sid, int dd,
+                                             int32_t* M, double* Wout, gsword_trawl_record* rec) {
+    double W = 0.0;
+    for (int d = 0; d < dd; ++d) {
+        const PlanStep ps = plan_s[d];
+        const uint64_t r = philox_r(seed, sid, (uint32_t)d);
+        uint32_t lo = 0, len = 0, cnt = 0;
+        int p = 0;
+        int32_t v = -1;
+        if (d == 0) {
+            lo = plan_in.seed_lo;
+            cnt = len = plan_in.seed_len;
+            if (cnt > 0) {
+                const uint64_t k = __umul64hi(r, (uint64_t)cnt);
+                v = plan_in.seed_identity ? (int32_t)(lo + k) : __ldg(g.bucket + lo + k);
+            }
+        } else {
+            getmin_local<CG>(g, ps, eidx_s, d, M, &lo, &len, &p);
+            if (METHOD == GSWORD_WJ) {
+                cnt = len;
+                if (cnt > 0) {
+                    v = __ldg(g.clist + lo + __umul64hi(r, (uint64_t)cnt));
+                }
+            } else {
+                for (uint32_t i = 0; i < len; ++i) cnt += extends(g, ps, p, M, d, __ldg(g.clist + lo + i)) ? 1u : 0u;
+                if (cnt > 0) {
+                    uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
+                    for (uint32_t i = 0; i < len; ++i) {
+                        const int32_t x = __ldg(g.clist + lo + i);
+                        if (!extends(g, ps, p, M, d, x)) continue;
+                        if (k == 0) {
+                            v = x;
+                            break;
+                        }
+                        --k;
+                    }
+                }
+            }
+        }
+        W = (d == 0) ? (double)cnt : __dmul_rn(W, (double)cnt);
+        if (TRACE) {
+            rec->csize[d] = cnt;
+            rec->path[d] = cnt > 0 ? v : -1;
+        }
+        *Wout = W;
+        if (cnt == 0) return false;
+        if (METHOD == GSWORD_WJ && d > 0 && !extends(g, ps, p, M, d, v)) return false;  // Validate
+        M[d] = v;
+    }
+    *Wout = W;
+    return true;
+}
+
+// T = W * count into the lane's compensated sums (status 1 = complete, 2 = timeout)
+__device__ __forceinline__ void trawl_accumulate(uint8_t status, double W, unsigned long long cnt_all, double& s_sum,
+                                                 double& c_sum, double& s_sq, double& c_sq, double& n_timeout,
+                                                 unsigned long long& n_nonzero, unsigned long long& n_done) {
+    if (status == 2) {
+        n_timeout += 1.0;
+    } else {
+        n_done += 1;
+        if (status == 1 && cnt_all > 0) {
+            const double T = __dmul_rn(W, (double)cnt_all);
+            n_nonzero += 1;
+            nsum(s_sum, c_sum, T);
+            nsum(s_sq, c_sq, __dmul_rn(T, T));
+        }
+    }
+}
+
 template <int METHOD, bool TRACE, bool CG>
 __global__ void __launch_bounds__(128) trawl_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
                                                     const uint64_t count, const uint64_t seed, const uint64_t budget,
@@ -1196,9 +1270,9 @@ __global__ void __launch_bounds__(128) trawl_kernel(const DeviceGraph g, const P
     __shared__ PlanStep plan_s[kMaxQV];
     __shared__ uint8_t eidx_s[kMaxQV][kMaxQV];
     __shared__ Partial warp_part[32];
-    const int tid = threadIdx.x, lane = tid & 31;
+    const int tid = threadIdx.x;
     if (tid < kMaxQV) plan_s[tid] = plan_in.step[tid];
-    if (tid < kMaxQV * kMaxQV) eidx_s[tid / kMaxQV][tid % kMaxQV] = plan_in.eidx[tid / kMaxQV][tid % kMaxQV];
+    for (int i = tid; i < kMaxQV * kMaxQV; i += blockDim.x) eidx_s[i / kMaxQV][i % kMaxQV] = plan_in.eidx[i / kMaxQV][i % kMaxQV];
     __syncthreads();
     const int nq = plan_in.nq;
     double s_sum = 0.0, c_sum = 0.0, s_sq = 0.0, c_sq = 0.0, n_timeout = 0.0;
@@ -1220,58 +1294,9 @@ __global__ void __launch_bounds__(128) trawl_kernel(const DeviceGraph g, const P
                 rec->csize[i] = 0;
             }
         }
-        // ---- sampled prefix: positions 0 .. dd-1 (same rules and draws as the sampler)
         double W = 0.0;
-        bool alive = true;
-        for (int d = 0; d < dd && alive; ++d) {
-            const PlanStep ps = plan_s[d];
-            const uint64_t r = philox_r(seed, sid, (uint32_t)d);
-            uint32_t lo = 0, len = 0, cnt = 0;
-            int p = 0;
-            int32_t v = -1;
-            if (d == 0) {
-                lo = plan_in.seed_lo;
-                cnt = len = plan_in.seed_len;
-                if (cnt > 0) {
-                    const uint64_t k = __umul64hi(r, (uint64_t)cnt);
-                    v = plan_in.seed_identity ? (int32_t)(lo + k) : __ldg(g.bucket + lo + k);
-                }
-            } else {
-                getmin_local<CG>(g, ps, eidx_s, d, M, &lo, &len, &p);
-                if (METHOD == GSWORD_WJ) {
-                    cnt = len;
-                    if (cnt > 0) {
-                        v = __ldg(g.clist + lo + __umul64hi(r, (uint64_t)cnt));
-                    }
-                } else {
-                    for (uint32_t i = 0; i < len; ++i) cnt += extends(g, ps, p, M, d, __ldg(g.clist + lo + i)) ? 1u : 0u;
-                    if (cnt > 0) {
-                        uint32_t k = (uint32_t)__umul64hi(r, (uint64_t)cnt);
-                        for (uint32_t i = 0; i < len; ++i) {
-                            const int32_t x = __ldg(g.clist + lo + i);
-                            if (!extends(g, ps, p, M, d, x)) continue;
-                            if (k == 0) {
-                                v = x;
-                                break;
-                            }
-                            --k;
-                        }
-                    }
-                }
-            }
-            W = (d == 0) ? (double)cnt : __dmul_rn(W, (double)cnt);
-            if (TRACE) {
-                rec->csize[d] = cnt;
-                rec->path[d] = cnt > 0 ? v : -1;
-            }
-            if (cnt == 0) {
-                alive = false;
-                break;
-            }
-            if (METHOD == GSWORD_WJ && d > 0 && !extends(g, ps, p, M, d, v)) alive = false;  // Validate
-            M[d] = v;
-        }
-        // ---- enumeration of positions dd .. nq-1
+        const bool alive = trawl_prefix<METHOD, TRACE, CG>(g, plan_in, plan_s, eidx_s, seed, sid, dd, M, &W, rec);
+        // ---- enumeration of positions dd .. nq-1 (depth first, ascending candidates)
         unsigned long long cnt_all = 0, nodes = 0;
         bool timeout = false;
         if (alive) {
@@ -1316,19 +1341,134 @@ __global__ void __launch_bounds__(128) trawl_kernel(const DeviceGraph g, const P
             rec->count = cnt_all;
             rec->nodes = nodes;
         }
-        if (status == 2) {
-            n_timeout += 1.0;
-        } else {
-            n_done += 1;
-            if (status == 1 && cnt_all > 0) {
-                const double T = __dmul_rn(W, (double)cnt_all);
-                n_nonzero += 1;
-                nsum(s_sum, c_sum, T);
-                nsum(s_sq, c_sq, __dmul_rn(T, T));
-            }
-        }
+        trawl_accumulate(status, W, cnt_all, s_sum, c_sum, s_sq, c_sq, n_timeout, n_nonzero, n_done);
     }
     // block partial (fixed order); timeouts ride in the `sectors` slot
+    write_cta_partial(warp_part, partials, s_sum, c_sum, s_sq, c_sq, n_nonzero, n_done, n_timeout, 0.0);
+}
+
+// Warp-cooperative trawling (estimates; gsword_trawl_range with GSWORD_OPT_TRAWL_WARP = 1).
+// A warp takes 32 sample ids, every lane samples its own prefix, then the warp enumerates the
+// completions of its lanes' samples one sample at a time: the candidate run of a level is
+// tested 32 elements per round (one lane each, ballot), survivors at the last position are
+// counted by popcount without descending, and the depth-first descent takes the survivors
+// of a round in ascending order.  The node total of a sample's enumeration tree does not
+// depend on the visiting order, so "more than `budget` nodes" (the timeout, reading A23) is
+// decided exactly as the per-lane depth-first kernel decides it; a sample that does not
+// time out gets the same count.  (Traces keep the per-lane kernel: a timed-out record's
+// partial count depends on the visiting order.)
+template <int METHOD, bool CG>
+__global__ void __launch_bounds__(128) trawl_warp_kernel(const DeviceGraph g, const Plan plan_in, const uint64_t first,
+                                                         const uint64_t count, const uint64_t seed,
+                                                         const uint64_t budget, unsigned long long* __restrict__ queue,
+                                                         Partial* __restrict__ partials) {
+    constexpr int kW = 4;  // warps per CTA
+    __shared__ PlanStep plan_s[kMaxQV];
+    __shared__ uint8_t eidx_s[kMaxQV][kMaxQV];
+    __shared__ Partial warp_part[32];
+    __shared__ int32_t Mw[kW][kMaxQV];  // the enumerated sample's matched vertices
+    __shared__ uint32_t st_lo[kW][kMaxQV], st_len[kW][kMaxQV], st_pos[kW][kMaxQV], st_mask[kW][kMaxQV],
+        st_base[kW][kMaxQV];
+    __shared__ int st_p[kW][kMaxQV];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    if (tid < kMaxQV) plan_s[tid] = plan_in.step[tid];
+    for (int i = tid; i < kMaxQV * kMaxQV; i += blockDim.x) eidx_s[i / kMaxQV][i % kMaxQV] = plan_in.eidx[i / kMaxQV][i % kMaxQV];
+    __syncthreads();
+    const int nq = plan_in.nq;
+    double s_sum = 0.0, c_sum = 0.0, s_sq = 0.0, c_sq = 0.0, n_timeout = 0.0;
+    unsigned long long n_nonzero = 0, n_done = 0;
+    int32_t M[kMaxQV];
+    int32_t* const Ms = Mw[w];
+    while (true) {
+        unsigned long long base_id = 0;
+        if (lane == 0) base_id = atomicAdd(queue, 32ull);
+        base_id = __shfl_sync(kFull, base_id, 0);
+        if (base_id >= count) break;
+        const unsigned long long idx = base_id + (unsigned long long)lane;
+        const bool has = idx < count;
+        const uint64_t sid = first + idx;
+        int dd = nq;
+        double W = 0.0;
+        bool alive = false;
+        if (has) {
+            dd = choose_d(seed, sid, nq);
+            alive = trawl_prefix<METHOD, false, CG>(g, plan_in, plan_s, eidx_s, seed, sid, dd, M, &W, nullptr);
+        }
+        unsigned long long cnt_all = (alive && dd == nq) ? 1ull : 0ull;
+        bool timeout = false;
+        uint32_t todo = __ballot_sync(kFull, alive && dd < nq);
+        while (todo) {
+            const int L = __ffs(todo) - 1;
+            todo &= todo - 1;
+            const int d0 = __shfl_sync(kFull, dd, L);
+            if (lane == L)
+                for (int j = 0; j < d0; ++j) Ms[j] = M[j];
+            __syncwarp();
+            unsigned long long nodes = 0, cnt = 0;
+            bool to = false;
+            int t = d0, p = 0;
+            uint32_t lo = 0, len = 0, pos = 0, mask = 0, base = 0;
+            getmin_local<CG>(g, plan_s[t], eidx_s, t, Ms, &lo, &len, &p);
+            while (true) {
+                if (mask == 0u) {
+                    if (pos >= len) {  // level exhausted: back to the parent's pending survivors
+                        if (t == d0) break;
+                        --t;
+                        lo = st_lo[w][t];
+                        len = st_len[w][t];
+                        pos = st_pos[w][t];
+                        mask = st_mask[w][t];
+                        base = st_base[w][t];
+                        p = st_p[w][t];
+                        __syncwarp();  // every lane has read the level before lane 0 rewrites it
+                        continue;
+                    }
+                    const uint32_t i = pos + (uint32_t)lane;
+                    const bool ok = i < len && extends(g, plan_s[t], p, Ms, t, __ldg(g.clist + lo + i));
+                    mask = __ballot_sync(kFull, ok);
+                    base = pos;
+                    pos += 32u;
+                    nodes += (unsigned long long)__popc(mask);
+                    if (nodes > budget) {
+                        to = true;
+                        break;
+                    }
+                    if (t + 1 == nq) {
+                        cnt += (unsigned long long)__popc(mask);
+                        mask = 0u;
+                    }
+                    continue;
+                }
+                const int b = __ffs(mask) - 1;
+                mask &= mask - 1u;
+                const int32_t x = __ldg(g.clist + lo + base + (uint32_t)b);
+                if (lane == 0) {
+                    st_lo[w][t] = lo;
+                    st_len[w][t] = len;
+                    st_pos[w][t] = pos;
+                    st_mask[w][t] = mask;
+                    st_base[w][t] = base;
+                    st_p[w][t] = p;
+                    Ms[t] = x;
+                }
+                __syncwarp();
+                ++t;
+                getmin_local<CG>(g, plan_s[t], eidx_s, t, Ms, &lo, &len, &p);
+                pos = 0u;
+                mask = 0u;
+                base = 0u;
+            }
+            if (lane == L) {
+                cnt_all = cnt;
+                timeout = to;
+            }
+            __syncwarp();
+        }
+        if (has) {
+            const uint8_t status = !alive ? 0 : (timeout ? 2 : 1);
+            trawl_accumulate(status, W, cnt_all, s_sum, c_sum, s_sq, c_sq, n_timeout, n_nonzero, n_done);
+        }
+    }
     write_cta_partial(warp_part, partials, s_sum, c_sum, s_sq, c_sq, n_nonzero, n_done, n_timeout, 0.0);
 }
 
@@ -1720,20 +1860,26 @@ cudaError_t launch_scan(uint32_t* data, int64_t n, const unsigned long long* d_b
     return cudaGetLastError();
 }
 
-cudaError_t launch_trawl(int method, bool trace, bool cg, const DeviceGraph& g, const Plan& plan, int grid,
+cudaError_t launch_trawl(int method, bool trace, bool warp, bool cg, const DeviceGraph& g, const Plan& plan, int grid,
                          uint64_t first, uint64_t count, uint64_t seed, uint64_t budget, unsigned long long* d_queue,
                          Partial* d_partials, gsword_trawl_record* d_records, cudaStream_t stream) {
     cudaError_t e = cudaMemsetAsync(d_queue, 0, sizeof(unsigned long long), stream);
     if (e != cudaSuccess) return e;
 #define GSWORD_TRAWL(M, TR, CGF) \
     trawl_kernel<M, TR, CGF><<<grid, 128, 0, stream>>>(g, plan, first, count, seed, budget, d_queue, d_partials, d_records)
-    if (method == GSWORD_WJ) {
+#define GSWORD_TRAWL_WARP(M, CGF) \
+    trawl_warp_kernel<M, CGF><<<grid, 128, 0, stream>>>(g, plan, first, count, seed, budget, d_queue, d_partials)
+    if (warp && !trace) {
+        if (method == GSWORD_WJ) { if (cg) GSWORD_TRAWL_WARP(GSWORD_WJ, true); else GSWORD_TRAWL_WARP(GSWORD_WJ, false); }
+        else { if (cg) GSWORD_TRAWL_WARP(GSWORD_ALLEY, true); else GSWORD_TRAWL_WARP(GSWORD_ALLEY, false); }
+    } else if (method == GSWORD_WJ) {
         if (trace) { if (cg) GSWORD_TRAWL(GSWORD_WJ, true, true); else GSWORD_TRAWL(GSWORD_WJ, true, false); }
         else { if (cg) GSWORD_TRAWL(GSWORD_WJ, false, true); else GSWORD_TRAWL(GSWORD_WJ, false, false); }
     } else {
         if (trace) { if (cg) GSWORD_TRAWL(GSWORD_ALLEY, true, true); else GSWORD_TRAWL(GSWORD_ALLEY, true, false); }
         else { if (cg) GSWORD_TRAWL(GSWORD_ALLEY, false, true); else GSWORD_TRAWL(GSWORD_ALLEY, false, false); }
     }
+#undef GSWORD_TRAWL_WARP
 #undef GSWORD_TRAWL
     return cudaGetLastError();
 }

@@ -172,7 +172,7 @@ cudaError_t launch_pair_hist(const int64_t* row_ptr, const int32_t* col, const i
 cudaError_t launch_label_bucket(const int32_t* labels, int64_t n, int32_t l, uint32_t* counts,
                                 const unsigned long long* d_base, uint32_t* d_tmp, unsigned long long* d_total,
                                 int32_t* bucket, cudaStream_t stream);
-cudaError_t launch_trawl(int method, bool trace, bool cg, const DeviceGraph& g, const Plan& plan, int grid,
+cudaError_t launch_trawl(int method, bool trace, bool warp, bool cg, const DeviceGraph& g, const Plan& plan, int grid,
                          uint64_t first, uint64_t count, uint64_t seed, uint64_t budget, unsigned long long* d_queue,
                          Partial* d_partials, gsword_trawl_record* d_records, cudaStream_t stream);
 // candidate graph build (NEXT-1)

@@ -37,6 +37,7 @@ OPT_STREAMING = 12  # Alley by warp streaming (Alg. 3, reading A25)
 OPT_VARIANT = 13  # comparison variants of readings A3/A5 (bit flags below)
 OPT_OCCUPANCY = 14  # estimate-kernel occupancy variant: -1 autotuned, 0/1/2 forced
 OPT_FAULT_QUEUE = 15  # fault injection: the next launch's queue starts here (one-shot)
+OPT_TRAWL_WARP = 16  # trawl_range: 1 warp-cooperative enumeration (default), 0 one lane per sample
 VARIANT_WJ_PARENT_FIRST = 2
 VARIANT_ALLEY_DUPCHECK_POST = 4
 SCHED_REFILL, SCHED_SAMPLE_SYNC, SCHED_INHERIT = 0, 1, 2

@@ -28,12 +28,16 @@ with G.Context(0) as ctx:
         for q in qs:
             ctx.load_query_obj(q)
             for m in (G.WJ, G.ALLEY):
-                for mode in ("plain", "trawl"):
+                for mode in ("plain", "trawl", "trawl_lane"):
                     if mode == "plain":
                         r = ctx.estimate(m, int(args.samples), 42)
                         r["n_timeout"] = 0
                     else:
+                        # trawl: warp-cooperative enumeration (default); trawl_lane: one lane
+                        # per sample, depth first (round 1's kernel)
+                        ctx.set_option(G.OPT_TRAWL_WARP, 1 if mode == "trawl" else 0)
                         r = ctx.trawl(m, int(args.trawl_samples), 42, node_budget=args.budget)
+                        ctx.set_option(G.OPT_TRAWL_WARP, 1)
                     se = math.sqrt(r["variance"]) if r["variance"] > 0 else 0.0
                     print(json.dumps({"config": args.config, "query": q.name, "filter": filt,
                                       "method": "wj" if m == G.WJ else "alley", "mode": mode, "n": r["n"],

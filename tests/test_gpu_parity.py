@@ -399,6 +399,26 @@ def test_filtered_parity_small_and_c0(ctx, G, c0, filt):
         ctx.set_option(G.OPT_FILTER, 0)
 
 
+@pytest.mark.parametrize("threads", [64, 96, 256])
+def test_filtered_large_query_any_cta_size(ctx, G, threads):
+    """Candidate-graph runs of positions >= 8 under every CTA size: the per-query-edge index
+    table staged in shared memory must be complete however many threads stage it (a
+    12-vertex query with NLF at 64 / 96 / 256 threads per CTA, sampling and trawling)."""
+    g = gen.chung_lu(3000, 60_000, gamma=2.2, max_over_mean=40.0, seed=21, labels=gen.uniform_labels(3000, 2, 22),
+                     n_labels=2)
+    q = gen.extract_query(g, 12, seed=23, dense=True)
+    ctx.load_graph_obj(g)
+    ctx.set_option(G.OPT_FILTER, 2)
+    ctx.set_option(G.OPT_THREADS, threads)
+    try:
+        for m in (0, 1):
+            _parity_filtered(ctx, G, g, q, m, 5, 0, 20_000, 2)
+            _trawl_parity(ctx, G, g, q, m, 6, 0, 3000, 20_000, filt=2)
+    finally:
+        ctx.set_option(G.OPT_FILTER, 0)
+        ctx.set_option(G.OPT_THREADS, 256)
+
+
 @pytest.mark.parametrize("filt", [1, 2])
 def test_filtered_parity_c2_c1(ctx, G, c1, filt):
     ctx.set_option(G.OPT_FILTER, filt)
@@ -468,11 +488,23 @@ def _trawl_parity(ctx, G, g, q, method, seed, first, count, budget, filt=0, thre
     rec = ctx.trace_trawl(method, first, count, seed, budget)
     t, st, ref = oracle.trawl_range(g, q, method, seed, first, count, budget=budget, filter=filt, threads=threads)
     assert rec.tobytes() == ref.tobytes(), f"trawl records differ ({q.name}, m{method}, budget {budget})"
-    r = ctx.trawl(method, count, seed, first=first, node_budget=budget)
     agg = oracle.trawl_aggregate(t, st)
-    assert r["n_timeout"] == agg["n_timeout"] and r["n"] == agg["n"] and r["n_valid"] == agg["n_valid"]
-    assert r["sum"] == pytest.approx(agg["sum"], rel=REL)
-    assert r["sumsq"] == pytest.approx(agg["sumsq"], rel=REL)
+    # both enumeration kernels of gsword_trawl_range: warp-cooperative (default) and per-lane
+    for warp in (1, 0):
+        ctx.set_option(G.OPT_TRAWL_WARP, warp)
+        try:
+            r = ctx.trawl(method, count, seed, first=first, node_budget=budget)
+        finally:
+            ctx.set_option(G.OPT_TRAWL_WARP, 1)
+        assert r["n_timeout"] == agg["n_timeout"] and r["n"] == agg["n"] and r["n_valid"] == agg["n_valid"], warp
+        assert r["sum"] == pytest.approx(agg["sum"], rel=REL)
+        assert r["sumsq"] == pytest.approx(agg["sumsq"], rel=REL)
+    # the warp-cooperative kernel sample by sample: a one-id range gives T (bit-exact) or
+    # the timeout of that sample
+    for i in list(np.nonzero(st == 1)[0][:12]) + list(np.nonzero(st == 2)[0][:4]) + list(np.nonzero(st == 0)[0][:2]):
+        r = ctx.trawl(method, 1, seed, first=first + int(i), node_budget=budget)
+        assert r["n_timeout"] == int(st[i] == 2)
+        assert r["sum"] == (float(t[i]) if st[i] == 1 else 0.0), (q.name, method, int(i), r["sum"], float(t[i]))
 
 
 @pytest.mark.parametrize("method", [0, 1])
