@@ -38,3 +38,15 @@ with G.Context(0) as ctx:
         r = ctx.estimate(m, 20_000, 1)
         rec = ctx.trace_samples(m, 0, 2000, 1)
         print("nlf", q.name, m, r["n_valid"], int(rec["valid"].sum()), ctx.query_info()["cg_bytes"])
+    # trawling: the warp-cooperative enumeration (shared-memory stack; estimates) and the
+    # per-lane kernel (traces), label-only and under the candidate graph
+    for filt in (0, 2):
+        ctx.set_option(G.OPT_FILTER, filt)
+        ctx.load_query_obj(q)
+        for m in (G.WJ, G.ALLEY):
+            for warp in (1, 0):
+                ctx.set_option(G.OPT_TRAWL_WARP, warp)
+                r = ctx.trawl(m, 3000, 1, node_budget=5000)
+            ctx.set_option(G.OPT_TRAWL_WARP, 1)
+            tr = ctx.trace_trawl(m, 0, 500, 1, 5000)
+            print("trawl", filt, m, r["n_valid"], r["n_timeout"], int((tr["status"] == 1).sum()))

@@ -408,12 +408,13 @@ def test_filtered_large_query_any_cta_size(ctx, G, threads):
                      n_labels=2)
     q = gen.extract_query(g, 12, seed=23, dense=True)
     ctx.load_graph_obj(g)
-    ctx.set_option(G.OPT_FILTER, 2)
     ctx.set_option(G.OPT_THREADS, threads)
     try:
-        for m in (0, 1):
-            _parity_filtered(ctx, G, g, q, m, 5, 0, 20_000, 2)
-            _trawl_parity(ctx, G, g, q, m, 6, 0, 3000, 20_000, filt=2)
+        for filt in (0, 2):
+            ctx.set_option(G.OPT_FILTER, filt)
+            for m in (0, 1):
+                _parity_filtered(ctx, G, g, q, m, 5, 0, 20_000, filt)
+                _trawl_parity(ctx, G, g, q, m, 6, 0, 3000, 20_000, filt=filt)
     finally:
         ctx.set_option(G.OPT_FILTER, 0)
         ctx.set_option(G.OPT_THREADS, 256)
