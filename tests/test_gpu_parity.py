@@ -420,6 +420,27 @@ def test_filtered_large_query_any_cta_size(ctx, G, threads):
         ctx.set_option(G.OPT_THREADS, 256)
 
 
+def test_many_labels(ctx, G):
+    """A label alphabet far larger than the configs' (1,000 labels, half the vertices on label
+    0, the rest spread over 999): the label-segment table has |V| x 1,000 + 1 entries; records
+    and aggregates against the oracle, label-only and NLF, both methods, and trawling."""
+    n = 4000
+    rng = np.random.default_rng(77)
+    lab = np.where(rng.random(n) < 0.5, 0, rng.integers(1, 1000, size=n)).astype(np.int32)
+    g = gen.chung_lu(n, 80_000, gamma=2.2, max_over_mean=40.0, seed=78, labels=lab, n_labels=1000)
+    ctx.load_graph_obj(g)
+    for qs, dense in ((79, True), (80, False)):
+        q = gen.extract_query(g, 7, seed=qs, dense=dense)
+        for filt in (0, 2):
+            ctx.set_option(G.OPT_FILTER, filt)
+            try:
+                for m in (0, 1):
+                    _parity_filtered(ctx, G, g, q, m, 9, 0, 20_000, filt)
+                    _trawl_parity(ctx, G, g, q, m, 10, 0, 2000, 50_000, filt=filt)
+            finally:
+                ctx.set_option(G.OPT_FILTER, 0)
+
+
 @pytest.mark.parametrize("filt", [1, 2])
 def test_filtered_parity_c2_c1(ctx, G, c1, filt):
     ctx.set_option(G.OPT_FILTER, filt)
