@@ -13,6 +13,7 @@ out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-so
                      capture_output=True, text=True).stdout
 kernel = None
 blocks = {}
+hdrs = {}  # the source page's column set can differ per kernel
 hdr = None
 for row in csv.reader(io.StringIO(out)):
     if not row:
@@ -23,12 +24,15 @@ for row in csv.reader(io.StringIO(out)):
         continue
     if row[0] == "Line No":
         hdr = row
+        if kernel is not None:
+            hdrs[kernel] = row
         continue
     if hdr and kernel and row[0].isdigit() and len(row) == len(hdr) and row[2] == "-":
         blocks[kernel].append(row)
 for k, rows in blocks.items():
     if want not in k:
         continue
+    hdr = hdrs[k]
     i_st = hdr.index("Warp Stall Sampling (All Samples)")
     i_ie = hdr.index("Instructions Executed")
     i_te = hdr.index("Thread Instructions Executed")
