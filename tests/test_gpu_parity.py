@@ -243,6 +243,17 @@ def test_c2_parity(ctx, G):
     for i, q in enumerate(qs):
         for m in (0, 1):
             _parity(ctx, G, g, q, m, seed=10 + i, first=0, count=50_000, loaded=True)
+            # BASELINE configs[2] budget (1e8 samples): windows deep in the id range, and the
+            # whole 1e8 aggregate equal to the sum of two split ranges
+            for first in (50_000_000, 100_000_000 - 4000):
+                rec = ctx.trace_samples(m, first, 4000, 10 + i)
+                _, ref = oracle.sample_range(g, q, m, 10 + i, first, 4000, records=True, threads=8)
+                _records_equal(rec, ref, f"C2/{q.name}/m{m}@{first}")
+            full = ctx.estimate(m, 100_000_000, 10 + i)
+            a = ctx.estimate(m, 61_000_000, 10 + i)
+            b = ctx.estimate(m, 39_000_000, 10 + i, first=61_000_000)
+            assert full["n_valid"] == a["n_valid"] + b["n_valid"]
+            assert full["sum"] == pytest.approx(a["sum"] + b["sum"], rel=REL)
 
 
 @pytest.fixture(scope="module")
