@@ -581,6 +581,8 @@ def run_ours(args):
         "dram_frac": traffic / dom_s / 1e9 / peak if traffic else None,
         "gather_sectors_per_s": gather, "alg_sectors_per_s": sec_rate,
         "gather_frac": sec_rate / gather["l2_resident_64MB"], "gather_frac_hbm": sec_rate / gather["hbm_2GB"],
+        # against uniform random gathers over a buffer the size of `col` (the graph's adjacency)
+        "gather_frac_col": sec_rate / gather["col_size"],
         "ncu_counters": ncu_counters,
         "model": "reading A26 (DESIGN.md §3): offsets + drawn/selected vertices + Alley driver scans at "
                  "|B(d)|>=2 + one sector per membership question; counted by the kernel's counting build "
