@@ -279,7 +279,7 @@ def run_reference(args):
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
-    print(json.dumps(line), flush=True)
+    emit(line)
     return 0
 
 
@@ -633,7 +633,7 @@ def run_ours(args):
         "gpu_launches": 2 * len(methods) * args.steps,
         "clocks": clocks.summary(),
     }
-    print(json.dumps(line), flush=True)
+    emit(line)
     ctx.close()
     if combine:
         dist.barrier()
@@ -641,8 +641,36 @@ def run_ours(args):
     return 0
 
 
+_JSON_FD = None  # the process's original stdout, kept for the one JSON line
+
+
+def reserve_stdout():
+    """stdout carries exactly one JSON line (the driver's contract).  Native libraries write
+    banners to file descriptor 1 directly — NCCL prints "NCCL version ..." at communicator
+    init when NCCL_DEBUG=VERSION, which the GPU boxes set — so fd 1 is pointed at stderr for
+    the whole run and the JSON line is written to a duplicate of the original stdout."""
+    global _JSON_FD
+    try:
+        sys.stdout.flush()
+        fd = os.dup(1)
+        os.dup2(2, 1)
+        _JSON_FD = fd
+    except OSError:
+        _JSON_FD = None
+
+
+def emit(line) -> None:
+    text = json.dumps(line) + "\n"
+    if _JSON_FD is None:
+        sys.stdout.write(text)
+        sys.stdout.flush()
+    else:
+        os.write(_JSON_FD, text.encode())
+
+
 def main():
     args = parse()
+    reserve_stdout()
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

@@ -140,8 +140,10 @@ def _bench_line(args, nproc, torchrun=False):
                "--master-addr", "127.0.0.1", "--master-port", str(_free_port())] + common + ["--gpus", str(nproc)]
     out = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=900)
     assert out.returncode == 0, out.stderr[-3000:]
-    lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
-    assert len(lines) == 1, out.stdout[-2000:]
+    # stdout is the one JSON line and nothing else (native banners such as NCCL's version line
+    # under NCCL_DEBUG=VERSION go to stderr)
+    lines = [ln for ln in out.stdout.splitlines() if ln.strip()]
+    assert len(lines) == 1 and lines[0].startswith("{"), out.stdout[-2000:]
     return json.loads(lines[0])
 
 
