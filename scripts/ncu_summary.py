@@ -38,7 +38,9 @@ raw = page("raw")
 h, units = raw[0], raw[1]
 want = ['gpu__time_duration.sum', 'dram__bytes_read.sum', 'dram__bytes_write.sum', 'lts__t_sectors.sum',
         'lts__t_sector_hit_rate.pct', 'smsp__thread_inst_executed_per_inst_executed.ratio',
-        'l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum']
+        'l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum', 'l1tex__throughput.avg.pct_of_peak_sustained_active',
+        'lts__throughput.avg.pct_of_peak_sustained_elapsed',
+        'l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed']
 scale = {'Gbyte': 1e9, 'Mbyte': 1e6, 'Kbyte': 1e3, 'byte': 1.0, 'Tbyte': 1e12}
 traffic = {}
 for r in raw[2:]:
@@ -73,6 +75,10 @@ for k in ('wj', 'alley'):
         "l1_global_load_sectors_per_sample": (num(k, 'l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum') or 0) / samples,
         "l2_sectors_per_sample": (num(k, 'lts__t_sectors.sum') or 0) / samples,
         "dram_sectors_per_sample": traffic.get(k, 0.0) / 32.0,
+        # no unit saturated: L1TEX and L2 throughput against their peaks
+        "l1tex_throughput_pct": num(k, 'l1tex__throughput.avg.pct_of_peak_sustained_active'),
+        "lts_throughput_pct": num(k, 'lts__throughput.avg.pct_of_peak_sustained_elapsed'),
+        "shared_wavefronts_pct": num(k, 'l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed'),
     }
 json.dump({"workload": WORKLOAD, "captured_samples_per_launch": samples, "dram_bytes_per_sample": traffic,
            "counters": counters,

@@ -18,7 +18,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--samples", type=float, default=1e7)
 ap.add_argument("--config", default="C1")
 ap.add_argument("--query", type=int, default=1)
-ap.add_argument("--l2", type=int, default=0)
+ap.add_argument("--l2", type=int, default=-1, help="GSWORD_OPT_L2_PERSIST; -1 = the product default (the bench's)")
 ap.add_argument("--coop", type=int, default=-1)
 ap.add_argument("--threads", type=int, default=0)
 ap.add_argument("--chunk", type=int, default=0)
@@ -29,7 +29,8 @@ args = ap.parse_args()
 g, qs = gen.CONFIGS[args.config]()
 q = qs[args.query]
 with G.Context(0) as ctx:
-    ctx.set_option(G.OPT_L2_PERSIST, args.l2)
+    if args.l2 >= 0:
+        ctx.set_option(G.OPT_L2_PERSIST, args.l2)
     if args.coop >= 0:
         ctx.set_option(G.OPT_COOP_THRESHOLD, args.coop)
     if args.threads:
