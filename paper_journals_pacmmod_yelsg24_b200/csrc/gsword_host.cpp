@@ -1252,9 +1252,9 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
     if (ctx->opt_autotune && ctx->opt_sched == 0 && ctx->tuned_refill[0] == 0) {
         // schedule autotune (no effect on any result).  Phase 1: refill thresholds
         // 16/8/24/32/28 (samples of long-lived walks favour depth-synchronous warps, short-lived
-        // ones frequent refills).  Phase 2, at the chosen threshold: the
-        // estimate kernel compiled for one CTA/SM less (more registers, fewer spills) and one
-        // more.  Every candidate is timed over the same id range of `big` samples, preceded
+        // ones frequent refills).  Phase 2 (below): the estimate kernel compiled
+        // for one CTA/SM less (more registers, fewer spills) and one more, against the default.
+        // Every phase-1 candidate is timed over the same id range of `big` samples, preceded
         // by a warm-up over a range of its own (short or repeated pilots favour whichever
         // candidate profits from the tail or from a warm L2); each phase queues its runs back
         // to back on the context stream, timed by events, with one host synchronisation.
@@ -1287,7 +1287,7 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
                 for (int c = 0; c < ncand && e == cudaSuccess; ++c)
                     e = cudaEventElapsedTime(&times[m][c], ev[m][c][0], ev[m][c][1]);
         };
-        float t1[2][5] = {}, t2[2][5] = {};
+        float t1[2][5] = {};
         time_phase(5, [&](int m, int c) { ctx->tuned_refill[m] = cand[c]; }, t1);
         float best[2] = {0.f, 0.f};
         for (int m = 0; m < 2; ++m) {
@@ -1297,14 +1297,47 @@ int gsword_load_query(gsword_ctx* ctx, int32_t n_qv, const int32_t* q_row_ptr, c
             ctx->tuned_refill[m] = cand[bc];
             best[m] = t1[m][bc];
         }
-        if (ctx->opt_occ < 0) time_phase(2, [&](int m, int c) { ctx->tuned_occ[m] = 1 + c; }, t2);
-        for (int m = 0; m < 2; ++m) {
-            ctx->tuned_occ[m] = 0;
-            for (int c = 0; c < 2 && ctx->opt_occ < 0; ++c)
-                if (t2[m][c] < 0.99f * best[m]) {  // a variant must win by 1 % (pilot noise)
-                    best[m] = t2[m][c];
-                    ctx->tuned_occ[m] = 1 + c;
+        // Phase 2, at the chosen threshold: occupancy variants 0, 1, 2 compared by their
+        // steady-state cost t(2N) - t(N), so the per-launch tail (a third of an 8e6-sample
+        // pilot on C1 dense Alley) cancels; N is sized from phase 1 to ~4 ms per method, and the
+        // two runs cover disjoint id ranges (neither finds the other's samples in L2).
+        for (int m = 0; m < 2; ++m) ctx->tuned_occ[m] = 0;
+        if (ctx->opt_occ < 0) {
+            uint64_t n2[2];
+            for (int m = 0; m < 2; ++m) {
+                const double rate = best[m] > 0.f ? (double)big / (double)best[m] : 1e6;  // samples per ms
+                // at least 4e6 samples: slow, heavy-tailed queries (C1 cyclic Alley, 8 ms of
+                // per-launch tail) need the longer runs for a stable difference
+                n2[m] = (uint64_t)std::min(1e8, std::max(4e6, 4.0 * rate));
+            }
+            cudaEvent_t ev[2][3][3];
+            for (int m = 0; m < 2 && rc2 == GSWORD_OK && e == cudaSuccess; ++m)
+                for (int c = 0; c < 3 && rc2 == GSWORD_OK && e == cudaSuccess; ++c) {
+                    ctx->tuned_occ[m] = c;
+                    rc2 = run(ctx, m, gsword::kModeEstimate, range0 + (3 * n2[m] + warm) * (uint64_t)(8 + 3 * m + c), warm,
+                              0x5EEDull, ctx->d_out4, nullptr, nullptr);
+                    for (int k = 0; k < 3; ++k) event(&ev[m][c][k]);
+                    for (int k = 0; k < 2 && rc2 == GSWORD_OK && e == cudaSuccess; ++k) {
+                        e = cudaEventRecord(ev[m][c][k], ctx->stream);
+                        if (e == cudaSuccess)
+                            rc2 = run(ctx, m, gsword::kModeEstimate, range0 + k * n2[m], n2[m] << k, 0x5EEDull,
+                                      ctx->d_out4, nullptr, nullptr);
+                    }
+                    if (rc2 == GSWORD_OK && e == cudaSuccess) e = cudaEventRecord(ev[m][c][2], ctx->stream);
                 }
+            if (rc2 == GSWORD_OK && e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+            for (int m = 0; m < 2 && rc2 == GSWORD_OK && e == cudaSuccess; ++m) {
+                float steady[3];
+                for (int c = 0; c < 3 && e == cudaSuccess; ++c) {
+                    float a = 0.f, b = 0.f;
+                    e = cudaEventElapsedTime(&a, ev[m][c][0], ev[m][c][1]);
+                    if (e == cudaSuccess) e = cudaEventElapsedTime(&b, ev[m][c][1], ev[m][c][2]);
+                    steady[c] = b - a;
+                }
+                ctx->tuned_occ[m] = 0;
+                for (int c = 1; c < 3 && e == cudaSuccess; ++c)
+                    if (steady[c] < 0.99f * steady[ctx->tuned_occ[m]]) ctx->tuned_occ[m] = c;  // 1 % margin
+            }
         }
         for (cudaEvent_t x : evs) cudaEventDestroy(x);
         if (rc2 != GSWORD_OK || e != cudaSuccess) {

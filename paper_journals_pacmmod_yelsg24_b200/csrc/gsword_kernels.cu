@@ -53,7 +53,7 @@ using namespace dev;
 template <bool COUNT>
 __device__ __forceinline__ void coop_refine(const DeviceGraph& g, const uint32_t* Ms, int T, int lane, int colL,
                                             uint32_t Llo, uint32_t Llen, uint32_t others, const PlanStep& Lps,
-                                            uint32_t Lsig, uint32_t Lr_lo, uint32_t Lr_hi, double& sectors,
+                                            uint32_t Lsig, uint64_t r_lane, int L, double& sectors,
                                             uint32_t& total_out, int32_t& chosen_out) {
     uint32_t total = 0, my_bal = 0;
     // lists longer than 32 chunks: lane g also counts the survivors of chunk group
@@ -79,6 +79,9 @@ __device__ __forceinline__ void coop_refine(const DeviceGraph& g, const uint32_t
     }
     int32_t chosen = -1;
     if (total > 0) {
+        // lane L's random word, fetched only now (not live across the count loop)
+        const uint32_t Lr_lo = __shfl_sync(kFull, (uint32_t)r_lane, L);
+        const uint32_t Lr_hi = __shfl_sync(kFull, (uint32_t)(r_lane >> 32), L);
         const uint64_t Lr = ((uint64_t)Lr_hi << 32) | Lr_lo;
         const uint32_t k = (uint32_t)__umul64hi(Lr, (uint64_t)total);
         if (Llen <= 32u * 32u) {
@@ -287,7 +290,7 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     __shared__ uint8_t uq_s[kMaxQV];
     __shared__ uint32_t pdup_s[kMaxQV];  // variant A5: post-draw DupCheck positions
     __shared__ Partial warp_part[8];
-    // dynamic shared memory, rows of blockDim.x words (sized on the host by the query and
+    // dynamic shared memory, rows of kSampleLanes words (sized on the host by the query and
     // the coop threshold, so the rest of the SM's L1/shared array stays L1):
     //   Ms[j * T + tid]          = M[j] of this lane, j < n_q
     //   pool_s[w * T + tid]      (Alley) w = 0: task-pool results "matched vertex j lies in
@@ -295,7 +298,9 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     extern __shared__ uint32_t Ms[];
 
     const int tid = threadIdx.x;
-    const int T = blockDim.x;
+    // row stride of Ms: a compile-time constant (no register) where multi-list steps raise the
+    // register pressure; tree orders keep blockDim.x (measured 2 % faster there)
+    const int T = TREE ? (int)blockDim.x : kSampleLanes;
     const int lane = tid & 31;
     const int wbase = tid - lane;
     const unsigned lt_mask = (1u << lane) - 1u;
@@ -312,9 +317,8 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
     uint32_t* const pool_s = Ms + (size_t)nq * (size_t)T;
     const uint32_t mask_words = (coop_threshold + 31u) >> 5;  // refine-mask rows (<= 4)
     const int sched = SYNC ? sched_arg : 0;
-    bool multi_back = false;  // some position has |B(d)| >= 2 (Alley refine kinds 2/3 can occur)
-    if (!TREE)
-        for (int dd = 1; dd < nq; ++dd) multi_back |= plan_s[dd].nback >= 2;
+    // some position has |B(d)| >= 2 (Alley refine kinds 2/3 can occur): a launch constant
+    const bool multi_back = !TREE && plan_in.multi_back != 0;
 
     // lane state
     bool has = false;
@@ -758,15 +762,13 @@ __global__ void __launch_bounds__(256, kOccBlocks(METHOD, OCC))
                 const uint32_t Llen = __shfl_sync(kFull, len_p, L);
                 const int Lp = __shfl_sync(kFull, p, L);
                 const int Ld = __shfl_sync(kFull, d, L);
-                const uint32_t Lr_lo = __shfl_sync(kFull, (uint32_t)r, L);
-                const uint32_t Lr_hi = __shfl_sync(kFull, (uint32_t)(r >> 32), L);
                 const PlanStep Lps = plan_s[Ld];
                 const uint32_t others = Lps.back & ~(1u << Lp);
                 const int colL = wbase + L;
                 const uint32_t Lsig = __shfl_sync(kFull, msig, L);
                 uint32_t total;
                 int32_t chosen;
-                coop_refine<MODE == kModeCount>(g, Ms, T, lane, colL, Llo, Llen, others, Lps, Lsig, Lr_lo, Lr_hi, sectors,
+                coop_refine<MODE == kModeCount>(g, Ms, T, lane, colL, Llo, Llen, others, Lps, Lsig, r, L, sectors,
                                                 total, chosen);
                 if (lane == L) {
                     cnt = total;
@@ -1771,7 +1773,8 @@ int sm_grid(int per_sm) {
 int occ_blocks(int method, int occ_variant) { return kOccBlocks(method, occ_variant); }
 
 int max_blocks_per_sm(int method, int mode, int threads, int ms_rows, size_t* smem_bytes) {
-    const size_t smem = (size_t)ms_rows * (size_t)threads * sizeof(uint32_t);  // rows: sample_smem_rows
+    (void)threads;  // every sampling kernel's rows are kSampleLanes words (rows: sample_smem_rows)
+    const size_t smem = (size_t)ms_rows * (size_t)kSampleLanes * sizeof(uint32_t);
     if (smem_bytes) *smem_bytes = smem;
     int blocks = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, select_kernel(method, mode), threads, smem) !=
@@ -1793,9 +1796,12 @@ cudaError_t launch_sample(int method, int mode, const DeviceGraph& g, const Plan
     // rows of the dynamic array (sample_smem_rows): sizing it by the query and the coop
     // threshold leaves the rest of the 256 KB L1/shared array to the L1 cache (spill slots,
     // hot CSR entries; measured: Alley is L1-capacity sensitive)
-    const size_t smem = (size_t)cfg.ms_rows * (size_t)cfg.threads * sizeof(uint32_t);
+    const size_t smem = (size_t)cfg.ms_rows * (size_t)kSampleLanes * sizeof(uint32_t);
     const uint32_t thr = (uint32_t)cfg.coop_threshold;
-    void* args[] = {(void*)&g,      (void*)&plan,  (void*)&first,   (void*)&count,     (void*)&seed,
+    Plan pl = plan;
+    pl.multi_back = 0;
+    for (int d = 1; d < pl.nq; ++d) pl.multi_back |= pl.step[d].nback >= 2 ? 1 : 0;
+    void* args[] = {(void*)&g,      (void*)&pl,  (void*)&first,   (void*)&count,     (void*)&seed,
                     (void*)&cfg.chunk, (void*)&thr, (void*)&cfg.sched, (void*)&cfg.refill_min, (void*)&d_queue,
                     (void*)&d_partials,
                     (void*)&d_records,

@@ -35,6 +35,7 @@ struct Plan {
     // comparison variants (GSWORD_OPT_VARIANT, readings A3/A5), applied per launch:
     int32_t wj_parent_first;  // A3: WanderJoin draws from the first backward position's list
     uint32_t pdup[kMaxQV];    // A5: Alley DupCheck after the draw (step[d].dup is then 0)
+    int32_t multi_back;       // some position d >= 1 has |B(d)| >= 2 (set per launch)
 };
 
 // Candidate filter of one query vertex (NEXT-1): label, degree, and the per-label
@@ -200,6 +201,9 @@ cudaError_t launch_build_bloom(const int64_t* d_row_ptr, const int32_t* col, int
 // Rows of blockDim.x words of the sampling kernel's dynamic shared memory: n_q rows of
 // matched vertices, plus for Alley the task-pool result row and ceil(coop/32) refine-mask
 // rows.
+// Row stride (words) of the sampling kernel's dynamic shared matrix: the largest CTA, a
+// compile-time constant so the row indexing holds no register; smaller CTAs leave rows' tails unused.
+constexpr int kSampleLanes = 256;
 inline int sample_smem_rows(int method, int nq, int coop_threshold) {
     return nq + (method == GSWORD_ALLEY ? 1 + (coop_threshold + 31) / 32 : 0);
 }
