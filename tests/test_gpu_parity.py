@@ -874,3 +874,35 @@ def test_estimate_instance_per_sample(ctx, G, c0, c1):
                     assert r["n"] == 64 and r["n_valid"] == int((ref["valid"][first:first + 64] != 0).sum())
                     assert r["sum"] == pytest.approx(float(np.sum(w)), rel=REL, abs=0.0)
                     assert r["sumsq"] == pytest.approx(float(np.sum(w * w)), rel=REL, abs=0.0)
+
+
+
+@pytest.mark.parametrize("occ", [0, 1, 2])
+def test_estimate_instance_per_sample_each_occupancy(ctx, G, c1, occ):
+    """Every occupancy variant of the estimate kernel, forced (the autotune picks variant 2 for C1
+    dense Alley since the register trims), checked sample by sample on the C1
+    dense and cyclic queries: one-id ranges bit-exact against the oracle's weight, 64-id windows
+    at 1e-12 with n_valid exact."""
+    g, qs = c1
+    ctx.load_graph_obj(g)
+    ctx.set_option(G.OPT_OCCUPANCY, occ)
+    try:
+        for q in qs[1:]:
+            ctx.load_query_obj(q)
+            for m in (0, 1):
+                y, ref = oracle.sample_range(g, q, m, 43, 0, 3200, records=True, threads=8)
+                y = np.asarray(y, dtype=np.float64)
+                valid = np.nonzero(ref["valid"])[0]
+                invalid = np.nonzero(ref["valid"] == 0)[0]
+                for i in list(valid[:24]) + list(invalid[:6]):
+                    r = ctx.estimate(m, 1, 43, first=int(i))
+                    assert r["n"] == 1 and r["n_valid"] == int(ref["valid"][i])
+                    assert r["sum"] == float(y[i]), (q.name, m, occ, int(i))
+                for first in range(0, 3200, 640):
+                    r = ctx.estimate(m, 64, 43, first=first)
+                    w = y[first:first + 64]
+                    assert r["n_valid"] == int((ref["valid"][first:first + 64] != 0).sum())
+                    assert r["sum"] == pytest.approx(float(np.sum(w)), rel=REL, abs=0.0)
+                    assert r["sumsq"] == pytest.approx(float(np.sum(w * w)), rel=REL, abs=0.0)
+    finally:
+        ctx.set_option(G.OPT_OCCUPANCY, -1)
